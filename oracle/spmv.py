@@ -1,0 +1,72 @@
+"""fp64 SpMV oracle.  TEST INFRASTRUCTURE ONLY.
+
+y*_i = sum_{k in row i} (double)val_k * (double)x[col_k], accumulated in CSR
+order — the plain definition of y = A x for the SHOC spmv-csr kernels the paper
+selects between ("spmv with scalar dot products on a CSR format matrix without
+padding", §4.2; scalar vs vector versions, §4.4).
+DySel changes only *which variant computes each row*, never *what* is computed
+(productive profiling, §2.2), so this is the oracle for every variant
+and every profiling mode.
+
+Pinned by tests/test_oracle_spmv.py: small-integer exactness, identity /
+diagonal closed forms, dense brute force, scipy.sparse.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+def _rows_of(row_ptr: np.ndarray) -> np.ndarray:
+    rp = np.asarray(row_ptr, np.int64)
+    return np.repeat(np.arange(rp.shape[0] - 1), np.diff(rp))
+
+
+def spmv(row_ptr, col, val, x) -> np.ndarray:
+    """y = A x in fp64, per-row sums accumulated in CSR order (np.add.at is
+    unbuffered and applies the products in index order)."""
+    rp = np.asarray(row_ptr, np.int64)
+    n = rp.shape[0] - 1
+    prod = np.asarray(val, np.float64) * np.asarray(x, np.float64)[np.asarray(col, np.int64)]
+    y = np.zeros(n, np.float64)
+    np.add.at(y, _rows_of(rp), prod)
+    return y
+
+
+def spmv_abs(row_ptr, col, val, x) -> np.ndarray:
+    """d_i = sum |val_k| * |x[col_k]| — the error denominator of c-1."""
+    return spmv(row_ptr, col, np.abs(np.asarray(val, np.float64)), np.abs(np.asarray(x, np.float64)))
+
+
+def spmv_rows(row_ptr, col, val, x, rows):
+    """(y*, d) for a sample of rows, each computed on its own (full-size parity)."""
+    rp = np.asarray(row_ptr, np.int64)
+    xs = np.asarray(x, np.float64)
+    y = np.empty(len(rows), np.float64)
+    d = np.empty(len(rows), np.float64)
+    for j, r in enumerate(rows):
+        b, e = rp[r], rp[r + 1]
+        v = np.asarray(val[b:e], np.float64)
+        xv = xs[np.asarray(col[b:e], np.int64)]
+        s = 0.0
+        a = 0.0
+        for p, q in zip(v, xv):   # CSR order, one term at a time
+            s += p * q
+            a += abs(p) * abs(q)
+        y[j] = s
+        d[j] = a
+    return y, d
+
+
+def rel_error(y_hat, y_star, denom) -> float:
+    """max_i |y_hat_i - y*_i| / d_i with 0/0 := 0 (c-1).  Non-finite values in
+    y_hat where y* is finite count as +inf error."""
+    y_hat = np.asarray(y_hat, np.float64)
+    diff = np.abs(y_hat - y_star)
+    denom = np.asarray(denom, np.float64)
+    with np.errstate(invalid="ignore", divide="ignore"):
+        e = np.where(diff == 0, 0.0, diff / denom)
+    e = np.where(np.isnan(e), np.inf, e)
+    return float(e.max()) if e.size else 0.0
+
+
+SPMV_TOL = 1e-5   # north_star: "max relative error 1e-5 of the fp64 oracle for fp32 SpMV"

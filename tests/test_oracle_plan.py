@@ -1,0 +1,152 @@
+"""Pins for oracle/slice_plan.py and oracle/selection.py (SURVEY c-5, c-7, c-8)."""
+import itertools
+import os
+
+import pytest
+
+from oracle import selection as S
+from oracle import slice_plan as P
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def test_fig3_worked_example():
+    # WA 3:2 -> A launches 2 WGs, B launches 3.
+    for line in open(os.path.join(GOLD, "fig3_worked_example.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        lhs, rhs = line.split("->")
+        wa_a, wa_b = map(int, lhs.split())
+        g, n_a, n_b = map(int, rhs.split())
+        p = P.plan((600,), [(wa_a,), (wa_b,)], 0.1, 148, 0, P.FULLY | P.FORCE_PROFILE)
+        assert p.g[0] == g
+        assert p.h == [n_a, n_b]
+
+
+def test_table1_counts():
+    rows = {}
+    for line in open(os.path.join(GOLD, "table1_modes.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        m, prod, extra, asy = line.split()
+        rows[m] = (prod, extra, asy)
+    for K in (2, 3, 4, 7):
+        wa = [(1,)] * K
+        for name, mode in (("fully", P.FULLY), ("hybrid", P.HYBRID), ("swap", P.SWAP)):
+            p = P.plan((10000,), wa, 0.05, 148, 0, mode | P.FORCE_PROFILE)
+            prod, extra = P.table1_counts(p)
+            e_prod = K if rows[name][0] == "K" else int(rows[name][0])
+            e_extra = {"0": 0, "K-1": K - 1, "K": K}[rows[name][1]]
+            assert prod == e_prod and extra == e_extra, (name, K)
+            if rows[name][2] == "no":
+                with pytest.raises(P.Unsupported):
+                    P.plan((10000,), wa, 0.05, 148, 0, mode | P.ASYNC)
+            else:
+                P.plan((10000,), wa, 0.05, 148, 0, mode | P.ASYNC)
+
+
+def test_fig6_defaults_are_fully_async():
+    vals = dict(l.split() for l in open(os.path.join(GOLD, "fig6_api_defaults.txt"))
+                if l.strip() and not l.startswith("#"))
+    assert vals == {"profiling": "true", "mode": "fully_async"}
+    default_mode = P.FULLY | P.ASYNC
+    p = P.plan((10000,), [(1,)] * 4, 0.02, 148, 0, default_mode)
+    assert p.active and p.mode == P.FULLY
+
+
+def test_small_workload_deactivation():
+    # < 128 work-groups => profiling off.
+    p = P.plan((127,), [(1,)] * 2, 1.0, 148, 0, P.FULLY)
+    assert not p.active
+    p = P.plan((128,), [(1,)] * 2, 0.5, 148, 0, P.FULLY)
+    assert p.active
+    p = P.plan((128,), [(1,)] * 2, 0.5, 148, 0, P.FULLY | P.NO_PROFILE)   # activation flag
+    assert not p.active and p.remainder == list(range(128))
+
+
+def test_survey_sgemm_d2m_numbers():
+    # SGEMM medium 1024x992x1056, unit = 32x32 tile: U = (33, 32); tilings
+    # 64x64 (2,2), 128x128 (4,4), 128x64 (N=64 -> 2, M=128 -> 4), 128x128.
+    U = (33, 32)
+    wa = [(2, 2), (4, 4), (2, 4), (4, 4)]
+    p = P.plan(U, wa, 0.02, 148, 0, P.FULLY)
+    assert p.g == (4, 4, 1) and p.G == (9, 8, 1) and p.Gn == 72
+    assert not p.active                                   # c = floor(0.36) = 0
+    p = P.plan(U, wa, 0.06, 148, 0, P.FULLY)
+    assert p.active and p.c == 1 and p.h == [4, 1, 2, 1]
+
+
+def test_sm_rounding_reading_a2():
+    # D4-like: G_n = 39063, K = 3, f = 0.02: c = 260 -> multiple of floor(148/3) = 49
+    p = P.plan((39063,), [(1,)] * 3, 0.02, 148, 0, P.HYBRID)
+    assert p.c == 245
+    p = P.plan((574,), [(1,)] * 4, 0.02, 148, 0, P.FULLY)     # D3: c = 2
+    assert p.c == 2
+
+
+@pytest.mark.parametrize("mode", [P.FULLY, P.FULLY | P.CONTIGUOUS, P.HYBRID, P.SWAP])
+def test_cover_invariant_exhaustive(mode):
+    for U in (1, 5, 17, 64):
+        for K in (2, 3, 4):
+            for wa in itertools.product((1, 2, 3, 4, 8), repeat=K):
+                for f in (0.1, 0.5, 1.0):
+                    p = P.plan((U,), [(w,) for w in wa], f, 148, 0, mode | P.FORCE_PROFILE)
+                    for sel in range(K):
+                        owner = P.productive_cover(p, sel)
+                        assert all(o >= 0 for o in owner)            # each granule exactly once
+                    if p.active:
+                        assert p.c * K <= max(1, f * p.Gn) + 1e-9 or p.c == 1
+                        if p.mode == P.FULLY:
+                            assert len(p.remainder) == p.Gn - K * p.c
+                        else:
+                            assert len(p.remainder) == p.Gn - p.c
+                        # per-variant CTA count = c * lcm / wa
+                        for v in range(K):
+                            assert p.profiled_ctas(v) == p.c * p.g[0] // wa[v]
+
+
+def test_ticket_order_covers_granules():
+    for mode in (P.FULLY, P.FULLY | P.CONTIGUOUS, P.HYBRID):
+        p = P.plan((50,), [(1,)] * 3, 0.3, 148, 1, mode | P.FORCE_PROFILE)
+        seen = {}
+        for t in range(P.n_tickets(p)):
+            j, v, role = P.ticket(p, t, mode, 1)
+            if role in (P.ROLE_PRODUCTIVE, P.ROLE_BATCH):
+                assert j not in seen
+                seen[j] = v
+        assert sorted(seen) == list(range(p.Gn))
+        # profiling tickets come first
+        roles = [P.ticket(p, t, mode, 1)[2] for t in range(P.n_tickets(p))]
+        first_batch = roles.index(P.ROLE_BATCH)
+        assert all(r == P.ROLE_BATCH for r in roles[first_batch:])
+        assert first_batch == 3 * p.c
+
+
+def test_granule_units_2d_edges():
+    p = P.plan((33, 32), [(2, 2), (4, 4)], 0.5, 148, 0, P.FULLY)
+    allu = [u for j in range(p.Gn) for u in P.granule_units(p, j, (33, 32))]
+    assert sorted(allu) == sorted((x, y, 0) for x in range(33) for y in range(32))
+    assert len(P.granule_units(p, 8, (33, 32))) == 4      # last column granule: 1 x 4 units
+
+
+def test_mode_resolution():
+    assert P.resolve_mode(P.AUTO, [0, 0]) == P.FULLY
+    assert P.resolve_mode(P.AUTO, [0, P.V_NONUNIFORM]) == P.HYBRID
+    assert P.resolve_mode(P.AUTO, [P.V_ATOMICS, P.V_NONUNIFORM]) == P.SWAP
+    with pytest.raises(P.Unsupported):
+        P.resolve_mode(P.AUTO | P.ASYNC, [P.V_ATOMICS])
+    assert P.resolve_mode(P.HYBRID | P.ASYNC, [P.V_ATOMICS]) == P.HYBRID   # user override wins
+
+
+def test_selection_packed_argmin():
+    assert S.select([5, 3, 3, 9]) == 1              # tie -> lowest id (A-8)
+    assert S.select([7]) == 0
+    assert S.pack(3, 2) < S.pack(3, 5) < S.pack(4, 0)
+    assert S.makespan(100, 350) == 250
+    assert S.cycles_per_unit(1000, 4) == 250
+    # known-cost variants: c_v ns per unit => argmin c_v
+    costs = [40, 10, 25, 10]
+    units = 7
+    assert S.select([c * units for c in costs]) == 1
+    assert S.exhaustive_best([3.0, 1.0, 1.0]) == 1
+    assert S.within(1.04, 1.0) and not S.within(1.06, 1.0)
