@@ -1,0 +1,406 @@
+"""DySel benchmark — one JSON line (driver contract).
+
+Step = one DySel SpMV launch over the D4 power-law matrix (10^7 rows, ~2*10^8
+nnz): profiling ON every step (single-shot, AUTO mode ->
+hybrid, async), i.e. format-prepared pool -> micro-profiling -> device-side
+selection -> remainder, all in libdysel.so.  `value` = algorithmic SpMV bytes
+(8 nnz + 4 (n+1) + 4 n_cols + 4 n) / step time, aggregated over ranks.
+Inputs (1.72 GB) are larger than L2, so no flush is needed between steps.
+
+Also reported in the same line: the exhaustive-oracle best pure variant T*
+ and DySel's overhead vs it, amortised overhead with the
+activation flag, and secondary workloads (D3 SpMV, D2m SGEMM).
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl dysel|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM = 6650.0
+
+
+def peaks():
+    try:
+        return json.load(open(PEAKS_PATH)), "measured"
+    except Exception:
+        return {"hbm_gbs": FALLBACK_HBM, "bf16_tflops": 1590.0}, "fallback"
+
+
+def spmv_bytes(n_rows, n_cols, nnz):
+    return 8 * nnz + 4 * (n_rows + 1) + 4 * n_cols + 4 * n_rows
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled DURING the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([c.strip() for c in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.1)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------- CPU oracle
+def cpu_oracle_spmv(A, x, reps=3):
+    """The oracle as it stands (plain C fp64 loops, OpenMP over all cores)."""
+    from oracle import ref_c
+    cores = len(os.sched_getaffinity(0))
+    ref_c.spmv_f64(A.row_ptr, A.col, A.val, x, cores)    # warm
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        ref_c.spmv_f64(A.row_ptr, A.col, A.val, x, cores)
+        ts.append(time.perf_counter() - t0)
+    return float(np.median(ts)), cores
+
+
+# ------------------------------------------------------------- workloads
+def make_d4(n):
+    from workloads import d4_powerlaw, uniform_f32
+    A = d4_powerlaw(n=n)
+    x = uniform_f32(10010, A.n_cols)
+    return A, x
+
+
+def reference_arm(args, world, rank):
+    """--impl reference: the oracle timed on the host cores, same metric/unit."""
+    if rank != 0:
+        return
+    A, x = make_d4(args.rows)
+    nbytes = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
+    from oracle import ref_c
+    cores = len(os.sched_getaffinity(0))
+    for _ in range(args.warmup):
+        ref_c.spmv_f64(A.row_ptr, A.col, A.val, x, cores)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        ref_c.spmv_f64(A.row_ptr, A.col, A.val, x, cores)
+        ts.append(time.perf_counter() - t0)
+    T = float(np.mean(ts))
+    v = nbytes / T / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(T * 1e3, 3),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": config(A, world),
+            "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
+                             "sample": f"full D4 matrix ({A.nnz} nnz), one fp64 SpMV per step"},
+            "e2e": {"value": round(v, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+METRIC = "DySel SpMV GB/s (power-law 1e7 rows, profiling on every call) + overhead % vs best-variant oracle"
+
+
+def config(A, world):
+    return {"workload": "D4 power-law SpMV: 10^7 rows, p(L)~L^-1.761 on [1,16384], uniform cols, fp32 CSR",
+            "n_rows": int(A.n_rows), "nnz": int(A.nnz), "parallelism": f"row-shard{world}",
+            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": "AUTO|ASYNC (hybrid), f=0.02"}
+
+
+# ------------------------------------------------------------------ timing
+def time_events(fn, reps, stream):
+    import torch
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+    torch.cuda.synchronize()
+    for a, b in evs:
+        a.record(stream)
+        fn()
+        b.record(stream)
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) * 1e-3 for a, b in evs]
+
+
+def dysel_arm(args, world, rank, local_rank):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    ctx = D.Context(local_rank)
+    if world > 1:
+        uid = [D.comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        ctx.comm_init(rank, world, uid[0])
+    A, x = make_d4(args.rows)
+    nbytes_total = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
+    bounds = D.partition_rows(A.row_ptr, world)
+    r0, r1 = bounds[rank], bounds[rank + 1]
+    rp_local = (A.row_ptr[r0:r1 + 1].astype(np.int64) - A.row_ptr[r0]).astype(np.int32)
+    lo, hi = int(A.row_ptr[r0]), int(A.row_ptr[r1])
+    rp = torch.from_numpy(rp_local).to(dev)
+    col = torch.from_numpy(A.col[lo:hi]).to(dev)
+    val = torch.from_numpy(A.val[lo:hi]).to(dev)
+    xd = torch.from_numpy(x).to(dev)
+    y = torch.empty(A.n_rows, device=dev)
+    stream = torch.cuda.current_stream()
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_CSR_VECTOR)
+    mode = D.AUTO | D.ASYNC
+    f = args.f
+
+    def step():
+        if world > 1:
+            ctx.spmv_sharded(plan, bounds, xd, y, f=f, mode=mode)
+        else:
+            ctx.spmv(plan, xd, y[r0:r1], f=f, mode=mode)
+
+    # ---- exhaustive oracle: every pure variant, full grid
+    yl = y[r0:r1]
+    T_v = {}
+    for v in plan.variant_ids:
+        for _ in range(2):
+            ctx.spmv_variant(plan, v, xd, yl)
+        ts = time_events(lambda: ctx.spmv_variant(plan, v, xd, yl), args.oracle_reps, stream)
+        T_v[D.SPMV_NAMES[v]] = float(np.median(ts))
+    best_name = min(T_v, key=T_v.get)
+    T_star = T_v[best_name]
+    # ---- warmup, then K timed steps (barrier + sync on both sides)
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches0 = ctx.kernel_launches()
+    with ClockSampler(local_rank) as clk:
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        torch.cuda.synchronize()
+        t_all0 = torch.cuda.Event(enable_timing=True)
+        t_all1 = torch.cuda.Event(enable_timing=True)
+        t_all0.record(stream)
+        for a, b in ev:
+            a.record(stream)
+            step()
+            b.record(stream)
+        t_all1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = ctx.kernel_launches() - launches0
+    per_step = [a.elapsed_time(b) * 1e-3 for a, b in ev]
+    T_total = t_all0.elapsed_time(t_all1) * 1e-3
+    if world > 1:
+        t = torch.tensor([T_total], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        T_total = float(t.item())
+    T_step = T_total / args.steps
+    value = nbytes_total / T_step / 1e9
+    # report of one extra (untimed) launch: selection, scores
+    rep = ctx.spmv(plan, xd, yl, f=f, mode=mode, report=True)
+    # ---- amortised: profile once, then the activation flag
+    I = args.amortize
+    def amort():
+        ctx.spmv(plan, xd, yl, f=f, mode=mode)
+        for _ in range(I - 1):
+            ctx.spmv(plan, xd, yl, mode=D.NO_PROFILE)
+    ta = float(np.median(time_events(amort, 3, stream))) / I
+    # ---- e2e through the public API with host buffers: x H2D, y D2H per step
+    xh = torch.from_numpy(x).pin_memory()
+    yh = torch.empty(r1 - r0, dtype=torch.float32).pin_memory()
+    def e2e_step():
+        xd.copy_(xh, non_blocking=True)
+        step()
+        yh.copy_(yl, non_blocking=True)
+    for _ in range(2):
+        e2e_step()
+    te = time_events(e2e_step, args.steps, stream)
+    T_e2e = float(np.mean(te))
+    # ---- roofline for the dominant kernel (the persistent dispatcher)
+    pk, src = peaks()
+    kern_bytes = spmv_bytes(r1 - r0, A.n_cols, hi - lo)
+    k_time = float(np.mean(per_step)) if world == 1 else float(np.mean(per_step))
+    achieved = kern_bytes / k_time / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic_d4.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    # ---- secondary workloads (1 GPU, rank 0): D3 SpMV and D2m SGEMM
+    secondary = {}
+    if rank == 0 and not args.no_secondary:
+        secondary = secondary_workloads(ctx, D, args, stream)
+    # ---- CPU baseline: the oracle as it stands, on the host cores (rank 0, N=1)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        Tc, cores = cpu_oracle_spmv(A, x, reps=args.cpu_reps)
+        cpu = {"value": round(nbytes_total / Tc / 1e9, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
+               "sample": f"full D4 matrix ({A.nnz} nnz), fp64 CSR SpMV in plain C/OpenMP, median of "
+                         f"{args.cpu_reps} passes"}
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(T_step * 1e3, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": config(A, world),
+            "overhead_pct_vs_best_variant": round((T_step - T_star) / T_star * 100, 3) if world == 1 else None,
+            "best_variant_oracle": {"variant": best_name, "ms": round(T_star * 1e3, 4),
+                                    "gbs": round(nbytes_total / T_star / 1e9, 2),
+                                    "all_ms": {k: round(v * 1e3, 4) for k, v in T_v.items()}},
+            "selected": rep["selected_name"], "selection_matches_oracle": rep["selected_name"] == best_name,
+            "mode_used": rep["mode_used"], "profiled_units_per_variant": rep["c"],
+            "amortized_overhead_pct": round((ta - T_star) / T_star * 100, 3) if world == 1 else None,
+            "amortized_iters": I,
+            "e2e": {"value": round(nbytes_total / T_e2e / 1e9, 3), "unit": "GB/s",
+                    "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int((r1 - r0) * 4),
+                    "ms_per_step": round(T_e2e * 1e3, 4)},
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": pk["hbm_gbs"], "unit": "GB/s",
+                         "frac": round(achieved / pk["hbm_gbs"], 4), "traffic": traffic,
+                         "kernel": "dysel::spmv_persistent_kernel", "peak_source": src},
+            "gpu_launches": int(launches), "clocks": clk.summary(),
+            "cpu_baseline": cpu, "secondary": secondary,
+        }
+        print(json.dumps(line), flush=True)
+    plan.destroy()
+    ctx.close()
+
+
+def secondary_workloads(ctx, D, args, stream):
+    import torch
+    from workloads import d3_fem, sgemm_inputs, uniform_f32
+    out = {}
+    # D3: Dubcova3-shaped FEM SpMV (30.9 MB: L2-resident when warm)
+    A = d3_fem()
+    x = torch.from_numpy(uniform_f32(384, A.n_cols)).cuda()
+    rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_CSR_VECTOR)
+    y = torch.empty(A.n_rows, device="cuda")
+    nb = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    res = {}
+    for v in plan.variant_ids:
+        ts = []
+        for _ in range(20):
+            flush.zero_()
+            ts += time_events(lambda: ctx.spmv_variant(plan, v, x, y), 1, stream)
+        res[D.SPMV_NAMES[v]] = float(np.median(ts))
+    best = min(res, key=res.get)
+    ts = []
+    for _ in range(20):
+        flush.zero_()
+        ts += time_events(lambda: ctx.spmv(plan, x, y, f=0.02, mode=D.AUTO | D.ASYNC), 1, stream)
+    td = float(np.median(ts))
+    ta = float(np.median(time_events(lambda: ctx.spmv(plan, x, y, mode=D.NO_PROFILE), 50, stream)))
+    rep = ctx.spmv(plan, x, y, f=0.02, mode=D.AUTO | D.ASYNC, report=True)
+    out["d3_spmv"] = {"cold_l2": True, "best_variant": best, "best_us": round(res[best] * 1e6, 2),
+                      "best_gbs": round(nb / res[best] / 1e9, 1), "dysel_us": round(td * 1e6, 2),
+                      "dysel_gbs": round(nb / td / 1e9, 1), "overhead_pct": round((td / res[best] - 1) * 100, 2),
+                      "selected": rep["selected_name"], "profiled": rep["profiled"],
+                      "warm_no_profile_us": round(ta * 1e6, 2),
+                      "all_us": {k: round(v * 1e6, 2) for k, v in res.items()}}
+    plan.destroy()
+    # D2m: Parboil-medium SGEMM 1024 x 992 x 1056
+    M, K, N = 1024, 992, 1056
+    Ah, Bh, _ = sgemm_inputs(M, K, N)
+    Ad, Bd = torch.from_numpy(Ah).cuda(), torch.from_numpy(Bh).cuda()
+    C = torch.empty((M, N), device="cuda")
+    flops = 2.0 * M * N * K
+    tv = {}
+    for v in range(4):
+        for _ in range(3):
+            ctx.sgemm_variant(v, Ad, Bd, C)
+        tv[D.SGEMM_NAMES[v]] = float(np.median(time_events(lambda: ctx.sgemm_variant(v, Ad, Bd, C), 30, stream)))
+    bestg = min(tv, key=tv.get)
+    f_sg = 0.06
+    for _ in range(3):
+        ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY)
+    tdg = float(np.median(time_events(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY), 30, stream)))
+    repg = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY, report=True)
+    I = 100
+    def amort():
+        ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY)
+        for _ in range(I - 1):
+            ctx.sgemm(Ad, Bd, C, mode=D.NO_PROFILE)
+    tam = float(np.median(time_events(amort, 3, stream))) / I
+    out["d2m_sgemm"] = {"best_variant": bestg, "best_us": round(tv[bestg] * 1e6, 2),
+                        "best_tflops": round(flops / tv[bestg] / 1e12, 2),
+                        "dysel_single_shot_us": round(tdg * 1e6, 2),
+                        "single_shot_overhead_pct": round((tdg / tv[bestg] - 1) * 100, 2),
+                        "amortized_overhead_pct": round((tam / tv[bestg] - 1) * 100, 2),
+                        "selected": repg["selected_name"], "f": f_sg,
+                        "all_us": {k: round(v * 1e6, 2) for k, v in tv.items()}}
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="dysel", choices=["dysel", "reference"])
+    ap.add_argument("--rows", type=int, default=10_000_000)
+    ap.add_argument("--f", type=float, default=0.02)
+    ap.add_argument("--oracle-reps", type=int, default=15)
+    ap.add_argument("--amortize", type=int, default=20)
+    ap.add_argument("--cpu-reps", type=int, default=5)
+    ap.add_argument("--no-secondary", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        reference_arm(args, world, rank)
+        return
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl")
+    dysel_arm(args, world, rank, local_rank)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,342 @@
+/*
+ * dysel.h — C ABI of libdysel.so, a B200-native (sm_100a) implementation of
+ * DySel's data-parallel hot path: micro-profiled dynamic selection among
+ * candidate kernel variants (Chang, Kim, Hwu, ASPLOS '16).
+ *
+ * Citations are PAPER.md line numbers (P:L<a>-<b>) with section / figure /
+ * table.  Readings of ambiguous passages are numbered A-<n> and listed in
+ * DESIGN.md §Readings.
+ *
+ * The method (§2.1, §2.2): K variants of one
+ * data-parallel kernel each run on a small slice of the real work-groups
+ * ("micro-profiling"), each slice writes its part of the final output
+ * ("productive profiling"), the slices are timed on the device
+ * (§3.3, Fig. 7), the fastest variant is selected and the rest of
+ * the NDRange is launched with it (§2.4).
+ *
+ * Conventions for every call below
+ *   - Pointers named d_* are DEVICE pointers, caller-owned (normally torch
+ *     tensors).  The library never frees them and never keeps them after the
+ *     call returns, except the CSR arrays a dysel_spmv_plan refers to (the
+ *     caller must keep them alive until dysel_spmv_plan_destroy).
+ *   - `stream` is a cudaStream_t passed as void*; NULL = the legacy default
+ *     stream.  All device work is stream-ordered on it.  Profiling streams fork
+ *     from and join back to it through events.  Device-path calls never block
+ *     the host; DYSEL_HOST_ORCH calls block inside the call (as the paper's
+ *     cudaDeviceSynchronize did).
+ *   - Every call returns a dysel_status and never aborts or throws; CUDA /
+ *     NCCL failures return DYSEL_ERR_CUDA / DYSEL_ERR_NCCL with the message in
+ *     dysel_last_error(ctx).
+ *   - A dysel_ctx is bound to one device and is NOT thread-safe; use one ctx
+ *     per host thread, and do not run two launches of one ctx concurrently on
+ *     different streams (they share the ctx's timer / ticket state).
+ */
+#ifndef DYSEL_H_
+#define DYSEL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ------------------------------------------------------------------ status */
+typedef enum {
+  DYSEL_OK = 0,
+  DYSEL_ERR_INVALID = 1,     /* NULL pointer, bad size, f not in [0,1], unknown sig, n not in [1,16], wa = 0 */
+  DYSEL_ERR_UNSUPPORTED = 2, /* SWAP|ASYNC (Table 1), ELL over the cap (A-15), ... */
+  DYSEL_ERR_NOMEM = 3,
+  DYSEL_ERR_CUDA = 4,
+  DYSEL_ERR_NOT_FOUND = 5,   /* no cached selection for the key */
+  DYSEL_ERR_NCCL = 6
+} dysel_status;
+
+const char *dysel_status_str(dysel_status s);
+
+/* ------------------------------------------------------------------- modes
+ * Low two bits: productive-profiling mode (§2.2, Table 1).
+ *   FULLY  — each variant runs a disjoint slice and writes the final output.
+ *   HYBRID — all variants run the same slice; only default_variant writes the
+ *            output, the others write sandboxes (≤ K-1 extra, A-4).
+ *   SWAP   — each variant writes a private full output; the winner's is
+ *            swapped in; synchronous only.
+ *   AUTO   — resolved from variant flags: any DYSEL_V_ATOMICS -> SWAP, any
+ *            DYSEL_V_NONUNIFORM -> HYBRID, else FULLY (replaces the compiler's
+ *            side-effect / uniform-workload analyses, §3.4; A-10,
+ *            A-11, A-13).  Explicit bits are a programmer override
+ *            (P:L974-975).
+ * Orchestration (§2.4): SYNC waits for all profiling slices before
+ * the remainder; ASYNC starts the remainder at once with the best variant so
+ * far ("eager execution"), default_variant first.
+ * Default = DYSEL_FULLY | DYSEL_ASYNC ("mode=fully_async", Fig. 6b).
+ */
+#define DYSEL_FULLY 0u
+#define DYSEL_HYBRID 1u
+#define DYSEL_SWAP 2u
+#define DYSEL_AUTO 3u
+#define DYSEL_SYNC 0u
+#define DYSEL_ASYNC 4u
+#define DYSEL_NO_PROFILE 8u     /* profiling activation flag = false: cached or default variant, plain full grid */
+#define DYSEL_HOST_ORCH 16u     /* paper-faithful host orchestration: streams + host sync / polling */
+#define DYSEL_FORCE_PROFILE 32u /* ignore the small-workload deactivation (< 128 CTAs); ablation */
+#define DYSEL_CONTIGUOUS 64u    /* fully mode: contiguous per-variant slices instead of interleaved granules (A-24) */
+#define DYSEL_SCORE_CYCLES 128u /* score = sum of per-CTA clock64 cycles / units instead of %globaltimer makespan (A-6) */
+#define DYSEL_DEFAULT_MODE (DYSEL_FULLY | DYSEL_ASYNC)
+
+/* variant flags (replace the compiler analyses, A-10/A-11) */
+#define DYSEL_V_ATOMICS 1u     /* global atomics / overlapping outputs -> SWAP */
+#define DYSEL_V_NONUNIFORM 2u  /* data-dependent loop bounds -> HYBRID */
+
+/* roles of a slice — the paper's three extended copies of each variant
+ * (profiling / batch / eager, §3.3) folded into one parameter */
+enum {
+  DYSEL_ROLE_PRODUCTIVE = 0, /* profiling copy writing the real output */
+  DYSEL_ROLE_SANDBOX = 1,    /* profiling copy writing a sandbox (hybrid) */
+  DYSEL_ROLE_BATCH = 2,      /* non-profiling batch copy (remainder, or whole grid when profiling is off) */
+  DYSEL_ROLE_PRIVATE = 3,    /* profiling copy writing a private output (swap) */
+  DYSEL_ROLE_EAGER = 4       /* async eager chunk of the best-so-far variant */
+};
+
+#define DYSEL_MAX_VARIANTS 16
+
+/* ------------------------------------------------------------------ context */
+typedef struct dysel_ctx dysel_ctx;
+
+/* Create a context on CUDA device `cuda_device` (calls cudaSetDevice).  Owns
+ * its scratch (timer slots, selection words, tickets, sandboxes), streams and
+ * events.  Queries #SM (cudaDevAttrMultiProcessorCount) and calibrates the
+ * %globaltimer resolution (A-6). */
+dysel_status dysel_create(int cuda_device, dysel_ctx **out);
+void dysel_destroy(dysel_ctx *ctx);
+const char *dysel_last_error(const dysel_ctx *ctx);
+/* SM count, measured %globaltimer tick (ns) and L2 size of the ctx's device. */
+dysel_status dysel_device_info(const dysel_ctx *ctx, int *n_sm, uint64_t *globaltimer_tick_ns,
+                               uint64_t *l2_bytes);
+
+/* ------------------------------------------------------------ device timing
+ * One per variant, in device memory.  Written by the profiling copies
+ * (Fig. 7b): earliest CTA start / latest CTA end (%globaltimer,
+ * ns), profiled units, sum over CTAs of (end - start) in clock64 cycles. */
+typedef struct {
+  uint64_t t_start_min;
+  uint64_t t_end_max;
+  uint64_t units;
+  uint64_t cycles;
+} dysel_timer_slot;
+
+/* What one launch of a variant must cover: `granule_count` granules starting
+ * at linear granule `granule_begin`, every `granule_stride`-th (interleaved
+ * fully mode, A-24).  A granule is g[0]*g[1]*g[2] units (the LCM of the
+ * variants' work-assignment factors); granules are numbered x
+ * fastest over G[0] x G[1] x G[2]; edge granules may be partial (clip to U).
+ * A variant with wa units per CTA launches granule_count * prod(g/wa) CTAs. */
+typedef struct {
+  uint64_t granule_begin;
+  uint64_t granule_count;
+  uint64_t granule_stride;
+  uint32_t g[3];
+  uint32_t G[3];
+  uint64_t U[3];
+  int32_t role;
+  int32_t variant;
+  /* device-side profiling bookkeeping; NULL when the copy is untimed */
+  dysel_timer_slot *timer;   /* this variant's slot */
+  uint32_t *ctas_done;       /* per-variant count of finished profiling CTAs */
+  uint32_t ctas_total;       /* profiling CTAs of this variant */
+  uint64_t *best;            /* packed (score<<8 | v), atomicMin'd when a variant completes */
+  uint32_t *variants_done;   /* completed variants; the last one copies *best into *sel */
+  uint32_t n_variants;
+  uint32_t score_cycles;     /* 1 => score by cycles/units */
+  uint64_t *sel;             /* final packed selection (~0 until profiling completes) */
+  /* gated batch: when non-NULL the copy runs only if (*gate & 0xff) == variant */
+  const uint64_t *gate;
+} dysel_slice;
+
+/* A variant = a host function that launches its kernel(s) over a slice on
+ * `stream` (a cudaStream_t).  args are the dysel_launch args with sandbox /
+ * private-output substitutions applied; `user` is dysel_variant.user.  Every
+ * CTA of a timed launch (s->timer != NULL) must call dysel_prof_begin/end
+ * exactly once, also CTAs whose tile is out of range (units = 0).
+ * Device-side helpers for slice mapping and timing are in dysel_device.cuh. */
+typedef dysel_status (*dysel_variant_fn)(const dysel_slice *s, void *const *args, void *stream, void *user);
+
+typedef struct {
+  const char *name;
+  dysel_variant_fn fn;
+  uint32_t wa[3];            /* work-assignment factor: units per CTA per dim */
+  const int *sandbox_args;   /* indices into args[] of output pointers to redirect */
+  int n_sandbox_args;
+  uint32_t flags;            /* DYSEL_V_* */
+  void *user;                /* passed to fn */
+} dysel_variant;
+
+/* Register K = n variants under kernel_sig (DySelAddKernel, Fig. 6a
+ * P:L761-767).  default_variant is the "initial version" async mode starts
+ * with (A-5) and the productive variant in hybrid mode (A-4).
+ * Re-registering a sig replaces it and clears its cached selection. */
+dysel_status dysel_register_variants(dysel_ctx *ctx, const char *kernel_sig, const dysel_variant *v,
+                                     int n, int default_variant);
+
+/* ------------------------------------------------------------------ report */
+typedef struct {
+  uint64_t granule_begin, granule_count, granule_stride;
+  int32_t variant, role;
+} dysel_slice_rec;
+
+typedef struct {
+  int32_t mode_used;        /* resolved FULLY/HYBRID/SWAP | ASYNC bit */
+  int32_t profiled;         /* 1 if profiling ran */
+  int32_t selected;         /* variant used for the remainder (final selection) */
+  int32_t n_variants;
+  uint64_t c;               /* granules per profiling slice */
+  uint64_t n_granules;      /* G_n */
+  uint64_t score[DYSEL_MAX_VARIANTS];   /* ns (makespan) or cycles/unit */
+  uint64_t makespan_ns[DYSEL_MAX_VARIANTS];
+  uint64_t units[DYSEL_MAX_VARIANTS];
+  uint64_t cycles[DYSEL_MAX_VARIANTS];
+  uint64_t eager_units;     /* remainder units run before the final selection (async) */
+  uint64_t host_ns;         /* host time inside the call */
+  dysel_slice_rec *slices;  /* optional caller array */
+  int32_t slices_cap, n_slices;
+  uint8_t *unit_variant;    /* optional caller HOST array, one byte per granule: variant that
+                               productively computed it (debug / c-6 tests; costs a D2H copy + sync) */
+  uint64_t unit_variant_cap;
+} dysel_report;
+
+/* Launch kernel_sig over an NDRange of ndrange_units[3] units
+ * (DySelLaunchKernel, Fig. 6b).  profile_fraction f in [0,1]: each
+ * variant profiles c = floor(f * G_n / K) granules (A-1, rounding A-2);
+ * profiling is off when c = 0, when the default variant's full grid has < 128
+ * CTAs (A-3), with DYSEL_NO_PROFILE (activation flag, P:L796-804:
+ * the cached selection or the default runs the whole grid), or for K = 1.
+ * args[0..n_args) are passed to the variant functions (device pointers or
+ * pointers to host scalars; the library only replaces sandbox entries).
+ * sandbox_arg_bytes[i] gives the size of args[sandbox_args[i]] (hybrid
+ * sandboxes / swap private outputs are allocated in the ctx).  On success the
+ * selection is cached under kernel_sig (A-22).  rep may be NULL. */
+dysel_status dysel_launch(dysel_ctx *ctx, const char *kernel_sig, const uint64_t ndrange_units[3],
+                          float profile_fraction, uint32_t mode, void *const *args, int n_args,
+                          const size_t *sandbox_arg_bytes, void *stream, dysel_report *rep);
+
+/* Selection cache (profiling activation flag; key A-22). */
+dysel_status dysel_get_selection(dysel_ctx *ctx, const char *key, int *variant);
+dysel_status dysel_set_selection(dysel_ctx *ctx, const char *key, int variant);
+dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key); /* NULL key: all */
+
+/* ------------------------------------------------------------------- SpMV
+ * y = A x (overwrite), fp32 CSR input (SHOC spmv-csr / Parboil spmv-jds,
+ * P:L1128-1131).  Unit = 256 consecutive original rows.
+ * Built-in variants (ids): 0 CSR-scalar (thread per row), 1 CSR-vector (warp
+ * per row), 2 ELL (column-major, padded), 3 block-local JDS (A-14). */
+enum { DYSEL_SPMV_CSR_SCALAR = 0, DYSEL_SPMV_CSR_VECTOR = 1, DYSEL_SPMV_ELL = 2, DYSEL_SPMV_JDS = 3,
+       DYSEL_SPMV_NVARIANTS = 4 };
+#define DYSEL_FMT_ELL 1u
+#define DYSEL_FMT_JDS 2u
+
+typedef struct dysel_spmv_plan dysel_spmv_plan;
+
+typedef struct {
+  int64_t n_rows, n_cols, nnz;
+  int32_t n_variants;            /* variants in the pool (ELL dropped when inapplicable, A-15) */
+  int32_t variant_ids[DYSEL_SPMV_NVARIANTS]; /* pool index -> DYSEL_SPMV_* id */
+  int32_t ell_width;             /* W (0 if no ELL) */
+  int32_t uniform;               /* max row length <= 2 * mean (A-13) */
+  int32_t max_row_len;
+  uint64_t prep_ns;              /* device time of format preparation (a-1) */
+  uint64_t ell_bytes, jds_bytes; /* extra device memory held by the plan */
+} dysel_spmv_plan_info;
+
+/* Build the variant pool for one CSR matrix: CSR -> ELL and CSR -> block JDS
+ * on the device (a-1).  d_row_ptr int32 [n_rows+1], d_col int32
+ * [nnz] (sorted or not), d_val fp32 [nnz]; nnz < 2^31.  formats_mask selects
+ * which extra formats to build (DYSEL_FMT_*); ELL is skipped (and absent from
+ * the pool) when W * n_rows > 4 * nnz.  default_variant is a DYSEL_SPMV_* id
+ * (must be in the pool).  Blocks on `stream` (reads back sizes). */
+dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, int64_t nnz,
+                                const int32_t *d_row_ptr, const int32_t *d_col, const float *d_val,
+                                uint32_t formats_mask, int default_variant, void *stream,
+                                dysel_spmv_plan **out);
+dysel_status dysel_spmv_plan_get_info(const dysel_spmv_plan *plan, dysel_spmv_plan_info *info);
+/* Test / debug: copy one of the plan's format arrays (layouts in DESIGN.md
+ * §Data layout) to HOST memory, synchronously.  which: 0 ell_col (int32),
+ * 1 ell_val (f32), 2 perm (int32), 3 jds_len (int32), 4 blk_off (int64),
+ * 5 jd_off (int64), 6 jd_ptr (int32), 7 jds_col (int32), 8 jds_val (f32).
+ * *bytes: in = capacity of dst, out = size of the array; dst NULL = query.
+ * DYSEL_ERR_NOT_FOUND if the plan has no such format. */
+dysel_status dysel_spmv_plan_copy_array(const dysel_spmv_plan *plan, int which, void *dst, size_t *bytes);
+void dysel_spmv_plan_destroy(dysel_spmv_plan *plan);
+
+/* One DySel SpMV launch: y = A x.  d_x fp32 [n_cols], d_y fp32 [n_rows].
+ * Device path (default): ONE persistent launch; tickets claim granules, the
+ * profiling tickets first; the last profiling CTA publishes the selection on
+ * the device; sync mode spins on it, async mode reads the best so far
+ * (SURVEY §8a device protocol).  With DYSEL_HOST_ORCH: one kernel per variant
+ * on forked streams, host reads the selection, then the remainder kernel
+ * (paper-faithful).  Mode AUTO uses the plan's uniformity flag. */
+dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,
+                        float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+
+/* One full-grid run of pool variant `variant_id` (a DYSEL_SPMV_* id) with no
+ * profiling: the "single pure version" the exhaustive oracle times
+ * and what DYSEL_NO_PROFILE runs. */
+dysel_status dysel_spmv_variant(dysel_ctx *ctx, dysel_spmv_plan *plan, int variant_id, const float *d_x,
+                                float *d_y, void *stream);
+
+/* ------------------------------------------------------------------ SGEMM
+ * C = alpha * A B + beta * C, fp32, row-major, no transposes (Parboil sgemm,
+ * P:L1286-1294, L1427; A-17).  Unit = one 32x32 tile of C.  Built-in variants:
+ * 0 S64 (SIMT FFMA 64x64), 1 S128 (SIMT 128x128), 2 T128x64 and 3 T128x128
+ * (tcgen05.mma kind::tf32, 3xTF32 split in shared memory, TMEM accumulator).
+ * lda >= K, ldb >= N, ldc >= N; M, N, K >= 0.  M*N = 0: no-op; K = 0: C = beta C. */
+enum { DYSEL_SGEMM_S64 = 0, DYSEL_SGEMM_S128 = 1, DYSEL_SGEMM_T128x64 = 2, DYSEL_SGEMM_T128x128 = 3,
+       DYSEL_SGEMM_NVARIANTS = 4 };
+dysel_status dysel_sgemm(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A, int lda,
+                         const float *d_B, int ldb, float beta, float *d_C, int ldc,
+                         float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+/* Full-grid run of one SGEMM variant (exhaustive oracle timing). */
+dysel_status dysel_sgemm_variant(dysel_ctx *ctx, int variant_id, int M, int N, int K, float alpha,
+                                 const float *d_A, int lda, const float *d_B, int ldb, float beta,
+                                 float *d_C, int ldc, void *stream);
+
+/* --------------------------------------------------------------- multi-GPU
+ * Row-sharded SpMV / M-sharded SGEMM over NCCL (the paper is
+ * single-GPU).  nccl_unique_id points to the 128-byte
+ * ncclUniqueId rank 0 created (dysel_comm_unique_id) and the caller broadcast
+ * (e.g. over torch.distributed). */
+dysel_status dysel_comm_unique_id(void *out_128_bytes);
+dysel_status dysel_comm_init(dysel_ctx *ctx, const void *nccl_unique_id, int rank, int world);
+/* nnz-balanced row partition: bounds[g] = smallest r with row_ptr[r] >= g*nnz/world, snapped down
+ * to a multiple of 256 rows, bounds[0] = 0, bounds[world] = n_rows.  h_row_ptr is HOST memory. */
+dysel_status dysel_partition_rows(const int32_t *h_row_ptr, int64_t n_rows, int world, int64_t *bounds);
+/* y (full length, every rank) = A x where this rank's plan holds rows
+ * [bounds[rank], bounds[rank+1]) with a rebased row_ptr; x full length on
+ * every rank.  Local DySel launch into d_y + bounds[rank], then an allgatherv of
+ * y (grouped ncclBroadcast per root) in place. */
+dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local_plan, const int64_t *bounds,
+                                const float *d_x, float *d_y, float profile_fraction, uint32_t mode,
+                                void *stream, dysel_report *rep);
+/* Broadcast n floats from `root` in place (x or B distribution). */
+dysel_status dysel_comm_broadcast(dysel_ctx *ctx, float *d_buf, size_t n, int root, void *stream);
+/* C rows [m0, m1) computed locally with DySel (B replicated), then C allgathered. */
+dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A,
+                                 int lda, const float *d_B, int ldb, float beta, float *d_C, int ldc,
+                                 float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+
+/* ------------------------------------------------------------------- debug */
+/* Number of dysel kernels launched by this ctx so far (bench.py's gpu_launches). */
+uint64_t dysel_kernel_launches(const dysel_ctx *ctx);
+/* Calibration microbenchmark (c-9): minimum non-zero %globaltimer delta over
+ * `samples` reads and the clock64 rate (cycles per ns) over a `spin_ns` spin. */
+dysel_status dysel_timer_calibrate(dysel_ctx *ctx, uint64_t samples, uint64_t spin_ns,
+                                   uint64_t *tick_ns, double *cycles_per_ns);
+/* Known-cost test variants (c-8): registers sig with n variants whose CTAs
+ * spin cost_ns[v] per unit (wa = 1) and write out[u] = v+1 for each unit u
+ * (args[0] = uint32_t* out).  Used to check selection end to end. */
+dysel_status dysel_register_spin_variants(dysel_ctx *ctx, const char *sig, const uint32_t *cost_ns, int n,
+                                          int default_variant);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DYSEL_H_ */

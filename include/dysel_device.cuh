@@ -1,0 +1,146 @@
+/*
+ * dysel_device.cuh — device-side helpers for DySel variant kernels (sm_100a).
+ *
+ * 1. Slice mapping: the paper's profiling / eager copies shift the block index
+ *    so a variant processes "a particular part of the workload"; the batch
+ *    copy skips blocks already profiled (§3.3).  Here a launch
+ *    covers exactly the granules of its dysel_slice (reading A-10: launch the
+ *    remainder grid with an offset instead of suppressing blocks), so
+ *    dysel_cta_origin() maps blockIdx -> the first unit of the CTA's tile.
+ *
+ * 2. Timing (Fig. 7b): the paper's thread 0 reads the 32-bit
+ *    per-SM %clock, atomicMin's a global start stamp, the last block
+ *    (atomicInc) computes the diff and a racy atomicMin/atomicExch picks the
+ *    winner.  B200 form (readings A-6, A-7): lane 0 of every warp samples
+ *    %globaltimer (ns, chip-global) and clock64 at entry and exit; warp 0
+ *    reduces the per-warp samples with __shfl_xor_sync (min start, max end);
+ *    thread 0 does atomicMin(t_start_min) / atomicMax(t_end_max) /
+ *    atomicAdd(cycles, units) on the variant's slot, then counts its CTA.
+ *    The last CTA of a variant computes the score and does ONE atomicMin on
+ *    the packed word (score << 8 | v) — ties go to the lower id (A-8) — and
+ *    the last variant to finish publishes the packed minimum as the
+ *    selection.
+ */
+#ifndef DYSEL_DEVICE_CUH_
+#define DYSEL_DEVICE_CUH_
+
+#include <stdint.h>
+
+#include "dysel.h"
+
+__device__ __forceinline__ uint64_t dysel_globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ uint64_t dysel_clock64() {
+  uint64_t c;
+  asm volatile("mov.u64 %0, %%clock64;" : "=l"(c));
+  return c;
+}
+
+__device__ __forceinline__ uint64_t dysel_ld_acquire_u64(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+/* CTAs per granule for a variant of work-assignment factor wa. */
+__host__ __device__ __forceinline__ uint64_t dysel_ctas_per_granule(const dysel_slice &s, const uint32_t wa[3]) {
+  return (uint64_t)(s.g[0] / wa[0]) * (s.g[1] / wa[1]) * (s.g[2] / wa[2]);
+}
+
+__host__ __device__ __forceinline__ uint64_t dysel_slice_ctas(const dysel_slice &s, const uint32_t wa[3]) {
+  return s.granule_count * dysel_ctas_per_granule(s, wa);
+}
+
+/* First unit (ux, uy, uz) of CTA `cta` of a launch over slice s; returns false
+ * when that tile lies wholly outside U (edge granule). */
+__host__ __device__ __forceinline__ bool dysel_cta_origin(const dysel_slice &s, const uint32_t wa[3], uint64_t cta,
+                                                          uint64_t u[3]) {
+  const uint32_t h0 = s.g[0] / wa[0], h1 = s.g[1] / wa[1], h2 = s.g[2] / wa[2];
+  const uint64_t hper = (uint64_t)h0 * h1 * h2;
+  const uint64_t gi = cta / hper, sub = cta % hper;
+  const uint64_t j = s.granule_begin + gi * s.granule_stride;
+  const uint64_t gx = j % s.G[0], gy = (j / s.G[0]) % s.G[1], gz = j / ((uint64_t)s.G[0] * s.G[1]);
+  const uint64_t sx = sub % h0, sy = (sub / h0) % h1, sz = sub / ((uint64_t)h0 * h1);
+  u[0] = gx * s.g[0] + sx * wa[0];
+  u[1] = gy * s.g[1] + sy * wa[1];
+  u[2] = gz * s.g[2] + sz * wa[2];
+  return u[0] < s.U[0] && u[1] < s.U[1] && u[2] < s.U[2];
+}
+
+/* Gated batch copy: false => this CTA must exit (another variant was selected). */
+__device__ __forceinline__ bool dysel_gate_open(const dysel_slice &s) {
+  if (s.gate == nullptr) return true;
+  return (int32_t)(dysel_ld_acquire_u64(s.gate) & 0xffu) == s.variant;
+}
+
+struct dysel_prof_smem {
+  unsigned long long t0[32], t1[32], c0[32], c1[32];
+};
+
+/* Call with all threads of the CTA at kernel entry (after any early exit
+ * that is uniform for the CTA).  No-op when s.timer == NULL. */
+__device__ __forceinline__ void dysel_prof_begin(const dysel_slice &s, dysel_prof_smem &sm) {
+  if (s.timer == nullptr) return;
+  if ((threadIdx.x & 31) == 0) {
+    const uint32_t w = (threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z)) >> 5;
+    sm.c0[w] = dysel_clock64();
+    sm.t0[w] = dysel_globaltimer();
+  }
+}
+
+/* Call with all threads at the end of the CTA's work.  `units` = units this
+ * CTA processed (for cycles/unit scoring). */
+__device__ __forceinline__ void dysel_prof_end(const dysel_slice &s, dysel_prof_smem &sm, uint32_t units) {
+  if (s.timer == nullptr) return;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const uint32_t nw = (blockDim.x * blockDim.y * blockDim.z + 31) >> 5;
+  if ((tid & 31) == 0) {
+    sm.t1[tid >> 5] = dysel_globaltimer();
+    sm.c1[tid >> 5] = dysel_clock64();
+  }
+  __syncthreads();
+  if (tid < 32) {
+    const uint32_t l = tid;
+    unsigned long long t0 = l < nw ? sm.t0[l] : ~0ull, t1 = l < nw ? sm.t1[l] : 0ull;
+    unsigned long long c0 = l < nw ? sm.c0[l] : ~0ull, c1 = l < nw ? sm.c1[l] : 0ull;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      t0 = min(t0, __shfl_xor_sync(0xffffffffu, t0, o));
+      t1 = max(t1, __shfl_xor_sync(0xffffffffu, t1, o));
+      c0 = min(c0, __shfl_xor_sync(0xffffffffu, c0, o));
+      c1 = max(c1, __shfl_xor_sync(0xffffffffu, c1, o));
+    }
+    if (l == 0) {
+      dysel_timer_slot *slot = s.timer;
+      atomicMin((unsigned long long *)&slot->t_start_min, t0);
+      atomicMax((unsigned long long *)&slot->t_end_max, t1);
+      atomicAdd((unsigned long long *)&slot->cycles, c1 - c0);
+      atomicAdd((unsigned long long *)&slot->units, (unsigned long long)units);
+      __threadfence();
+      const uint32_t done = atomicAdd(s.ctas_done, 1u) + 1u;
+      if (done == s.ctas_total) {           /* last CTA of this variant */
+        __threadfence();
+        const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
+        const unsigned long long b = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
+        const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
+        const unsigned long long un = atomicAdd((unsigned long long *)&slot->units, 0ull);
+        unsigned long long score = s.score_cycles ? (un ? cy / un : (1ull << 56) - 1) : (b - a);
+        if (score > (1ull << 56) - 1) score = (1ull << 56) - 1;
+        atomicMin((unsigned long long *)s.best, (score << 8) | (unsigned)s.variant);
+        __threadfence();
+        const uint32_t vd = atomicAdd(s.variants_done, 1u) + 1u;
+        if (vd == s.n_variants) {           /* last variant: publish the selection */
+          __threadfence();
+          const unsigned long long fin = atomicAdd((unsigned long long *)s.best, 0ull);
+          atomicExch((unsigned long long *)s.sel, fin);
+        }
+      }
+    }
+  }
+}
+
+#endif /* DYSEL_DEVICE_CUH_ */

@@ -1,0 +1,182 @@
+// Multi-GPU DySel: row-sharded SpMV and M-sharded SGEMM over
+// NCCL (NVLink 5 / NVSwitch).  The paper is single-GPU over PCIe
+// (P:L1000-1002); each shard micro-profiles and selects on its own slice, so
+// different shards may run different variants — the paper's "mixed version"
+// (P:L1100-1104).  The only exchange step is the allgather of the output
+// (grouped ncclBroadcast, one root per shard = allgatherv, in place).
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "internal.h"
+
+using namespace dysel;
+
+// NCCL is resolved lazily with dlopen: no link-time dependency, and when
+// torch has already loaded its libnccl.so.2 the same copy is reused (two
+// NCCL versions in one process would clash).
+namespace {
+struct NcclApi {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId *);
+  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int);
+  ncclResult_t (*CommDestroy)(ncclComm_t);
+  ncclResult_t (*GroupStart)();
+  ncclResult_t (*GroupEnd)();
+  ncclResult_t (*Broadcast)(const void *, void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
+  const char *(*GetErrorString)(ncclResult_t);
+};
+NcclApi &nccl() {
+  static NcclApi api = [] {
+    NcclApi a{};
+    void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return a;
+    a.GetUniqueId = (decltype(a.GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    a.CommInitRank = (decltype(a.CommInitRank))dlsym(h, "ncclCommInitRank");
+    a.CommDestroy = (decltype(a.CommDestroy))dlsym(h, "ncclCommDestroy");
+    a.GroupStart = (decltype(a.GroupStart))dlsym(h, "ncclGroupStart");
+    a.GroupEnd = (decltype(a.GroupEnd))dlsym(h, "ncclGroupEnd");
+    a.Broadcast = (decltype(a.Broadcast))dlsym(h, "ncclBroadcast");
+    a.GetErrorString = (decltype(a.GetErrorString))dlsym(h, "ncclGetErrorString");
+    a.ok = a.GetUniqueId && a.CommInitRank && a.CommDestroy && a.GroupStart && a.GroupEnd && a.Broadcast &&
+           a.GetErrorString;
+    return a;
+  }();
+  return api;
+}
+}  // namespace
+
+#define DYSEL_NCCL_TRY(ctx, expr)                                                 \
+  do {                                                                            \
+    ncclResult_t r__ = (expr);                                                    \
+    if (r__ != ncclSuccess) {                                                     \
+      set_error((ctx), std::string(#expr) + ": " + nccl().GetErrorString(r__));   \
+      return DYSEL_ERR_NCCL;                                                      \
+    }                                                                             \
+  } while (0)
+
+void dysel::comm_free(dysel_ctx *ctx) {
+  if (ctx && ctx->nccl_comm) {
+    if (nccl().ok) nccl().CommDestroy((ncclComm_t)ctx->nccl_comm);
+    ctx->nccl_comm = nullptr;
+  }
+}
+
+extern "C" {
+
+dysel_status dysel_comm_unique_id(void *out) {
+  if (!out) return DYSEL_ERR_INVALID;
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  ncclUniqueId id;
+  if (!nccl().ok || nccl().GetUniqueId(&id) != ncclSuccess) return DYSEL_ERR_NCCL;
+  memcpy(out, &id, sizeof(id));
+  return DYSEL_OK;
+}
+
+dysel_status dysel_comm_init(dysel_ctx *ctx, const void *uid, int rank, int world) {
+  if (!ctx || !uid || world < 1 || rank < 0 || rank >= world) return DYSEL_ERR_INVALID;
+  comm_free(ctx);
+  ctx->rank = rank;
+  ctx->world = world;
+  if (world == 1) return DYSEL_OK;
+  ncclUniqueId id;
+  memcpy(&id, uid, sizeof(id));
+  ncclComm_t comm;
+  DYSEL_CUDA_TRY(ctx, cudaSetDevice(ctx->device));
+  if (!nccl().ok) {
+    set_error(ctx, "libnccl.so.2 could not be loaded");
+    return DYSEL_ERR_NCCL;
+  }
+  DYSEL_NCCL_TRY(ctx, nccl().CommInitRank(&comm, world, id, rank));
+  ctx->nccl_comm = comm;
+  return DYSEL_OK;
+}
+
+// bounds[g] = smallest r with row_ptr[r] * world >= g * nnz, snapped down to a
+// multiple of 256 rows (one SpMV unit), bounds[0] = 0, bounds[world] = n.
+dysel_status dysel_partition_rows(const int32_t *rp, int64_t n, int world, int64_t *bounds) {
+  if (!rp || n < 0 || world < 1 || !bounds) return DYSEL_ERR_INVALID;
+  const int64_t nnz = rp[n];
+  bounds[0] = 0;
+  for (int g = 1; g < world; ++g) {
+    const int64_t target = (int64_t)g * nnz;   // compare row_ptr[r] * world >= g * nnz (exact integers)
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi) / 2;
+      if ((int64_t)rp[mid] * world >= target)
+        hi = mid;
+      else
+        lo = mid + 1;
+    }
+    bounds[g] = std::max<int64_t>(bounds[g - 1], (lo / 256) * 256);
+  }
+  bounds[world] = n;
+  return DYSEL_OK;
+}
+
+static dysel_status allgatherv(dysel_ctx *ctx, float *buf, const int64_t *offs, const int64_t *counts,
+                               cudaStream_t st) {
+  if (ctx->world == 1 || !ctx->nccl_comm) return DYSEL_OK;
+  ncclComm_t comm = (ncclComm_t)ctx->nccl_comm;
+  DYSEL_NCCL_TRY(ctx, nccl().GroupStart());
+  for (int r = 0; r < ctx->world; ++r)
+    if (counts[r] > 0)
+      DYSEL_NCCL_TRY(ctx, nccl().Broadcast(buf + offs[r], buf + offs[r], (size_t)counts[r], ncclFloat, r, comm, st));
+  DYSEL_NCCL_TRY(ctx, nccl().GroupEnd());
+  return DYSEL_OK;
+}
+
+dysel_status dysel_comm_broadcast(dysel_ctx *ctx, float *d_buf, size_t n, int root, void *stream) {
+  if (!ctx || (n > 0 && !d_buf) || root < 0 || root >= ctx->world) return DYSEL_ERR_INVALID;
+  if (ctx->world == 1 || !ctx->nccl_comm || n == 0) return DYSEL_OK;
+  DYSEL_NCCL_TRY(ctx, nccl().Broadcast(d_buf, d_buf, n, ncclFloat, root, (ncclComm_t)ctx->nccl_comm,
+                                    (cudaStream_t)stream));
+  return DYSEL_OK;
+}
+
+dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local, const int64_t *bounds, const float *d_x,
+                                float *d_y, float f, uint32_t mode, void *stream, dysel_report *rep) {
+  if (!ctx || !local || !bounds || !d_y) return DYSEL_ERR_INVALID;
+  const int R = ctx->world;
+  int64_t offs[1024], counts[1024];
+  if (R > 1024) return DYSEL_ERR_UNSUPPORTED;
+  for (int r = 0; r < R; ++r) {
+    offs[r] = bounds[r];
+    counts[r] = bounds[r + 1] - bounds[r];
+  }
+  dysel_spmv_plan_info info;
+  DYSEL_TRY(dysel_spmv_plan_get_info(local, &info));
+  if (info.n_rows != counts[ctx->rank]) {
+    set_error(ctx, "dysel_spmv_sharded: local plan rows != bounds slice");
+    return DYSEL_ERR_INVALID;
+  }
+  DYSEL_TRY(dysel_spmv(ctx, local, d_x, d_y + offs[ctx->rank], f, mode, stream, rep));
+  return allgatherv(ctx, d_y, offs, counts, (cudaStream_t)stream);
+}
+
+dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A, int lda,
+                                 const float *d_B, int ldb, float beta, float *d_C, int ldc, float f, uint32_t mode,
+                                 void *stream, dysel_report *rep) {
+  if (!ctx || M < 0) return DYSEL_ERR_INVALID;
+  const int R = ctx->world;
+  if (R > 1024) return DYSEL_ERR_UNSUPPORTED;
+  // M-blocks of ceil(M/R) rounded up to 128 rows (one tcgen05 tile)
+  const int64_t per = (((int64_t)M + R - 1) / R + 127) / 128 * 128;
+  int64_t offs[1024], counts[1024];
+  for (int r = 0; r < R; ++r) {
+    const int64_t m0 = std::min<int64_t>((int64_t)r * per, M), m1 = std::min<int64_t>((int64_t)(r + 1) * per, M);
+    offs[r] = m0 * ldc;
+    counts[r] = (m1 - m0) * ldc;
+  }
+  const int64_t m0 = std::min<int64_t>((int64_t)ctx->rank * per, M);
+  const int64_t m1 = std::min<int64_t>((int64_t)(ctx->rank + 1) * per, M);
+  if (m1 > m0)
+    DYSEL_TRY(dysel_sgemm(ctx, (int)(m1 - m0), N, K, alpha, d_A + m0 * lda, lda, d_B, ldb, beta, d_C + m0 * ldc, ldc, f,
+                          mode, stream, rep));
+  return allgatherv(ctx, d_C, offs, counts, (cudaStream_t)stream);
+}
+
+}  // extern "C"

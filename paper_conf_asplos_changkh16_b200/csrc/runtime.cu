@@ -1,0 +1,746 @@
+// libdysel runtime: context, slice planner, variant registry, selection cache
+// and the generic dysel_launch orchestrator.
+//
+// Paper passages: runtime interface Fig. 6 (§3.1); GPU runtime —
+// three extended copies, in-kernel timers, streams, sync / async host code
+// (§3.3); safe-point / uniform / side-effect analyses
+// (§3.4); orchestration (§2.4); Table 1.
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+
+#include "dysel_device.cuh"
+#include "internal.h"
+
+namespace dysel {
+
+void set_error(dysel_ctx *ctx, const std::string &msg) {
+  if (ctx) ctx->last_error = msg;
+}
+
+dysel_status check_launch(dysel_ctx *ctx, const char *what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    set_error(ctx, std::string(what) + ": " + cudaGetErrorString(e));
+    return DYSEL_ERR_CUDA;
+  }
+  if (ctx) ctx->launches++;
+  return DYSEL_OK;
+}
+
+dysel_status scratch(dysel_ctx *ctx, ScratchBuf &b, size_t bytes) {
+  if (b.bytes >= bytes) return DYSEL_OK;
+  if (b.ptr) {
+    cudaDeviceSynchronize();
+    cudaFree(b.ptr);
+    b.ptr = nullptr;
+    b.bytes = 0;
+  }
+  size_t want = std::max<size_t>(bytes, 4096);
+  if (cudaMalloc(&b.ptr, want) != cudaSuccess) {
+    cudaGetLastError();
+    set_error(ctx, "cudaMalloc scratch failed");
+    return DYSEL_ERR_NOMEM;
+  }
+  b.bytes = want;
+  return DYSEL_OK;
+}
+
+uint64_t now_ns() {
+  return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+             std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+dysel_status push_pending_sel(dysel_ctx *ctx, const std::string &sig, const uint64_t *d_sel, cudaStream_t st) {
+  int i = ctx->pending_head;
+  PendingSel &p = ctx->pending[i];
+  if (p.used) {   // ring full: retire the oldest entry first
+    cudaEventSynchronize(p.ev);
+    resolve_pending(ctx, nullptr);
+  }
+  DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&ctx->h_pending_sel[i], d_sel, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  DYSEL_CUDA_TRY(ctx, cudaEventRecord(p.ev, st));
+  p.sig = sig;
+  p.used = true;
+  ctx->pending_head = (i + 1) % kPendingRing;
+  return DYSEL_OK;
+}
+
+void resolve_pending(dysel_ctx *ctx, const char *block_sig) {
+  // oldest first, so the latest selection of a sig wins
+  for (int k = 0; k < kPendingRing; ++k) {
+    int i = (ctx->pending_head + k) % kPendingRing;
+    PendingSel &p = ctx->pending[i];
+    if (!p.used) continue;
+    if (block_sig && p.sig == block_sig) cudaEventSynchronize(p.ev);
+    if (cudaEventQuery(p.ev) != cudaSuccess) continue;
+    uint64_t w = ctx->h_pending_sel[i];
+    if (w != ~0ull) ctx->sel_cache[p.sig] = (int)(w & 0xff);
+    p.used = false;
+  }
+  cudaGetLastError();
+}
+
+static uint64_t lcm64(uint64_t a, uint64_t b) { return a / std::gcd(a, b) * b; }
+
+// Slice planning — a-2 / readings A-1, A-2, A-3.  Mirrors oracle/slice_plan.py
+// rule for rule (tests compare the two on the same inputs).
+dysel_status make_plan(dysel_ctx *ctx, const uint64_t U_in[3], const uint32_t (*wa)[3], int K, float f, int n_sm,
+                       int default_variant, uint32_t mode, const uint32_t *vflags, Plan *out) {
+  Plan p;
+  if (K < 1 || K > DYSEL_MAX_VARIANTS || !(f >= 0.0f && f <= 1.0f) || default_variant < 0 ||
+      default_variant >= K) {
+    set_error(ctx, "invalid plan arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  p.K = K;
+  for (int d = 0; d < 3; ++d) {
+    p.U[d] = U_in[d] == 0 ? 0 : U_in[d];
+    uint64_t g = 1;
+    for (int v = 0; v < K; ++v) {
+      if (wa[v][d] == 0) {
+        set_error(ctx, "wa = 0");
+        return DYSEL_ERR_INVALID;
+      }
+      g = lcm64(g, wa[v][d]);
+    }
+    if (g > 0xffffffffull) {
+      set_error(ctx, "LCM of wa too large");
+      return DYSEL_ERR_INVALID;
+    }
+    p.g[d] = (uint32_t)g;
+    uint64_t G = (p.U[d] + g - 1) / g;
+    if (G > 0xffffffffull) {
+      set_error(ctx, "too many granules");
+      return DYSEL_ERR_INVALID;
+    }
+    p.G[d] = (uint32_t)G;
+  }
+  p.Gn = (uint64_t)p.G[0] * p.G[1] * p.G[2];
+  for (int v = 0; v < K; ++v)
+    p.h[v] = (uint64_t)(p.g[0] / wa[v][0]) * (p.g[1] / wa[v][1]) * (p.g[2] / wa[v][2]);
+  // mode resolution (A-10, A-11, A-13; programmer override wins)
+  int base = (int)(mode & 3u);
+  if (base == DYSEL_AUTO) {
+    bool at = false, nu = false;
+    for (int v = 0; v < K; ++v) {
+      at |= (vflags[v] & DYSEL_V_ATOMICS) != 0;
+      nu |= (vflags[v] & DYSEL_V_NONUNIFORM) != 0;
+    }
+    base = at ? DYSEL_SWAP : (nu ? DYSEL_HYBRID : DYSEL_FULLY);
+  }
+  if (base == DYSEL_SWAP && (mode & DYSEL_ASYNC)) {
+    set_error(ctx, "swap-based profiling cannot run asynchronously (Table 1, P:L735-739)");
+    return DYSEL_ERR_UNSUPPORTED;
+  }
+  p.mode = base;
+  uint64_t c = (uint64_t)std::floor((double)f * (double)p.Gn / (double)K);   // A-1
+  uint64_t q = (uint64_t)(n_sm / K);                                          // A-2
+  if (q > 0) {
+    uint64_t hmin = p.h[0];
+    for (int v = 1; v < K; ++v) hmin = std::min(hmin, p.h[v]);
+    uint64_t cq = q / std::gcd(q, hmin);
+    if (c >= cq) c = (c / cq) * cq;
+  }
+  uint64_t def_ctas = 1;
+  for (int d = 0; d < 3; ++d) def_ctas *= (p.U[d] + wa[default_variant][d] - 1) / wa[default_variant][d];
+  bool active = !(mode & DYSEL_NO_PROFILE) && K >= 2 && p.Gn > 0;
+  if (active) {
+    if (mode & DYSEL_FORCE_PROFILE) {
+      if (c == 0) c = (base == DYSEL_FULLY ? p.Gn >= (uint64_t)K : p.Gn >= 1) ? 1 : 0;
+      active = c >= 1;
+    } else {
+      active = c >= 1 && def_ctas >= 128;   // P:L328-337 (A-3)
+    }
+  }
+  p.active = active;
+  p.c = active ? c : 0;
+  *out = p;
+  return DYSEL_OK;
+}
+
+// -------------------------------------------------------------- small kernels
+__global__ void init_prof_kernel(DevProf *p, int K, int def) {
+  int i = threadIdx.x;
+  if (i < DYSEL_MAX_VARIANTS) {
+    p->slot[i].t_start_min = ~0ull;
+    p->slot[i].t_end_max = 0;
+    p->slot[i].units = 0;
+    p->slot[i].cycles = 0;
+    p->ctas_done[i] = 0;
+  }
+  if (i == 0) {
+    p->variants_done = 0;
+    p->best = (((1ull << 56) - 1) << 8) | (uint64_t)def;
+    p->sel = ~0ull;
+  }
+}
+
+__global__ void gated_copy_kernel(uint4 *dst, const uint4 *src, size_t n16, const uint64_t *gate, int v) {
+  if ((int)(dysel_ld_acquire_u64(gate) & 0xffu) != v) return;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n16; i += (size_t)gridDim.x * blockDim.x)
+    dst[i] = src[i];
+}
+
+__global__ void timer_calib_kernel(uint64_t samples, uint64_t spin_ns, uint64_t *out) {
+  uint64_t prev = dysel_globaltimer(), best = ~0ull;
+  for (uint64_t i = 0; i < samples; ++i) {
+    uint64_t t = dysel_globaltimer();
+    if (t != prev) {
+      best = min(best, t - prev);
+      prev = t;
+    }
+  }
+  uint64_t t0 = dysel_globaltimer(), c0 = dysel_clock64(), t1;
+  do {
+    t1 = dysel_globaltimer();
+  } while (t1 - t0 < spin_ns);
+  uint64_t c1 = dysel_clock64();
+  out[0] = best;
+  out[1] = t1 - t0;
+  out[2] = c1 - c0;
+}
+
+// Known-cost variant (c-8): spins cost_ns per unit, writes out[u] = v + 1.
+__global__ void spin_variant_kernel(dysel_slice s, uint32_t cost_ns, uint32_t *out) {
+  __shared__ dysel_prof_smem psm;
+  if (!dysel_gate_open(s)) return;
+  const uint32_t wa[3] = {1, 1, 1};
+  dysel_prof_begin(s, psm);
+  uint64_t u[3];
+  bool ok = dysel_cta_origin(s, wa, blockIdx.x, u);
+  if (ok && threadIdx.x == 0) {
+    uint64_t t0 = dysel_globaltimer();
+    while (dysel_globaltimer() - t0 < cost_ns) {
+    }
+    out[u[0]] = (uint32_t)s.variant + 1;
+  }
+  __syncthreads();
+  dysel_prof_end(s, psm, ok ? 1u : 0u);
+}
+
+static dysel_status spin_fn(const dysel_slice *s, void *const *args, void *stream, void *user) {
+  uint64_t ctas = s->granule_count * (uint64_t)s->g[0] * s->g[1] * s->g[2];
+  if (ctas == 0) return DYSEL_OK;
+  spin_variant_kernel<<<(unsigned)ctas, 32, 0, (cudaStream_t)stream>>>(*s, (uint32_t)(uintptr_t)user,
+                                                                         (uint32_t *)args[0]);
+  return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
+}
+
+// ------------------------------------------------------------ launch helpers
+static dysel_slice base_slice(const Plan &p) {
+  dysel_slice s;
+  memset(&s, 0, sizeof(s));
+  for (int d = 0; d < 3; ++d) {
+    s.g[d] = p.g[d];
+    s.G[d] = p.G[d];
+    s.U[d] = p.U[d];
+  }
+  s.granule_stride = 1;
+  return s;
+}
+
+static uint64_t host_score(const dysel_timer_slot &t, bool cycles) {
+  const uint64_t cap = (1ull << 56) - 1;
+  uint64_t s = cycles ? (t.units ? t.cycles / t.units : cap) : (t.t_end_max - t.t_start_min);
+  return std::min(s, cap);
+}
+
+static void fill_report_common(dysel_report *rep, const Plan &p, int mode_used, int profiled, int selected) {
+  if (!rep) return;
+  rep->mode_used = mode_used;
+  rep->profiled = profiled;
+  rep->selected = selected;
+  rep->n_variants = p.K;
+  rep->c = p.c;
+  rep->n_granules = p.Gn;
+  rep->eager_units = 0;
+  rep->n_slices = 0;
+  for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v) {
+    rep->score[v] = rep->makespan_ns[v] = rep->units[v] = rep->cycles[v] = 0;
+  }
+}
+
+static void add_slice_rec(dysel_report *rep, const dysel_slice &s) {
+  if (!rep || !rep->slices || rep->n_slices >= rep->slices_cap) {
+    if (rep) rep->n_slices++;
+    return;
+  }
+  dysel_slice_rec &r = rep->slices[rep->n_slices++];
+  r.granule_begin = s.granule_begin;
+  r.granule_count = s.granule_count;
+  r.granule_stride = s.granule_stride;
+  r.variant = s.variant;
+  r.role = s.role;
+}
+
+static void mark_units(dysel_report *rep, const dysel_slice &s) {
+  if (!rep || !rep->unit_variant) return;
+  for (uint64_t i = 0; i < s.granule_count; ++i) {
+    uint64_t j = s.granule_begin + i * s.granule_stride;
+    if (j < rep->unit_variant_cap) rep->unit_variant[j] = (uint8_t)s.variant;
+  }
+}
+
+}  // namespace dysel
+
+using namespace dysel;
+
+// ===================================================================== C ABI
+extern "C" {
+
+const char *dysel_status_str(dysel_status s) {
+  switch (s) {
+    case DYSEL_OK: return "DYSEL_OK";
+    case DYSEL_ERR_INVALID: return "DYSEL_ERR_INVALID";
+    case DYSEL_ERR_UNSUPPORTED: return "DYSEL_ERR_UNSUPPORTED";
+    case DYSEL_ERR_NOMEM: return "DYSEL_ERR_NOMEM";
+    case DYSEL_ERR_CUDA: return "DYSEL_ERR_CUDA";
+    case DYSEL_ERR_NOT_FOUND: return "DYSEL_ERR_NOT_FOUND";
+    case DYSEL_ERR_NCCL: return "DYSEL_ERR_NCCL";
+  }
+  return "DYSEL_ERR_UNKNOWN";
+}
+
+const char *dysel_last_error(const dysel_ctx *ctx) { return ctx ? ctx->last_error.c_str() : "NULL ctx"; }
+
+dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
+  if (!out) return DYSEL_ERR_INVALID;
+  *out = nullptr;
+  dysel_ctx *ctx = new (std::nothrow) dysel_ctx();
+  if (!ctx) return DYSEL_ERR_NOMEM;
+  ctx->device = cuda_device;
+  auto fail = [&](dysel_status s) {
+    dysel_destroy(ctx);
+    return s;
+  };
+  if (cudaSetDevice(cuda_device) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(DYSEL_ERR_CUDA);
+  }
+  int v = 0;
+  cudaDeviceGetAttribute(&ctx->n_sm, cudaDevAttrMultiProcessorCount, cuda_device);
+  cudaDeviceGetAttribute(&v, cudaDevAttrL2CacheSize, cuda_device);
+  ctx->l2_bytes = (uint64_t)v;
+  for (int i = 0; i < DYSEL_MAX_VARIANTS; ++i) {
+    if (cudaStreamCreateWithFlags(&ctx->fork[i], cudaStreamNonBlocking) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+    if (cudaEventCreateWithFlags(&ctx->ev_join[i], cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  }
+  if (cudaStreamCreateWithFlags(&ctx->query, cudaStreamNonBlocking) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (cudaEventCreateWithFlags(&ctx->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (cudaEventCreateWithFlags(&ctx->ev_fork2, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (cudaMalloc(&ctx->d_prof, sizeof(DevProf)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+  if (cudaMallocHost(&ctx->h_prof, sizeof(DevProf)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+  if (cudaMallocHost(&ctx->h_pending_sel, kPendingRing * sizeof(uint64_t)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+  for (int i = 0; i < kPendingRing; ++i)
+    if (cudaEventCreateWithFlags(&ctx->pending[i].ev, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (spmv_ctx_init(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
+  if (sgemm_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
+  uint64_t tick = 0;
+  double cpn = 0;
+  if (dysel_timer_calibrate(ctx, 1u << 16, 20000, &tick, &cpn) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
+  ctx->gt_tick_ns = tick;
+  *out = ctx;
+  return DYSEL_OK;
+}
+
+void dysel_destroy(dysel_ctx *ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->device);
+  cudaDeviceSynchronize();
+  spmv_ctx_free(ctx);
+  for (int i = 0; i < DYSEL_MAX_VARIANTS; ++i) {
+    if (ctx->fork[i]) cudaStreamDestroy(ctx->fork[i]);
+    if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
+  }
+  if (ctx->query) cudaStreamDestroy(ctx->query);
+  if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
+  if (ctx->ev_fork2) cudaEventDestroy(ctx->ev_fork2);
+  if (ctx->d_prof) cudaFree(ctx->d_prof);
+  if (ctx->h_prof) cudaFreeHost(ctx->h_prof);
+  if (ctx->h_pending_sel) cudaFreeHost(ctx->h_pending_sel);
+  for (int i = 0; i < kPendingRing; ++i)
+    if (ctx->pending[i].ev) cudaEventDestroy(ctx->pending[i].ev);
+  for (auto &b : ctx->sandbox)
+    if (b.ptr) cudaFree(b.ptr);
+  if (ctx->unit_variant.ptr) cudaFree(ctx->unit_variant.ptr);
+  comm_free(ctx);
+  delete ctx;
+}
+
+dysel_status dysel_device_info(const dysel_ctx *ctx, int *n_sm, uint64_t *tick, uint64_t *l2) {
+  if (!ctx) return DYSEL_ERR_INVALID;
+  if (n_sm) *n_sm = ctx->n_sm;
+  if (tick) *tick = ctx->gt_tick_ns;
+  if (l2) *l2 = ctx->l2_bytes;
+  return DYSEL_OK;
+}
+
+uint64_t dysel_kernel_launches(const dysel_ctx *ctx) { return ctx ? ctx->launches : 0; }
+
+dysel_status dysel_timer_calibrate(dysel_ctx *ctx, uint64_t samples, uint64_t spin_ns, uint64_t *tick_ns,
+                                   double *cycles_per_ns) {
+  if (!ctx) return DYSEL_ERR_INVALID;
+  uint64_t *d = nullptr, h[3] = {0, 0, 0};
+  DYSEL_CUDA_TRY(ctx, cudaMalloc(&d, 3 * sizeof(uint64_t)));
+  timer_calib_kernel<<<1, 1>>>(samples, spin_ns, d);
+  dysel_status st = check_launch(ctx, "timer_calib_kernel");
+  if (st == DYSEL_OK && cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost) != cudaSuccess) st = DYSEL_ERR_CUDA;
+  cudaFree(d);
+  if (st != DYSEL_OK) return st;
+  if (tick_ns) *tick_ns = h[0];
+  if (cycles_per_ns) *cycles_per_ns = h[1] ? (double)h[2] / (double)h[1] : 0.0;
+  return DYSEL_OK;
+}
+
+dysel_status dysel_register_variants(dysel_ctx *ctx, const char *sig, const dysel_variant *v, int n,
+                                     int default_variant) {
+  if (!ctx || !sig || !v || n < 1 || n > DYSEL_MAX_VARIANTS || default_variant < 0 || default_variant >= n) {
+    set_error(ctx, "dysel_register_variants: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  Registered r;
+  for (int i = 0; i < n; ++i) {
+    if (!v[i].fn || v[i].wa[0] == 0 || v[i].wa[1] == 0 || v[i].wa[2] == 0 || v[i].n_sandbox_args < 0 ||
+        (v[i].n_sandbox_args > 0 && !v[i].sandbox_args)) {
+      set_error(ctx, "dysel_register_variants: bad variant descriptor");
+      return DYSEL_ERR_INVALID;
+    }
+    r.v.push_back(v[i]);
+    r.sandbox_args.emplace_back(v[i].sandbox_args, v[i].sandbox_args + v[i].n_sandbox_args);
+    r.names.emplace_back(v[i].name ? v[i].name : "");
+    r.v.back().sandbox_args = nullptr;
+    r.v.back().name = nullptr;
+  }
+  r.def = default_variant;
+  ctx->reg[sig] = std::move(r);
+  ctx->sel_cache.erase(sig);
+  return DYSEL_OK;
+}
+
+dysel_status dysel_register_spin_variants(dysel_ctx *ctx, const char *sig, const uint32_t *cost_ns, int n,
+                                          int default_variant) {
+  if (!ctx || !cost_ns || n < 1 || n > DYSEL_MAX_VARIANTS) return DYSEL_ERR_INVALID;
+  static const int sb[1] = {0};
+  dysel_variant vv[DYSEL_MAX_VARIANTS];
+  for (int i = 0; i < n; ++i) {
+    vv[i] = dysel_variant{"spin", spin_fn, {1, 1, 1}, sb, 1, 0, (void *)(uintptr_t)cost_ns[i]};
+  }
+  return dysel_register_variants(ctx, sig, vv, n, default_variant);
+}
+
+dysel_status dysel_get_selection(dysel_ctx *ctx, const char *key, int *variant) {
+  if (!ctx || !key || !variant) return DYSEL_ERR_INVALID;
+  resolve_pending(ctx, key);
+  auto it = ctx->sel_cache.find(key);
+  if (it == ctx->sel_cache.end()) return DYSEL_ERR_NOT_FOUND;
+  *variant = it->second;
+  return DYSEL_OK;
+}
+
+dysel_status dysel_set_selection(dysel_ctx *ctx, const char *key, int variant) {
+  if (!ctx || !key || variant < 0 || variant >= DYSEL_MAX_VARIANTS) return DYSEL_ERR_INVALID;
+  ctx->sel_cache[key] = variant;
+  return DYSEL_OK;
+}
+
+dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key) {
+  if (!ctx) return DYSEL_ERR_INVALID;
+  if (!key)
+    ctx->sel_cache.clear();
+  else
+    ctx->sel_cache.erase(key);
+  return DYSEL_OK;
+}
+
+// Generic DySel launch.  Device path (default): profiling copies of all K
+// variants concurrently on forked streams; the last profiling CTA publishes
+// the packed selection on the device; the remainder is launched as K gated
+// batch copies (only the selected one does work) — no host round trip.
+// DYSEL_HOST_ORCH: the paper's host code — sync waits and reads the selection
+// (P:L927-930); async polls the profiling streams and launches eager chunks of
+// the best-so-far variant until all profiles are in.
+dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrange_units[3], float f, uint32_t mode,
+                          void *const *args, int n_args, const size_t *sandbox_bytes, void *stream_v,
+                          dysel_report *rep) {
+  const uint64_t t_host0 = now_ns();
+  if (!ctx || !sig || !ndrange_units || n_args < 0 || (n_args > 0 && !args)) {
+    set_error(ctx, "dysel_launch: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  auto it = ctx->reg.find(sig);
+  if (it == ctx->reg.end()) {
+    set_error(ctx, std::string("dysel_launch: unknown kernel_sig ") + sig);
+    return DYSEL_ERR_INVALID;
+  }
+  const Registered &R = it->second;
+  const int K = (int)R.v.size();
+  uint32_t wa[DYSEL_MAX_VARIANTS][3], vflags[DYSEL_MAX_VARIANTS];
+  for (int v = 0; v < K; ++v) {
+    for (int d = 0; d < 3; ++d) wa[v][d] = R.v[v].wa[d];
+    vflags[v] = R.v[v].flags;
+  }
+  for (int v = 0; v < K; ++v)
+    for (int a : R.sandbox_args[v])
+      if (a < 0 || a >= n_args) {
+        set_error(ctx, "dysel_launch: sandbox arg index out of range");
+        return DYSEL_ERR_INVALID;
+      }
+  Plan P;
+  DYSEL_TRY(make_plan(ctx, ndrange_units, wa, K, f, ctx->n_sm, R.def, mode, vflags, &P));
+  resolve_pending(ctx, nullptr);
+  cudaStream_t st = (cudaStream_t)stream_v;
+  if (rep) rep->n_slices = 0;
+  if (P.Gn == 0) {
+    fill_report_common(rep, P, P.mode, 0, R.def);
+    return DYSEL_OK;
+  }
+  std::vector<void *> base_args(args, args + n_args);
+  if (!P.active) {   // activation flag off / small workload: one plain batch copy
+    int v = R.def;
+    resolve_pending(ctx, sig);
+    auto c = ctx->sel_cache.find(sig);
+    if (c != ctx->sel_cache.end() && c->second < K) v = c->second;
+    dysel_slice s = base_slice(P);
+    s.granule_count = P.Gn;
+    s.role = DYSEL_ROLE_BATCH;
+    s.variant = v;
+    DYSEL_TRY(R.v[v].fn(&s, base_args.data(), st, R.v[v].user));
+    DYSEL_TRY(check_launch(ctx, "variant batch"));
+    fill_report_common(rep, P, P.mode | (int)(mode & DYSEL_ASYNC), 0, v);
+    add_slice_rec(rep, s);
+    mark_units(rep, s);
+    if (rep) rep->host_ns = now_ns() - t_host0;
+    return DYSEL_OK;
+  }
+  const bool score_cycles = (mode & DYSEL_SCORE_CYCLES) != 0;
+  // generic ASYNC = the paper's host polling path: heterogeneous user kernels
+  // cannot share a device-side ticket scheduler (the SpMV pool does, spmv.cu)
+  const bool host_orch = (mode & DYSEL_HOST_ORCH) != 0 || (mode & DYSEL_ASYNC) != 0;
+  const bool async = (mode & DYSEL_ASYNC) != 0;
+  // ---- per-variant argument vectors (sandboxes / private outputs, Table 1)
+  std::vector<std::vector<void *>> vargs(K, base_args);
+  int nsb_max = 0;
+  for (int v = 0; v < K; ++v) nsb_max = std::max<int>(nsb_max, (int)R.sandbox_args[v].size());
+  if ((P.mode == DYSEL_HYBRID || P.mode == DYSEL_SWAP) && nsb_max > 0 && !sandbox_bytes) {
+    set_error(ctx, "dysel_launch: sandbox_arg_bytes required for hybrid / swap");
+    return DYSEL_ERR_INVALID;
+  }
+  if (P.mode == DYSEL_HYBRID || P.mode == DYSEL_SWAP) {
+    int slot = 0;
+    for (int v = 0; v < K; ++v) {
+      if (P.mode == DYSEL_HYBRID && v == R.def) continue;       // ≤ K-1 sandboxes
+      for (size_t k = 0; k < R.sandbox_args[v].size(); ++k) {
+        if ((size_t)slot >= sizeof(ctx->sandbox) / sizeof(ctx->sandbox[0])) {
+          set_error(ctx, "too many sandbox buffers");
+          return DYSEL_ERR_UNSUPPORTED;
+        }
+        size_t bytes = sandbox_bytes[k];
+        DYSEL_TRY(scratch(ctx, ctx->sandbox[slot], bytes));
+        int a = R.sandbox_args[v][k];
+        if (P.mode == DYSEL_SWAP)   // private output starts as the original output
+          DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(ctx->sandbox[slot].ptr, base_args[a], bytes,
+                                              cudaMemcpyDeviceToDevice, st));
+        vargs[v][a] = ctx->sandbox[slot].ptr;
+        slot++;
+      }
+    }
+  }
+  // ---- profiling copies, concurrently on forked streams
+  init_prof_kernel<<<1, 32, 0, st>>>(ctx->d_prof, K, R.def);
+  DYSEL_TRY(check_launch(ctx, "init_prof_kernel"));
+  DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_start, st));
+  fill_report_common(rep, P, P.mode | (async ? DYSEL_ASYNC : 0), 1, -1);
+  for (int v = 0; v < K; ++v) {
+    dysel_slice s = base_slice(P);
+    s.variant = v;
+    s.granule_count = P.c;
+    if (P.mode == DYSEL_FULLY) {
+      if (mode & DYSEL_CONTIGUOUS) {
+        s.granule_begin = (uint64_t)v * P.c;
+      } else {
+        s.granule_begin = (uint64_t)v;
+        s.granule_stride = (uint64_t)K;
+      }
+      s.role = DYSEL_ROLE_PRODUCTIVE;
+    } else if (P.mode == DYSEL_HYBRID) {
+      s.role = v == R.def ? DYSEL_ROLE_PRODUCTIVE : DYSEL_ROLE_SANDBOX;
+    } else {
+      s.role = DYSEL_ROLE_PRIVATE;
+    }
+    s.timer = &ctx->d_prof->slot[v];
+    s.ctas_done = &ctx->d_prof->ctas_done[v];
+    s.ctas_total = (uint32_t)(P.c * P.h[v]);
+    s.best = &ctx->d_prof->best;
+    s.variants_done = &ctx->d_prof->variants_done;
+    s.n_variants = (uint32_t)K;
+    s.score_cycles = score_cycles ? 1u : 0u;
+    s.sel = &ctx->d_prof->sel;
+    DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[v], ctx->ev_start, 0));
+    DYSEL_TRY(R.v[v].fn(&s, vargs[v].data(), ctx->fork[v], R.v[v].user));
+    DYSEL_TRY(check_launch(ctx, "variant profiling copy"));
+    DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[v], ctx->fork[v]));
+    add_slice_rec(rep, s);
+    if (s.role == DYSEL_ROLE_PRODUCTIVE) mark_units(rep, s);
+  }
+  uint64_t rem_begin = P.mode == DYSEL_FULLY ? (uint64_t)K * P.c : P.c;
+  const uint64_t rem_end = P.Gn;
+  int selected = -1;
+  uint64_t eager_units = 0;
+  if (!host_orch) {
+    // ---- device path: gated remainder, selection never leaves the device
+    for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
+    if (P.mode == DYSEL_SWAP) {
+      for (int v = 0; v < K; ++v)
+        for (size_t k = 0; k < R.sandbox_args[v].size(); ++k) {
+          int a = R.sandbox_args[v][k];
+          size_t n16 = sandbox_bytes[k] / 16;
+          gated_copy_kernel<<<2 * ctx->n_sm, 256, 0, st>>>((uint4 *)base_args[a], (const uint4 *)vargs[v][a], n16,
+                                                          &ctx->d_prof->sel, v);
+          DYSEL_TRY(check_launch(ctx, "gated_copy_kernel"));
+          if (sandbox_bytes[k] % 16)
+            DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync((char *)base_args[a] + n16 * 16, (char *)vargs[v][a] + n16 * 16,
+                                                sandbox_bytes[k] % 16, cudaMemcpyDeviceToDevice, st));
+        }
+    }
+    if (rem_begin < rem_end) {
+      DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, st));
+      for (int v = 0; v < K; ++v) {
+        dysel_slice s = base_slice(P);
+        s.variant = v;
+        s.role = DYSEL_ROLE_BATCH;
+        s.granule_begin = rem_begin;
+        s.granule_count = rem_end - rem_begin;
+        s.gate = &ctx->d_prof->sel;
+        DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[v], ctx->ev_fork2, 0));
+        DYSEL_TRY(R.v[v].fn(&s, base_args.data(), ctx->fork[v], R.v[v].user));
+        DYSEL_TRY(check_launch(ctx, "variant gated batch"));
+        DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[v], ctx->fork[v]));
+      }
+      for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
+    }
+    // selection for the activation-flag cache: async D2H, resolved lazily
+    DYSEL_TRY(push_pending_sel(ctx, sig, &ctx->d_prof->sel, st));
+    if (rep) {   // a report costs a D2H copy + sync
+      DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(ctx->h_prof, ctx->d_prof, sizeof(DevProf), cudaMemcpyDeviceToHost, st));
+      DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+      selected = (int)(ctx->h_prof->sel & 0xff);
+      ctx->sel_cache[sig] = selected;
+    }
+  } else if (!async) {
+    // ---- paper host path, synchronous
+    for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
+    DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(ctx->h_prof, ctx->d_prof, sizeof(DevProf), cudaMemcpyDeviceToHost, st));
+    DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+    selected = (int)(ctx->h_prof->sel & 0xff);
+  } else {
+    // ---- paper host path, asynchronous: poll + eager chunks
+    bool done[DYSEL_MAX_VARIANTS] = {};
+    int ndone = 0;
+    uint64_t best_pack = ~0ull;
+    int best_v = R.def;
+    cudaEvent_t chunk_ev = nullptr;
+    cudaEventCreateWithFlags(&chunk_ev, cudaEventDisableTiming);
+    bool chunk_inflight = false;
+    while (ndone < K) {
+      for (int v = 0; v < K; ++v) {
+        if (done[v]) continue;
+        cudaError_t q = cudaEventQuery(ctx->ev_join[v]);
+        if (q == cudaErrorNotReady) continue;
+        if (q != cudaSuccess) {
+          cudaEventDestroy(chunk_ev);
+          DYSEL_CUDA_TRY(ctx, q);
+        }
+        done[v] = true;
+        ndone++;
+        DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&ctx->h_prof->slot[v], &ctx->d_prof->slot[v], sizeof(dysel_timer_slot),
+                                            cudaMemcpyDeviceToHost, ctx->query));
+        DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(ctx->query));
+        uint64_t pk = (host_score(ctx->h_prof->slot[v], score_cycles) << 8) | (uint64_t)v;
+        if (pk < best_pack) {
+          best_pack = pk;
+          best_v = v;
+        }
+      }
+      if (ndone == K) break;
+      if (rem_begin < rem_end && (!chunk_inflight || cudaEventQuery(chunk_ev) == cudaSuccess)) {
+        uint64_t chunk = std::max<uint64_t>(1, (2ull * ctx->n_sm + P.h[best_v] - 1) / P.h[best_v]);
+        chunk = std::min(chunk, rem_end - rem_begin);
+        dysel_slice s = base_slice(P);
+        s.variant = best_v;
+        s.role = DYSEL_ROLE_EAGER;
+        s.granule_begin = rem_begin;
+        s.granule_count = chunk;
+        DYSEL_TRY(R.v[best_v].fn(&s, base_args.data(), st, R.v[best_v].user));
+        DYSEL_TRY(check_launch(ctx, "variant eager chunk"));
+        cudaEventRecord(chunk_ev, st);
+        chunk_inflight = true;
+        add_slice_rec(rep, s);
+        mark_units(rep, s);
+        rem_begin += chunk;
+        eager_units += chunk;
+      }
+    }
+    cudaEventDestroy(chunk_ev);
+    for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
+    selected = (int)(best_pack & 0xff);
+    ctx->h_prof->sel = best_pack;
+  }
+  if (host_orch) {
+    if (P.mode == DYSEL_SWAP) {
+      for (size_t k = 0; k < R.sandbox_args[selected].size(); ++k) {
+        int a = R.sandbox_args[selected][k];
+        DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(base_args[a], vargs[selected][a], sandbox_bytes[k],
+                                            cudaMemcpyDeviceToDevice, st));
+      }
+    }
+    if (rem_begin < rem_end) {
+      dysel_slice s = base_slice(P);
+      s.variant = selected;
+      s.role = DYSEL_ROLE_BATCH;
+      s.granule_begin = rem_begin;
+      s.granule_count = rem_end - rem_begin;
+      DYSEL_TRY(R.v[selected].fn(&s, base_args.data(), st, R.v[selected].user));
+      DYSEL_TRY(check_launch(ctx, "variant batch"));
+      add_slice_rec(rep, s);
+      mark_units(rep, s);
+    }
+    ctx->sel_cache[sig] = selected;
+  }
+  if (rep) {
+    if (!host_orch && rep) {
+      dysel_slice s = base_slice(P);
+      s.variant = selected;
+      s.role = DYSEL_ROLE_BATCH;
+      s.granule_begin = rem_begin;
+      s.granule_count = rem_end > rem_begin ? rem_end - rem_begin : 0;
+      add_slice_rec(rep, s);
+      mark_units(rep, s);
+    } else {
+      // host paths read slots already (sync) — refresh all for the report
+      DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(ctx->h_prof->slot, ctx->d_prof->slot, sizeof(ctx->h_prof->slot),
+                                          cudaMemcpyDeviceToHost, st));
+      DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+    }
+    if (P.mode == DYSEL_SWAP) {   // winner's private prefix became the output
+      for (uint64_t j = 0; j < P.c && j < rep->unit_variant_cap; ++j)
+        if (rep->unit_variant) rep->unit_variant[j] = (uint8_t)selected;
+    }
+    rep->selected = selected;
+    rep->eager_units = eager_units;
+    for (int v = 0; v < K; ++v) {
+      const dysel_timer_slot &t = ctx->h_prof->slot[v];
+      rep->makespan_ns[v] = t.t_end_max - t.t_start_min;
+      rep->units[v] = t.units;
+      rep->cycles[v] = t.cycles;
+      rep->score[v] = host_score(t, score_cycles);
+    }
+    rep->host_ns = now_ns() - t_host0;
+  }
+  return DYSEL_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,119 @@
+// DySel SGEMM: the built-in variant pool registered through the generic
+// launcher (dysel_launch), so SGEMM exercises the same slice planner, device
+// timing and gated device-side remainder as user-registered kernels.
+// Unit = one 32x32 tile of C; wa = (tile_N/32, tile_M/32) (SURVEY §8 notation).
+#include <cstring>
+
+#include "internal.h"
+#include "sgemm_simt.cuh"
+#include "sgemm_tc.cuh"
+
+namespace dysel {
+
+static const char *kSgemmSig = "dysel.sgemm";
+
+template <int VID>
+static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
+  const SgemmArgs &g = *(const SgemmArgs *)args[1];
+  float *C = (float *)args[0];
+  cudaStream_t st = (cudaStream_t)stream;
+  uint32_t wa[3];
+  if constexpr (VID == DYSEL_SGEMM_S64) {
+    wa[0] = 2; wa[1] = 2; wa[2] = 1;
+  } else if constexpr (VID == DYSEL_SGEMM_S128) {
+    wa[0] = 4; wa[1] = 4; wa[2] = 1;
+  } else if constexpr (VID == DYSEL_SGEMM_T128x64) {
+    wa[0] = 2; wa[1] = 4; wa[2] = 1;
+  } else {
+    wa[0] = 4; wa[1] = 4; wa[2] = 1;
+  }
+  const uint64_t ctas = dysel_slice_ctas(*s, wa);
+  if (ctas == 0) return DYSEL_OK;
+  if constexpr (VID == DYSEL_SGEMM_S64) {
+    sgemm_simt_kernel<64, 64, 16, 4, 4><<<(unsigned)ctas, 256, 0, st>>>(g, C, *s);
+  } else if constexpr (VID == DYSEL_SGEMM_S128) {
+    sgemm_simt_kernel<128, 128, 8, 8, 8><<<(unsigned)ctas, 256, 0, st>>>(g, C, *s);
+  } else if constexpr (VID == DYSEL_SGEMM_T128x64) {
+    DYSEL_TRY(launch_tc_sgemm<64>(g, C, *s, (unsigned)ctas, st));
+  } else {
+    DYSEL_TRY(launch_tc_sgemm<128>(g, C, *s, (unsigned)ctas, st));
+  }
+  return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
+}
+
+dysel_status sgemm_register(dysel_ctx *ctx) {
+  static const int sb[1] = {0};
+  dysel_variant v[DYSEL_SGEMM_NVARIANTS] = {
+      {"simt64x64", sgemm_variant_fn<0>, {2, 2, 1}, sb, 1, 0, nullptr},
+      {"simt128x128", sgemm_variant_fn<1>, {4, 4, 1}, sb, 1, 0, nullptr},
+      {"tc3xtf32_128x64", sgemm_variant_fn<2>, {2, 4, 1}, sb, 1, 0, nullptr},
+      {"tc3xtf32_128x128", sgemm_variant_fn<3>, {4, 4, 1}, sb, 1, 0, nullptr},
+  };
+  DYSEL_TRY(tc_sgemm_init());
+  return dysel_register_variants(ctx, kSgemmSig, v, DYSEL_SGEMM_NVARIANTS, DYSEL_SGEMM_S64);
+}
+
+static dysel_status check_args(dysel_ctx *ctx, int M, int N, int K, const float *A, int lda, const float *B, int ldb,
+                               float *C, int ldc) {
+  if (M < 0 || N < 0 || K < 0 || (M > 0 && N > 0 && (!C || ldc < N)) || (M > 0 && K > 0 && (!A || lda < K)) ||
+      (N > 0 && K > 0 && (!B || ldb < N))) {
+    set_error(ctx, "dysel_sgemm: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  return DYSEL_OK;
+}
+
+}  // namespace dysel
+
+using namespace dysel;
+
+extern "C" {
+
+dysel_status dysel_sgemm(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A, int lda, const float *d_B,
+                         int ldb, float beta, float *d_C, int ldc, float f, uint32_t mode, void *stream,
+                         dysel_report *rep) {
+  if (!ctx) return DYSEL_ERR_INVALID;
+  DYSEL_TRY(check_args(ctx, M, N, K, d_A, lda, d_B, ldb, d_C, ldc));
+  if (rep) rep->n_slices = 0;
+  if ((int64_t)M * N == 0) return DYSEL_OK;
+  SgemmArgs g{M, N, K, alpha, beta, d_A, lda, d_B, ldb, d_C, ldc};
+  // A single-wave SGEMM leaves no room for eager chunks: without HOST_ORCH,
+  // ASYNC runs the device-gated synchronous path (SURVEY §7 hard part 1).
+  if (!(mode & DYSEL_HOST_ORCH)) mode &= ~DYSEL_ASYNC;
+  const uint64_t U[3] = {(uint64_t)(N + 31) / 32, (uint64_t)(M + 31) / 32, 1};
+  void *args[2] = {d_C, &g};
+  const size_t sbytes[1] = {(size_t)M * ldc * sizeof(float)};
+  return dysel_launch(ctx, kSgemmSig, U, f, mode, args, 2, sbytes, stream, rep);
+}
+
+dysel_status dysel_sgemm_variant(dysel_ctx *ctx, int variant_id, int M, int N, int K, float alpha, const float *d_A,
+                                 int lda, const float *d_B, int ldb, float beta, float *d_C, int ldc, void *stream) {
+  if (!ctx || variant_id < 0 || variant_id >= DYSEL_SGEMM_NVARIANTS) {
+    set_error(ctx, "dysel_sgemm_variant: invalid variant");
+    return DYSEL_ERR_INVALID;
+  }
+  DYSEL_TRY(check_args(ctx, M, N, K, d_A, lda, d_B, ldb, d_C, ldc));
+  if ((int64_t)M * N == 0) return DYSEL_OK;
+  SgemmArgs g{M, N, K, alpha, beta, d_A, lda, d_B, ldb, d_C, ldc};
+  const uint64_t U[3] = {(uint64_t)(N + 31) / 32, (uint64_t)(M + 31) / 32, 1};
+  void *args[2] = {d_C, &g};
+  // one full-grid batch copy of the variant: a slice over every granule
+  dysel_slice s;
+  memset(&s, 0, sizeof(s));
+  const uint32_t gg[3] = {4, 4, 1};
+  for (int d = 0; d < 3; ++d) {
+    s.g[d] = gg[d];
+    s.U[d] = U[d];
+    s.G[d] = (uint32_t)((U[d] + gg[d] - 1) / gg[d]);
+  }
+  s.granule_count = (uint64_t)s.G[0] * s.G[1] * s.G[2];
+  s.granule_stride = 1;
+  s.role = DYSEL_ROLE_BATCH;
+  s.variant = variant_id;
+  static dysel_variant_fn fns[DYSEL_SGEMM_NVARIANTS] = {sgemm_variant_fn<0>, sgemm_variant_fn<1>, sgemm_variant_fn<2>,
+                                                        sgemm_variant_fn<3>};
+  DYSEL_TRY(fns[variant_id](&s, args, stream, nullptr));
+  return check_launch(ctx, "sgemm full-grid variant");
+}
+
+}  // extern "C"

@@ -150,3 +150,19 @@ def test_selection_packed_argmin():
     assert S.select([c * units for c in costs]) == 1
     assert S.exhaustive_best([3.0, 1.0, 1.0]) == 1
     assert S.within(1.04, 1.0) and not S.within(1.06, 1.0)
+
+
+def test_partition_balanced_and_cover():
+    import numpy as np
+    from oracle import partition
+    from workloads import d4_powerlaw, identity
+    I = identity(256 * 40)
+    assert partition.partition_rows(I.row_ptr, 4) == [0, 2560, 5120, 7680, 10240]
+    A = d4_powerlaw(n=20000, lmax=1000)
+    for G in (2, 3, 8):
+        b = partition.partition_rows(A.row_ptr, G)
+        assert b[0] == 0 and b[-1] == A.n_rows and all(x <= y for x, y in zip(b, b[1:]))
+        assert all(x % 256 == 0 for x in b[:-1])
+        nz = np.diff(A.row_ptr.astype(np.int64)[b])
+        # each shard within one unit's nnz of the ideal share
+        assert np.abs(nz - A.nnz / G).max() <= A.row_ptr[-1] / A.n_rows * 256 * 4 + A.lengths().max()

@@ -1,0 +1,260 @@
+"""GPU parity of the SpMV path through the C ABI vs the fp64 oracle (SURVEY c-1,
+c-3, c-4, c-6, c-7, c-10)."""
+import numpy as np
+import pytest
+
+from gpu_helpers import oracle_spmv, spmv_err, to_dev, unit_slices, vec
+from oracle import formats, slice_plan
+from oracle.spmv import SPMV_TOL
+from workloads import (d1_bus, d3_fem, d4_powerlaw, d6_diag, identity, random_lengths_csr, small_int_csr,
+                       small_int_vector, uniform_f32, CSR)
+
+pytestmark = pytest.mark.gpu
+
+MATS = {
+    "d1": lambda: d1_bus(),
+    "ragged": lambda: random_lengths_csr(5003, 4000, 300, 17, empty_frac=0.1),
+    "d3small": lambda: d3_fem(grid=101),
+    "powerlaw": lambda: d4_powerlaw(n=60_000, lmax=4000),
+    "diag": lambda: d6_diag(n=70_000),
+}
+
+
+@pytest.fixture(scope="module")
+def ctx(gpu):
+    from paper_conf_asplos_changkh16_b200 import dysel
+    c = dysel.Context(0)
+    yield c
+    c.close()
+
+
+@pytest.fixture(scope="module")
+def D():
+    from paper_conf_asplos_changkh16_b200 import dysel
+    return dysel
+
+
+def prepared(ctx, A, default=1):
+    import torch
+    rp, col, val = to_dev(A)
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=default)
+    torch.cuda.synchronize()
+    return plan
+
+
+@pytest.mark.parametrize("name", list(MATS))
+def test_formats_bit_exact(ctx, name):
+    A = MATS[name]()
+    plan = prepared(ctx, A)
+    if formats.ell_applicable(A.row_ptr):
+        W, npad, ec, ev = formats.csr_to_ell_fast(A.row_ptr, A.col, A.val)
+        assert plan.info.ell_width == W
+        assert np.array_equal(plan.array("ell_col"), ec)
+        assert np.array_equal(plan.array("ell_val").view(np.uint32), ev.view(np.uint32))
+    else:
+        assert 2 not in plan.variant_ids            # A-15
+    j = formats.csr_to_block_jds_fast(A.row_ptr, A.col, A.val)
+    for k in ("perm", "blk_off", "jd_off", "jd_ptr", "jds_col"):
+        assert np.array_equal(plan.array(k), j[k]), k
+    assert np.array_equal(plan.array("jds_val").view(np.uint32), j["jds_val"].view(np.uint32))
+    lens = A.lengths()
+    assert np.array_equal(plan.array("jds_len"), lens[j["perm"]])
+    assert plan.info.uniform == int(formats.uniform_rows(A.row_ptr))
+    plan.destroy()
+
+
+@pytest.mark.parametrize("name", list(MATS))
+def test_variants_parity(ctx, D, name):
+    import torch
+    A = MATS[name]()
+    x = uniform_f32(99, A.n_cols)
+    plan = prepared(ctx, A)
+    xd = vec(x)
+    outs = {}
+    for v in plan.variant_ids:
+        y = torch.full((A.n_rows,), float("nan"), device="cuda")
+        ctx.spmv_variant(plan, v, xd, y)
+        torch.cuda.synchronize()
+        assert spmv_err(A, x, y) <= SPMV_TOL, D.SPMV_NAMES[v]
+        outs[v] = y.cpu().numpy()
+    # CSR-S, ELL and JDS accumulate in CSR order with fmaf: bit-identical
+    ref = outs[0].view(np.uint32)
+    for v in (2, 3):
+        if v in outs:
+            assert np.array_equal(outs[v].view(np.uint32), ref), D.SPMV_NAMES[v]
+    plan.destroy()
+
+
+@pytest.mark.parametrize("name", ["d1", "ragged", "powerlaw"])
+def test_small_integer_bit_exact(ctx, name):
+    import torch
+    A = small_int_csr(MATS[name](), 5)
+    x = small_int_vector(A.n_cols, 6)
+    ys, _ = oracle_spmv(A, x)
+    plan = prepared(ctx, A)
+    for v in plan.variant_ids:
+        y = torch.empty(A.n_rows, device="cuda")
+        ctx.spmv_variant(plan, v, vec(x), y)
+        assert np.array_equal(y.cpu().numpy().astype(np.float64), ys), v
+    plan.destroy()
+
+
+def test_identity_and_diagonal_exact(ctx):
+    import torch
+    I = identity(3001)
+    x = uniform_f32(1, 3001)
+    plan = prepared(ctx, I)
+    for v in plan.variant_ids:
+        y = torch.empty(3001, device="cuda")
+        ctx.spmv_variant(plan, v, vec(x), y)
+        assert np.array_equal(y.cpu().numpy(), x)
+    Dg = d6_diag(n=10_000)
+    x = uniform_f32(2, 10_000)
+    plan2 = prepared(ctx, Dg)
+    expect = (Dg.val * x).astype(np.float32)      # one product, fl32(d_i x_i)
+    for v in plan2.variant_ids:
+        y = torch.empty(10_000, device="cuda")
+        ctx.spmv_variant(plan2, v, vec(x), y)
+        assert np.array_equal(y.cpu().numpy(), expect)
+
+
+MODES = ["fully_sync", "fully_async", "hybrid_sync", "hybrid_async", "fully_sync_host", "fully_async_host",
+         "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles"]
+
+
+def mode_bits(D, m):
+    b = D.FORCE_PROFILE
+    b |= D.HYBRID if m.startswith("hybrid") else D.FULLY
+    b |= D.ASYNC if "async" in m else D.SYNC
+    b |= D.HOST_ORCH if m.endswith("host") else 0
+    b |= D.CONTIGUOUS if "contig" in m else 0
+    b |= D.SCORE_CYCLES if "cycles" in m else 0
+    return b
+
+
+@pytest.mark.parametrize("m", MODES)
+@pytest.mark.parametrize("name", ["ragged", "powerlaw", "d3small"])
+def test_dysel_composition(ctx, D, name, m):
+    """c-6: y_dysel restricted to unit u == y_full[v(u)] restricted to u, bitwise;
+    every unit productively computed exactly once; parity vs oracle."""
+    import torch
+    A = MATS[name]()
+    x = uniform_f32(7, A.n_cols)
+    plan = prepared(ctx, A, default=0)
+    xd = vec(x)
+    full = {}
+    for v in plan.variant_ids:
+        y = torch.empty(A.n_rows, device="cuda")
+        ctx.spmv_variant(plan, v, xd, y)
+        full[v] = y.cpu().numpy().view(np.uint32)
+    mode = mode_bits(D, m)
+    y = torch.full((A.n_rows,), float("nan"), device="cuda")
+    rep = ctx.spmv(plan, xd, y, f=0.1, mode=mode, report=True, unit_map=True)
+    torch.cuda.synchronize()
+    assert rep["profiled"]
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    yy = y.cpu().numpy().view(np.uint32)
+    uv = rep["unit_variant"]
+    K = len(plan.variant_ids)
+    # oracle plan: same c, same granule count
+    p = slice_plan.plan((plan.n_units,), [(1,)] * K, 0.1, ctx.n_sm, plan.variant_ids.index(0), mode,
+                        [0 if plan.info.uniform else slice_plan.V_NONUNIFORM] * K)
+    assert rep["c"] == p.c and rep["n_granules"] == p.Gn
+    sel = rep["selected"]
+    assert sel in plan.variant_ids
+    for u, (r0, r1) in enumerate(unit_slices(A.n_rows)):
+        v = uv[u]
+        assert v in full, (u, v)
+        assert np.array_equal(yy[r0:r1], full[v][r0:r1]), (u, v)
+    # profiling granules carry the ticket's variant, remainder the selection (sync)
+    pool = plan.variant_ids
+    owner = slice_plan.productive_cover(p, pool.index(sel))
+    for j in range(p.Gn):
+        if j < len(owner) and (j < p.c * (K if p.mode == slice_plan.FULLY else 1)):
+            assert uv[j] == pool[owner[j]], j
+        elif "async" not in m:
+            assert uv[j] == sel, j
+    plan.destroy()
+
+
+def test_no_profile_and_cache(ctx, D):
+    import torch
+    A = MATS["ragged"]()
+    x = uniform_f32(8, A.n_cols)
+    plan = prepared(ctx, A, default=3)
+    xd = vec(x)
+    ref = torch.empty(A.n_rows, device="cuda")
+    ctx.spmv_variant(plan, 3, xd, ref)
+    y = torch.empty(A.n_rows, device="cuda")
+    rep = ctx.spmv(plan, xd, y, mode=D.NO_PROFILE, report=True)
+    assert not rep["profiled"] and rep["selected"] == 3
+    assert torch.equal(y.view(torch.int32), ref.view(torch.int32))       # P:L868-871 "0 profiled blocks"
+    rep = ctx.spmv(plan, xd, y, f=0.2, mode=D.FULLY | D.SYNC | D.FORCE_PROFILE, report=True)
+    sel = rep["selected"]
+    ctx.spmv_variant(plan, sel, xd, ref)
+    rep2 = ctx.spmv(plan, xd, y, mode=D.NO_PROFILE, report=True)   # activation flag: reuse the selection
+    assert rep2["selected"] == sel
+    assert torch.equal(y.view(torch.int32), ref.view(torch.int32))
+    plan.destroy()
+
+
+def test_small_workload_deactivated(ctx, D):
+    import torch
+    A = MATS["d1"]()        # 5 units < 128
+    x = uniform_f32(9, A.n_cols)
+    plan = prepared(ctx, A, default=1)
+    y = torch.empty(A.n_rows, device="cuda")
+    rep = ctx.spmv(plan, vec(x), y, f=0.5, mode=D.DEFAULT_MODE, report=True)
+    assert not rep["profiled"] and rep["selected"] == 1
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    rep = ctx.spmv(plan, vec(x), y, f=0.5, mode=D.DEFAULT_MODE | D.FORCE_PROFILE, report=True)
+    assert rep["profiled"]
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    plan.destroy()
+
+
+def test_edge_cases(ctx, D):
+    import torch
+    # all rows empty: y := 0
+    n = 1000
+    E = CSR(n, n, np.zeros(n + 1, np.int32), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    plan = prepared(ctx, E)
+    y = torch.full((n,), 5.0, device="cuda")
+    ctx.spmv(plan, vec(np.ones(n)), y, f=0.5, mode=D.FORCE_PROFILE | D.FULLY)
+    assert torch.count_nonzero(y).item() == 0
+    # single row, single column
+    S1 = CSR(1, 1, np.array([0, 1], np.int32), np.array([0], np.int32), np.array([2.5], np.float32))
+    plan = prepared(ctx, S1)
+    y = torch.empty(1, device="cuda")
+    for v in plan.variant_ids:
+        ctx.spmv_variant(plan, v, vec(np.array([4.0])), y)
+        assert y.item() == 10.0
+    # invalid arguments are rejected, never crash
+    with pytest.raises(D.DyselError):
+        ctx.spmv(plan, vec(np.array([1.0])), y, f=2.0)
+    with pytest.raises(D.DyselError) as e:
+        ctx.spmv(plan, vec(np.array([1.0])), y, mode=D.SWAP | D.ASYNC)
+    assert e.value.status == D.ERR_UNSUPPORTED
+
+
+def test_long_rows_vector_path(ctx):
+    """Rows >= 128 entries take CSR-V's 128-bit path (head / body / tail)."""
+    import torch
+    L = np.array([0, 1, 127, 128, 129, 131, 255, 256, 257, 1000, 4093, 5000] * 30)
+    A = d4_powerlaw(n=2, lmax=2)   # placeholder for type
+    from workloads import csr_from_lengths
+    A = csr_from_lengths(L, 6000, 3, 4)
+    x = uniform_f32(5, 6000)
+    plan = prepared(ctx, A)
+    y = torch.empty(A.n_rows, device="cuda")
+    ctx.spmv_variant(plan, 1, vec(x), y)
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    # unaligned base pointers disable the vector body but keep parity
+    rp, col, val = to_dev(A)
+    col2 = torch.empty(col.numel() + 1, dtype=torch.int32, device="cuda")[1:]
+    val2 = torch.empty(val.numel() + 1, dtype=torch.float32, device="cuda")[1:]
+    col2.copy_(col)
+    val2.copy_(val)
+    plan2 = ctx.spmv_prepare(rp, col2, val2, A.n_cols)
+    ctx.spmv_variant(plan2, 1, vec(x), y)
+    assert spmv_err(A, x, y) <= SPMV_TOL
