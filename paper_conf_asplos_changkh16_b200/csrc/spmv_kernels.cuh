@@ -112,13 +112,13 @@ __device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, fl
 __device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, int lane, uint64_t ps,
                                                uint64_t px) {
   float s = 0.0f;
-  int a = A.vec_ok ? ((b + 3) & ~3) : e;   // no vector body when unaligned
-  if (a > e) a = e;
+  // unaligned base pointers: no head / vector body, everything in the tail loop
+  const int a = A.vec_ok ? min((b + 3) & ~3, e) : b;
   if (b + lane < a) {
     const int k = b + lane;
     s = __fmaf_rn(ld_stream(A.val + k, ps), ld_x(A.x + ld_stream(A.col + k, ps), px), s);
   }
-  const int body_end = a + ((e - a) & ~3);
+  const int body_end = A.vec_ok ? a + ((e - a) & ~3) : b;
   int base = a;
   for (; base + 256 <= body_end; base += 256) {    // two 128-entry chunks in flight
     const int k0 = base + 4 * lane, k1 = k0 + 128;
@@ -214,17 +214,24 @@ __device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, float *__
   const float *vp = A.ell_val + r;
   float s = 0.0f;
   int k = 0;
+  bool live = true;   // pads (col = -1) only follow a row's entries
   for (; k + 2 <= A.ell_W; k += 2) {
     const int c0 = ld_stream(cp + (int64_t)k * A.n_pad, ps);
     const int c1 = ld_stream(cp + (int64_t)(k + 1) * A.n_pad, ps);
     const float v0 = ld_stream(vp + (int64_t)k * A.n_pad, ps);
     const float v1 = ld_stream(vp + (int64_t)(k + 1) * A.n_pad, ps);
-    if (c0 < 0) break;
+    if (c0 < 0) {
+      live = false;
+      break;
+    }
     s = __fmaf_rn(v0, ld_x(A.x + c0, px), s);
-    if (c1 < 0) break;
+    if (c1 < 0) {
+      live = false;
+      break;
+    }
     s = __fmaf_rn(v1, ld_x(A.x + c1, px), s);
   }
-  if (k < A.ell_W) {
+  if (live && k < A.ell_W) {
     const int c0 = ld_stream(cp + (int64_t)k * A.n_pad, ps);
     if (c0 >= 0) s = __fmaf_rn(ld_stream(vp + (int64_t)k * A.n_pad, ps), ld_x(A.x + c0, px), s);
   }

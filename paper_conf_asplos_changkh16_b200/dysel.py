@@ -9,6 +9,7 @@ from __future__ import annotations
 
 import ctypes
 import os
+import weakref
 
 import torch
 
@@ -189,9 +190,10 @@ class SpmvPlan:
         return out
 
     def destroy(self):
-        if self.handle:
+        # a plan must die before its context (it unregisters from it)
+        if self.handle and self.ctx is not None and self.ctx.h:
             dysel_spmv_plan_destroy(self.handle)
-            self.handle = None
+        self.handle = None
 
     def __del__(self):
         try:
@@ -211,6 +213,7 @@ class Context:
             raise DyselError(st, "dysel_create failed")
         self.h = h
         self.device = device
+        self._plans = weakref.WeakSet()
         n_sm, tick, l2 = c_int(), c_u64(), c_u64()
         dysel_device_info(h, ctypes.byref(n_sm), ctypes.byref(tick), ctypes.byref(l2))
         self.n_sm, self.globaltimer_tick_ns, self.l2_bytes = n_sm.value, tick.value, l2.value
@@ -220,9 +223,17 @@ class Context:
             raise DyselError(st, dysel_last_error(self.h).decode())
 
     def close(self):
+        for p in list(self._plans):
+            p.destroy()
         if self.h:
             dysel_destroy(self.h)
             self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
     def kernel_launches(self) -> int:
         return int(dysel_kernel_launches(self.h))
@@ -236,7 +247,9 @@ class Context:
         h = ctypes.c_void_p()
         self._check(dysel_spmv_prepare(self.h, n, int(n_cols), nnz, _ptr(row_ptr), _ptr(col), _ptr(val),
                                        formats, default, _stream(stream), ctypes.byref(h)))
-        return SpmvPlan(self, h, (row_ptr, col, val))
+        plan = SpmvPlan(self, h, (row_ptr, col, val))
+        self._plans.add(plan)
+        return plan
 
     def spmv(self, plan, x, y, f=0.02, mode=DEFAULT_MODE, report=False, unit_map=False, stream=None):
         rep, keep, uv = (_make_report(plan.n_units if unit_map else 0) if report else (None, None, None))

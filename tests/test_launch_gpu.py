@@ -64,7 +64,11 @@ def test_known_cost_selection(ctx, D, m):
 
 
 def test_async_eager_starts_with_default(ctx, D):
-    rep, out = run(ctx, D, "spin.eager", 3000, D.FULLY | D.ASYNC | D.HOST_ORCH, f=0.05, default=3)
+    # Profiling slow enough (tens of us) that the host poll loop can launch
+    # eager chunks before it finishes; with us-scale profiling the paper saw
+    # "few or even zero eager dispatches".
+    slow = [c * 50 for c in COSTS]
+    rep, out = run(ctx, D, "spin.eager", 3000, D.FULLY | D.ASYNC | D.HOST_ORCH, f=0.05, costs=slow, default=3)
     assert rep["selected"] == 1
     assert rep["eager_units"] > 0                 # eager chunks were launched
     eager = out[4 * rep["c"]: 4 * rep["c"] + rep["eager_units"]]
