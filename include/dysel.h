@@ -81,7 +81,13 @@ const char *dysel_status_str(dysel_status s);
 #define DYSEL_HOST_ORCH 16u     /* paper-faithful host orchestration: streams + host sync / polling */
 #define DYSEL_FORCE_PROFILE 32u /* ignore the small-workload deactivation (< 128 CTAs); ablation */
 #define DYSEL_CONTIGUOUS 64u    /* fully mode: contiguous per-variant slices instead of interleaved granules (A-24) */
-#define DYSEL_SCORE_CYCLES 128u /* score = sum of per-CTA clock64 cycles / units instead of %globaltimer makespan (A-6) */
+#define DYSEL_SCORE_CYCLES 128u /* score = sum of per-CTA clock64 cycles / units (A-6) */
+#define DYSEL_SCORE_MAKESPAN 256u /* score = latest CTA end - earliest CTA start (%globaltimer), Fig. 7b */
+#define DYSEL_NO_TAIL 512u      /* SpMV device path: run the remainder inside the dispatcher (no CDP2 tail launch) */
+#define DYSEL_NO_ABORT 1024u    /* SpMV device path: never stop dominated sandbox units early */
+/* Default score: generic launcher = makespan (variants are separate concurrent
+ * grids, Fig. 7b); SpMV dispatcher = mean per-unit busy time (%globaltimer end -
+ * start of each profiled unit; all variants share one launch and occupancy). */
 #define DYSEL_DEFAULT_MODE (DYSEL_FULLY | DYSEL_ASYNC)
 
 /* variant flags (replace the compiler analyses, A-10/A-11) */
@@ -195,6 +201,9 @@ typedef struct {
   uint64_t makespan_ns[DYSEL_MAX_VARIANTS];
   uint64_t units[DYSEL_MAX_VARIANTS];
   uint64_t cycles[DYSEL_MAX_VARIANTS];
+  uint64_t busy_ns[DYSEL_MAX_VARIANTS];   /* sum of per-unit busy time (SpMV dispatcher) */
+  uint64_t aborted[DYSEL_MAX_VARIANTS];   /* sandbox units stopped / skipped by dominance */
+  uint64_t tail_units;      /* remainder units run by the tail-launched plain kernel */
   uint64_t eager_units;     /* remainder units run before the final selection (async) */
   uint64_t host_ns;         /* host time inside the call */
   dysel_slice_rec *slices;  /* optional caller array */
@@ -228,9 +237,11 @@ dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key); /* NULL key
  * y = A x (overwrite), fp32 CSR input (SHOC spmv-csr / Parboil spmv-jds,
  * P:L1128-1131).  Unit = 256 consecutive original rows.
  * Built-in variants (ids): 0 CSR-scalar (thread per row), 1 CSR-vector (warp
- * per row), 2 ELL (column-major, padded), 3 block-local JDS (A-14). */
+ * per row), 2 ELL (column-major, padded), 3 block-local JDS (A-14), 4 CSR-W
+ * (warp-streaming CSR with a warp-level segmented reduction; B200 addition). */
 enum { DYSEL_SPMV_CSR_SCALAR = 0, DYSEL_SPMV_CSR_VECTOR = 1, DYSEL_SPMV_ELL = 2, DYSEL_SPMV_JDS = 3,
-       DYSEL_SPMV_NVARIANTS = 4 };
+       DYSEL_SPMV_CSR_STREAM = 4, DYSEL_SPMV_NVARIANTS = 5 };
+#define DYSEL_FMT_STREAM 4u   /* include CSR-W in the pool (reads the CSR arrays directly) */
 #define DYSEL_FMT_ELL 1u
 #define DYSEL_FMT_JDS 2u
 
@@ -271,7 +282,11 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *plan);
  * Device path (default): ONE persistent launch; tickets claim granules, the
  * profiling tickets first; the last profiling CTA publishes the selection on
  * the device; sync mode spins on it, async mode reads the best so far
- * (SURVEY §8a device protocol).  With DYSEL_HOST_ORCH: one kernel per variant
+ * (SURVEY §8a device protocol); hybrid sandbox units of a provably losing
+ * variant stop early (dominance, unless DYSEL_NO_ABORT), and once the
+ * selection is published the last profiling CTA hands every unclaimed unit to
+ * the winner's plain kernel with a CDP2 tail launch (unless DYSEL_NO_TAIL).
+ * With DYSEL_HOST_ORCH: one kernel per variant
  * on forked streams, host reads the selection, then the remainder kernel
  * (paper-faithful).  Mode AUTO uses the plan's uniformity flag. */
 dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,

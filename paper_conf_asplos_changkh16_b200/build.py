@@ -33,12 +33,15 @@ def _deps():
     return max(os.path.getmtime(h) for h in hdrs)
 
 
+RDC = {"spmv.cu"}   # device-side (CDP2 tail) launches need relocatable device code
+
+
 def _compile(src, verbose):
     obj = os.path.join(OBJ, src.replace(".cu", ".o"))
     path = os.path.join(CSRC, src)
     if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(path), _deps()):
         return obj, ""
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", path, "-o", obj]
+    cmd = [NVCC, *ARCH, *FLAGS, *(["-rdc=true"] if src in RDC else []), "-c", path, "-o", obj]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -57,7 +60,13 @@ def build(verbose: bool = False) -> str:
             if log:
                 sys.stderr.write(log)
     if not os.path.exists(LIB) or os.path.getmtime(LIB) < max(os.path.getmtime(o) for o in objs):
-        cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, "-ldl"]
+        rdc = [o for o in objs if os.path.basename(o).replace(".o", ".cu") in RDC]
+        dlink = os.path.join(OBJ, "dlink.o")
+        r = subprocess.run([NVCC, *ARCH, "-Xcompiler", "-fPIC", "-dlink", *rdc, "-o", dlink, "-lcudadevrt"],
+                           capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"device link failed:\n{r.stderr}")
+        cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, dlink, "-lcudadevrt", "-ldl"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")

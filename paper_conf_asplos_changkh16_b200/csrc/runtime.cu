@@ -258,9 +258,11 @@ static void fill_report_common(dysel_report *rep, const Plan &p, int mode_used, 
   rep->c = p.c;
   rep->n_granules = p.Gn;
   rep->eager_units = 0;
+  rep->tail_units = 0;
   rep->n_slices = 0;
   for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v) {
     rep->score[v] = rep->makespan_ns[v] = rep->units[v] = rep->cycles[v] = 0;
+    rep->busy_ns[v] = rep->aborted[v] = 0;
   }
 }
 

@@ -28,6 +28,13 @@
 
 namespace dysel {
 
+// Scores (reading A-6): the dispatcher scores a variant by the
+// mean busy time of its profiled units (sum over its units of the CTA's
+// %globaltimer end - start, / units).  All variants run inside the same
+// persistent launch with the same occupancy, so per-unit latency ranks their
+// throughput; the paper's makespan (first start .. last end, Fig. 7b) is
+// polluted here by ticket queueing, and stays available (DYSEL_SCORE_MAKESPAN)
+// as does the clock64 sum (DYSEL_SCORE_CYCLES).
 struct SpmvState {
   uint32_t ticket;
   uint32_t exited;
@@ -35,8 +42,14 @@ struct SpmvState {
   uint32_t release;
   uint64_t best;          // (score << 8) | pool variant, 0xff = none yet
   uint64_t sel;           // final packed selection, ~0 until published
-  uint64_t eager_units;   // remainder units started before `release`
+  uint64_t eager_units;   // remainder units started before the selection
+  uint64_t best_total;    // min over completed variants of their busy sum (ns)
+  uint64_t tail_begin;    // first unit handed to the tail launch (or ~0)
   uint32_t ctas_done[DYSEL_MAX_VARIANTS];
+  uint32_t dominated[DYSEL_MAX_VARIANTS];
+  uint64_t busy[DYSEL_MAX_VARIANTS];      // sum of unit durations (ns), completed units
+  uint64_t lb[DYSEL_MAX_VARIANTS];        // lower bound of the final busy sum (ns)
+  uint64_t aborted[DYSEL_MAX_VARIANTS];   // sandbox units stopped or skipped by dominance
   dysel_timer_slot slot[DYSEL_MAX_VARIANTS];
 };
 struct SpmvStateBlock {
@@ -49,8 +62,10 @@ struct DispatchParams {
   uint32_t c;            // profiling units per variant
   uint32_t n_tickets;
   uint32_t n_units;
-  uint32_t hybrid, async, contiguous, score_cycles;
+  uint32_t hybrid, async, contiguous, score_mode;   // score_mode 0 busy, 1 cycles, 2 makespan
   uint32_t def;          // pool index of default variant
+  uint32_t tail;         // hand the remainder to the winner's plain kernel (CDP2 tail launch)
+  uint32_t abort;        // dominance abort of hybrid sandbox units
   int32_t vids[DYSEL_SPMV_NVARIANTS];
   float *sandbox;        // (K-1) * c * 256 floats (hybrid)
   uint8_t *unit_variant; // optional debug map (pool index per unit)
@@ -64,8 +79,14 @@ __device__ __forceinline__ void reset_state(SpmvState *s) {
   s->best = (((1ull << 56) - 1) << 8) | 0xffull;
   s->sel = ~0ull;
   s->eager_units = 0;
+  s->best_total = ~0ull;
+  s->tail_begin = ~0ull;
   for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v) {
     s->ctas_done[v] = 0;
+    s->dominated[v] = 0;
+    s->busy[v] = 0;
+    s->lb[v] = 0;
+    s->aborted[v] = 0;
     s->slot[v].t_start_min = ~0ull;
     s->slot[v].t_end_max = 0;
     s->slot[v].units = 0;
@@ -85,6 +106,11 @@ __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
   uint64_t v;
   asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -94,20 +120,86 @@ __device__ __forceinline__ void st_release_u32(uint32_t *p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
+// Dominance abort for hybrid sandbox units: every
+// ~kPollNs one thread of the CTA adds the time elapsed since the last report
+// to lb[v].  lb[v] only ever sums time that variant v's units have really
+// spent, so it is a lower bound of v's final busy sum; once it exceeds the
+// busy sum of a COMPLETED variant (best_total), v can no longer be selected
+// (all variants profile the same c units in hybrid mode), so its sandbox work
+// stops and its remaining sandbox units are skipped.  The selection is the one
+// running them to completion would give.
+constexpr uint64_t kPollNs = 2000;
+struct SandboxPoll {
+  static constexpr bool active = true;
+  unsigned long long *s_last;   // smem: last report time
+  volatile int *s_abort;        // smem
+  unsigned long long *lb;
+  const uint64_t *best_total;
+  uint32_t *dominated;
+  __device__ __forceinline__ bool operator()() const {
+    if (*s_abort) return true;
+    const unsigned long long now = dysel_globaltimer();
+    const unsigned long long last = *(volatile unsigned long long *)s_last;
+    if (now - last < kPollNs) return false;
+    if (atomicCAS(s_last, last, now) != last) return *s_abort != 0;   // another thread reports
+    const unsigned long long l = atomicAdd(lb, now - last) + (now - last);
+    if (l > ld_relaxed_u64(best_total) || ld_relaxed_u32(dominated) != 0) {
+      *s_abort = 1;
+      atomicExch(dominated, 1u);
+      return true;
+    }
+    return false;
+  }
+};
+
 constexpr int kPersistMinBlocks = 4;
+
+// resident CTAs per SM each plain variant kernel is compiled for (register cap)
+constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 6};
+
+template <int VID>
+__global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
+    spmv_slice_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s, uint8_t *uv);
+
+__device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, uint64_t n_units, uint8_t *uv) {
+  dysel_slice s;
+  memset(&s, 0, sizeof(s));
+  s.granule_begin = u0;
+  s.granule_count = n_units - u0;
+  s.granule_stride = 1;
+  s.g[0] = s.g[1] = s.g[2] = 1;
+  s.G[0] = (uint32_t)n_units;
+  s.G[1] = s.G[2] = 1;
+  s.U[0] = n_units;
+  s.U[1] = s.U[2] = 1;
+  s.role = DYSEL_ROLE_BATCH;
+  s.variant = vid;
+  const unsigned grid = (unsigned)(n_units - u0);
+  switch (vid) {
+    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
+    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
+    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
+    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
+    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
+  }
+}
 
 __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
     spmv_persistent_kernel(SpmvDev A, float *__restrict__ y, SpmvStateBlock *sb, DispatchParams p) {
   __shared__ uint32_t s_ticket;
   __shared__ int32_t s_v;
+  __shared__ unsigned long long s_last;
+  __shared__ int s_abort;
   __shared__ dysel_prof_smem psm;
   SpmvState *st = &sb->live;
   const uint32_t tid = threadIdx.x;
   const uint32_t P = p.K * p.c;
+  // sync + tail: only the profiling tickets run here, the tail kernel takes [P, n)
+  const uint32_t limit = (p.tail && !p.async) ? P : p.n_tickets;
   if (tid == 0) s_ticket = atomicAdd(&st->ticket, 1u);
   __syncthreads();
   uint32_t t = s_ticket;
-  while (t < p.n_tickets) {
+  while (t < limit) {
     uint32_t next = 0;
     if (tid == 0) next = atomicAdd(&st->ticket, 1u);   // prefetch: latency hidden by the unit's work
     if (t < P) {
@@ -125,16 +217,33 @@ __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
         j = t;
         pv = t % p.K;
       }
+      const bool sandbox = !productive;
+      bool skipped = false;
+      if (tid == 0) {
+        s_abort = 0;
+        s_last = dysel_globaltimer();
+        skipped = sandbox && p.abort && ld_relaxed_u32(&st->dominated[pv]) != 0;
+        s_v = skipped ? 1 : 0;
+      }
+      __syncthreads();
+      skipped = s_v != 0;
       float *out = productive ? y + (size_t)j * kUnitRows
                               : p.sandbox + ((size_t)(pv < p.def ? pv : pv - 1) * p.c + j) * kUnitRows;
-      if ((tid & 31) == 0) {
-        psm.c0[tid >> 5] = dysel_clock64();
-        psm.t0[tid >> 5] = dysel_globaltimer();
-      }
-      run_unit_dyn(p.vids[pv], A, j, out);
-      if ((tid & 31) == 0) {
-        psm.t1[tid >> 5] = dysel_globaltimer();
-        psm.c1[tid >> 5] = dysel_clock64();
+      if (!skipped) {
+        if ((tid & 31) == 0) {
+          psm.c0[tid >> 5] = dysel_clock64();
+          psm.t0[tid >> 5] = dysel_globaltimer();
+        }
+        if (sandbox && p.abort) {
+          SandboxPoll poll{&s_last, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total, &st->dominated[pv]};
+          run_unit_dyn(p.vids[pv], A, j, out, poll);
+        } else {
+          run_unit_dyn(p.vids[pv], A, j, out, NoPoll());
+        }
+        if ((tid & 31) == 0) {
+          psm.t1[tid >> 5] = dysel_globaltimer();
+          psm.c1[tid >> 5] = dysel_clock64();
+        }
       }
       __syncthreads();
       if (tid < 32) {   // warp-shuffle reduction of the per-warp samples
@@ -149,11 +258,17 @@ __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
         }
         if (tid == 0) {
           dysel_timer_slot *slot = &st->slot[pv];
-          atomicMin((unsigned long long *)&slot->t_start_min, t0);
-          atomicMax((unsigned long long *)&slot->t_end_max, t1);
-          atomicAdd((unsigned long long *)&slot->cycles, c1 - c0);
+          const bool stopped = skipped || s_abort;
+          if (!skipped) {
+            atomicMin((unsigned long long *)&slot->t_start_min, t0);
+            atomicMax((unsigned long long *)&slot->t_end_max, t1);
+            atomicAdd((unsigned long long *)&slot->cycles, c1 - c0);
+            atomicAdd((unsigned long long *)&st->busy[pv], t1 - t0);
+            atomicAdd((unsigned long long *)&st->lb[pv], t1 - s_last);   // rest of this unit's time
+          }
+          if (stopped) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
           atomicAdd((unsigned long long *)&slot->units, 1ull);
-          if (productive && p.unit_variant) p.unit_variant[j] = (uint8_t)pv;
+          if (productive && p.unit_variant) p.unit_variant[j] = (uint8_t)p.vids[pv];
           __threadfence();
           const uint32_t done = atomicAdd(&st->ctas_done[pv], 1u) + 1u;
           if (done == p.c) {   // variant complete: score, packed atomicMin (A-7, A-8)
@@ -161,17 +276,29 @@ __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
             const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
             const unsigned long long b = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
             const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
-            unsigned long long score = p.score_cycles ? cy / p.c : (b - a);
-            if (score > (1ull << 56) - 1) score = (1ull << 56) - 1;
+            const unsigned long long bz = atomicAdd((unsigned long long *)&st->busy[pv], 0ull);
+            const bool dom = ld_relaxed_u32(&st->dominated[pv]) != 0;
+            unsigned long long score = p.score_mode == 1 ? cy / p.c : (p.score_mode == 2 ? b - a : bz / p.c);
+            if (dom || score > (1ull << 56) - 1) score = (1ull << 56) - 1;
+            if (!dom) atomicMin((unsigned long long *)&st->best_total, bz);
             atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
             __threadfence();
             const uint32_t vd = atomicAdd(&st->variants_done, 1u) + 1u;
-            if (vd == p.K) {   // last variant: publish and release the spinners
+            if (vd == p.K) {   // last variant: publish, hand off the remainder
               __threadfence();
               const unsigned long long fin = atomicAdd((unsigned long long *)&st->best, 0ull);
               atomicExch((unsigned long long *)&st->sel, fin);
               __threadfence();
               st_release_u32(&st->release, 1u);
+              if (p.tail) {
+                // grab every ticket not yet claimed; dispatcher CTAs then exit
+                const uint32_t old = p.async ? atomicAdd(&st->ticket, 1u << 30) : P;
+                const uint64_t u0 = p.hybrid ? (uint64_t)old - (uint64_t)(p.K - 1) * p.c : old;
+                if (old < p.n_tickets && u0 < p.n_units) {
+                  st->tail_begin = u0;
+                  tail_launch(p.vids[fin & 0xff], A, y, u0, p.n_units, p.unit_variant);
+                }
+              }
             }
           }
         }
@@ -196,10 +323,10 @@ __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
           if (ld_acquire_u32(&st->release) == 0) atomicAdd((unsigned long long *)&st->eager_units, 1ull);
         }
         s_v = v;
-        if (p.unit_variant) p.unit_variant[j] = (uint8_t)v;
+        if (p.unit_variant) p.unit_variant[j] = (uint8_t)p.vids[v];
       }
       __syncthreads();
-      run_unit_dyn(p.vids[s_v], A, j, y + (size_t)j * kUnitRows);
+      run_unit_dyn(p.vids[s_v], A, j, y + (size_t)j * kUnitRows, NoPoll());
     }
     __syncthreads();
     if (tid == 0) s_ticket = next;
@@ -220,8 +347,14 @@ __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
       r->best = vs->best;
       r->sel = vs->sel;
       r->eager_units = vs->eager_units;
+      r->best_total = vs->best_total;
+      r->tail_begin = vs->tail_begin;
       for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v) {
         r->ctas_done[v] = vs->ctas_done[v];
+        r->dominated[v] = vs->dominated[v];
+        r->busy[v] = vs->busy[v];
+        r->lb[v] = vs->lb[v];
+        r->aborted[v] = vs->aborted[v];
         r->slot[v].t_start_min = vs->slot[v].t_start_min;
         r->slot[v].t_end_max = vs->slot[v].t_end_max;
         r->slot[v].units = vs->slot[v].units;
@@ -233,15 +366,18 @@ __global__ void __launch_bounds__(kUnitRows, kPersistMinBlocks)
   }
 }
 
-// Plain full-grid / slice kernel of one variant (also the host path's
-// profiling, eager and batch copies; dysel_device.cuh handles timing/gating).
+// Plain full-grid / slice kernel of one variant: the exhaustive oracle's pure
+// version, the activation-flag-off path, the tail-launched remainder and the
+// host path's profiling / eager / batch copies (dysel_device.cuh timing).
 template <int VID>
-__global__ void __launch_bounds__(kUnitRows) spmv_slice_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s) {
+__global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
+    spmv_slice_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s, uint8_t *uv) {
   __shared__ dysel_prof_smem psm;
   if (!dysel_gate_open(s)) return;
   dysel_prof_begin(s, psm);
   const uint32_t j = (uint32_t)(s.granule_begin + (uint64_t)blockIdx.x * s.granule_stride);
   run_unit<VID>(A, j, y + (size_t)j * kUnitRows);
+  if (uv && threadIdx.x == 0) uv[j] = (uint8_t)VID;
   dysel_prof_end(s, psm, 1u);
 }
 
@@ -372,13 +508,14 @@ static dysel_status spmv_variant_fn(const dysel_slice *s, void *const *args, voi
   if (s->granule_count == 0) return DYSEL_OK;
   SpmvDev A = pl->dev;
   A.x = (const float *)args[1];
-  spmv_slice_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(A, (float *)args[0], *s);
+  spmv_slice_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(A, (float *)args[0], *s,
+                                                                                            nullptr);
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
 
-static dysel_variant_fn kVariantFns[DYSEL_SPMV_NVARIANTS] = {spmv_variant_fn<0>, spmv_variant_fn<1>,
-                                                             spmv_variant_fn<2>, spmv_variant_fn<3>};
-static const char *kVariantNames[DYSEL_SPMV_NVARIANTS] = {"csr_scalar", "csr_vector", "ell", "jds"};
+static dysel_variant_fn kVariantFns[DYSEL_SPMV_NVARIANTS] = {spmv_variant_fn<0>, spmv_variant_fn<1>, spmv_variant_fn<2>,
+                                                             spmv_variant_fn<3>, spmv_variant_fn<4>};
+static const char *kVariantNames[DYSEL_SPMV_NVARIANTS] = {"csr_scalar", "csr_vector", "ell", "jds", "csr_stream"};
 
 dysel_status spmv_ctx_init(dysel_ctx *ctx) {
   if (cudaMalloc(&ctx->d_spmv_state, sizeof(SpmvStateBlock)) != cudaSuccess) return DYSEL_ERR_NOMEM;
@@ -539,6 +676,7 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
     I.jds_bytes = (size_t)n_rows * 8 + (size_t)(nb + 1) * 16 + (size_t)total * 4 + (size_t)nnz * 8;
     pl->vids[pl->K++] = DYSEL_SPMV_JDS;
   }
+  if (formats_mask & DYSEL_FMT_STREAM) pl->vids[pl->K++] = DYSEL_SPMV_CSR_STREAM;
   if (cudaStreamSynchronize(st) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   pl->def = pool_index(pl, default_variant);
   if (pl->def < 0) {
@@ -692,7 +830,9 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
     rep->c = P.c;
     rep->n_granules = P.Gn;
     rep->eager_units = 0;
-    for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v) rep->score[v] = rep->makespan_ns[v] = rep->units[v] = rep->cycles[v] = 0;
+    rep->tail_units = 0;
+    for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v)
+      rep->score[v] = rep->makespan_ns[v] = rep->units[v] = rep->cycles[v] = rep->busy_ns[v] = rep->aborted[v] = 0;
   }
   uint8_t *d_uv = nullptr;
   if (rep && rep->unit_variant) {
@@ -721,8 +861,10 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.hybrid = P.mode == DYSEL_HYBRID;
   p.async = (mode & DYSEL_ASYNC) != 0;
   p.contiguous = (mode & DYSEL_CONTIGUOUS) != 0;
-  p.score_cycles = (mode & DYSEL_SCORE_CYCLES) != 0;
+  p.score_mode = (mode & DYSEL_SCORE_CYCLES) ? 1u : ((mode & DYSEL_SCORE_MAKESPAN) ? 2u : 0u);
   p.def = (uint32_t)pl->def;
+  p.tail = (mode & DYSEL_NO_TAIL) ? 0u : 1u;
+  p.abort = (mode & DYSEL_NO_ABORT) ? 0u : 1u;
   p.n_tickets = (uint32_t)(P.Gn + (p.hybrid ? (uint64_t)(pl->K - 1) * P.c : 0));
   for (int i = 0; i < pl->K; ++i) p.vids[i] = pl->vids[i];
   if (p.hybrid) {
@@ -732,7 +874,9 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.unit_variant = d_uv;
   SpmvDev A = pl->dev;
   A.x = d_x;
-  const int grid = (int)std::min<uint64_t>((uint64_t)pl->persist_grid, p.n_tickets);
+  // sync + tail: the dispatcher only runs the K*c profiling tickets
+  const uint64_t work = (p.tail && !p.async) ? (uint64_t)p.K * p.c : p.n_tickets;
+  const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)pl->persist_grid, work));
   SpmvStateBlock *sb = (SpmvStateBlock *)ctx->d_spmv_state;
   spmv_persistent_kernel<<<grid, kUnitRows, 0, st>>>(A, d_y, sb, p);
   DYSEL_TRY(check_launch(ctx, "spmv_persistent_kernel"));
@@ -744,19 +888,23 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(rep->unit_variant, d_uv, std::min<uint64_t>(P.Gn, rep->unit_variant_cap),
                                           cudaMemcpyDeviceToHost, st));
     DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
-    if (d_uv && rep->unit_variant)   // pool index -> variant id
-      for (uint64_t j = 0; j < P.Gn && j < rep->unit_variant_cap; ++j)
-        rep->unit_variant[j] = (uint8_t)pl->vids[rep->unit_variant[j] < pl->K ? rep->unit_variant[j] : 0];
     const int sel_pool = (int)(h->sel & 0xff);
     rep->selected = sel_pool < pl->K ? pl->vids[sel_pool] : -1;
     rep->eager_units = h->eager_units;
+    rep->tail_units = h->tail_begin != ~0ull ? pl->n_units - h->tail_begin : 0;
     for (int v = 0; v < pl->K; ++v) {
       const int id = pl->vids[v];
       const dysel_timer_slot &t = h->slot[v];
+      rep->busy_ns[id] = h->busy[v];
+      rep->aborted[id] = h->aborted[v];
       rep->makespan_ns[id] = t.t_end_max - t.t_start_min;
       rep->units[id] = t.units;
       rep->cycles[id] = t.cycles;
-      rep->score[id] = p.score_cycles ? (t.units ? t.cycles / t.units : 0) : rep->makespan_ns[id];
+      const uint64_t cap = (1ull << 56) - 1;
+      rep->score[id] = h->dominated[v] ? cap
+                       : p.score_mode == 1 ? (t.units ? t.cycles / t.units : cap)
+                       : p.score_mode == 2 ? rep->makespan_ns[id]
+                                           : (t.units ? h->busy[v] / t.units : cap);
     }
     if (sel_pool < pl->K) ctx->sel_cache[pl->sig] = sel_pool;
     rep->host_ns = now_ns() - t_host0;

@@ -13,8 +13,17 @@
 //         thread per row, coalesced; pad slots (col = -1) are skipped (A-16).
 //  JDS    Parboil spmv-jds, block-local (A-14): thread per
 //         permuted row of the unit, diagonal k of the block contiguous.
+//  CSR-W  (B200-native addition) warp-streaming CSR: each
+//         warp streams the contiguous nonzeros of its 32-row group with fully
+//         coalesced loads and forms the row sums with a warp-level segmented
+//         reduction (head flags from __reduce_or_sync, Hillis-Steele scan with
+//         __shfl_up_sync); chunks wholly inside one row skip the scan.
 // CSR-S, ELL and JDS accumulate each row's products in CSR order with fmaf
 // from +0, so the three are bit-identical to each other.
+//
+// Poll: the persistent dispatcher passes a SandboxPoll to hybrid-mode sandbox
+// runs so a provably-losing variant can stop early (spmv.cu, dominance rule);
+// NoPoll compiles to nothing.
 #pragma once
 
 #include <stdint.h>
@@ -24,6 +33,7 @@ namespace dysel {
 constexpr int kUnitRows = 256;
 constexpr int kVecMin = 128;   // CSR-V: rows at least this long use 128-bit loads
 constexpr int kRowBatch = 4;   // CSR-V: rows in flight per warp
+constexpr int kStreamUnroll = 4;   // CSR-W: 32-entry chunks in flight per warp
 
 struct SpmvDev {
   int32_t n_rows, n_cols;
@@ -45,6 +55,11 @@ struct SpmvDev {
   const float *__restrict__ jds_val;
   const float *__restrict__ x;
   int32_t vec_ok;   // col/val 16-byte aligned
+};
+
+struct NoPoll {
+  static constexpr bool active = false;
+  __device__ __forceinline__ bool operator()() const { return false; }
 };
 
 // ------------------------------------------------------------ load helpers
@@ -93,7 +108,9 @@ __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
 }
 
 // ------------------------------------------------------------------ CSR-S
-__device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, float *__restrict__ out) {
+template <class Poll>
+__device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, float *__restrict__ out,
+                                                const Poll &poll) {
   const int i = threadIdx.x;
   const int64_t r = (int64_t)j * kUnitRows + i;
   if (r >= A.n_rows) return;
@@ -101,7 +118,10 @@ __device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, fl
   const int b = __ldg(A.row_ptr + r), e = __ldg(A.row_ptr + r + 1);
   float s = 0.0f;
 #pragma unroll 4
-  for (int k = b; k < e; ++k) s = __fmaf_rn(__ldg(A.val + k), ld_x(A.x + __ldg(A.col + k), px), s);
+  for (int k = b; k < e; ++k) {
+    s = __fmaf_rn(__ldg(A.val + k), ld_x(A.x + __ldg(A.col + k), px), s);
+    if (Poll::active && ((k - b) & 63) == 63 && poll()) break;
+  }
   out[i] = s;
 }
 
@@ -109,8 +129,9 @@ __device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, fl
 // Long row (len >= kVecMin): lane l sums, in order, the head entries
 // [b, a) it owns (a = first 4-aligned index), its 4-entry groups of the body
 // (chunks of 128 entries), then the tail; the 32 lane sums are xor-reduced.
-__device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, int lane, uint64_t ps,
-                                               uint64_t px) {
+template <class Poll>
+__device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, int lane, uint64_t ps, uint64_t px,
+                                               const Poll &poll) {
   float s = 0.0f;
   // unaligned base pointers: no head / vector body, everything in the tail loop
   const int a = A.vec_ok ? min((b + 3) & ~3, e) : b;
@@ -136,6 +157,7 @@ __device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, i
     s = __fmaf_rn(v1.y, y1, s);
     s = __fmaf_rn(v1.z, y2, s);
     s = __fmaf_rn(v1.w, y3, s);
+    if (Poll::active && poll()) return s;
   }
   for (; base < body_end; base += 128) {
     const int k0 = base + 4 * lane;
@@ -153,7 +175,9 @@ __device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, i
   return s;
 }
 
-__device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, float *__restrict__ out) {
+template <class Poll>
+__device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, float *__restrict__ out,
+                                                const Poll &poll) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t base = (int64_t)j * kUnitRows + w * 32;
   const int nr = (int)min((int64_t)32, (int64_t)A.n_rows - base);
@@ -190,7 +214,7 @@ __device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, fl
         for (int k = b[r] + lane + 32; k < e[r]; k += 32)
           s[r] = __fmaf_rn(ld_stream(A.val + k, ps), ld_x(A.x + ld_stream(A.col + k, ps), px), s[r]);
       } else {
-        s[r] = csrv_long_row(A, b[r], e[r], lane, ps, px);
+        s[r] = csrv_long_row(A, b[r], e[r], lane, ps, px, poll);
       }
     }
 #pragma unroll
@@ -200,12 +224,14 @@ __device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, fl
 #pragma unroll
     for (int r = 0; r < kRowBatch; ++r)
       if (lane == i0 + r) mine = s[r];
+    if (Poll::active && poll()) break;
   }
   if (lane < nr) out[w * 32 + lane] = mine;
 }
 
 // -------------------------------------------------------------------- ELL
-__device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, float *__restrict__ out) {
+template <class Poll>
+__device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, float *__restrict__ out, const Poll &poll) {
   const int i = threadIdx.x;
   const int64_t r = (int64_t)j * kUnitRows + i;
   if (r >= A.n_rows) return;
@@ -230,6 +256,10 @@ __device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, float *__
       break;
     }
     s = __fmaf_rn(v1, ld_x(A.x + c1, px), s);
+    if (Poll::active && (k & 63) == 62 && poll()) {
+      live = false;
+      break;
+    }
   }
   if (live && k < A.ell_W) {
     const int c0 = ld_stream(cp + (int64_t)k * A.n_pad, ps);
@@ -239,7 +269,8 @@ __device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, float *__
 }
 
 // -------------------------------------------------------------------- JDS
-__device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, float *__restrict__ out) {
+template <class Poll>
+__device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, float *__restrict__ out, const Poll &poll) {
   const int p = threadIdx.x;
   const int64_t q = (int64_t)j * kUnitRows + p;
   if (q >= A.n_rows) return;
@@ -252,24 +283,113 @@ __device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, float *__
   for (int k = 0; k < len; ++k) {
     const int64_t idx = base + __ldg(jp + k);
     s = __fmaf_rn(ld_stream(A.jds_val + idx, ps), ld_x(A.x + ld_stream(A.jds_col + idx, ps), px), s);
+    if (Poll::active && (k & 63) == 63 && poll()) break;
   }
   out[__ldg(A.perm + q) - (int64_t)j * kUnitRows] = s;
 }
 
-template <int VID>
-__device__ __forceinline__ void run_unit(const SpmvDev &A, uint32_t j, float *out) {
-  if constexpr (VID == 0) unit_csr_scalar(A, j, out);
-  else if constexpr (VID == 1) unit_csr_vector(A, j, out);
-  else if constexpr (VID == 2) unit_ell(A, j, out);
-  else unit_jds(A, j, out);
+// ------------------------------------------------------------------ CSR-W
+// Warp-streaming CSR.  Lane i owns row i of the warp's 32-row group
+// (accumulator acc).  The group's nonzeros [s, e) are walked in 32-entry
+// chunks, entry k = cb + lane per lane (coalesced 128-byte col / val loads).
+// Chunk wholly inside the open row: per-lane partial `part += p`.  Otherwise:
+// fold `part` into the open row (butterfly), then a segmented inclusive scan
+// of the products (heads = row starts in the chunk, bit 0 always set); row i
+// takes the scan value at the last lane of its segment.  The per-row order
+// depends only on the row's offset inside its group: deterministic (c-6).
+template <class Poll>
+__device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, float *__restrict__ out,
+                                                const Poll &poll) {
+  const uint32_t FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t base = (int64_t)j * kUnitRows + w * 32;
+  const int nr = (int)min((int64_t)32, (int64_t)A.n_rows - base);
+  if (nr <= 0) return;
+  const uint64_t ps = policy_evict_first(), px = policy_evict_last();
+  const int gend = __ldg(A.row_ptr + base + nr);
+  const int re = lane < nr ? __ldg(A.row_ptr + base + lane + 1) : gend;
+  const int rs = lane < nr ? __ldg(A.row_ptr + base + lane) : gend;
+  const int s = __shfl_sync(FULL, rs, 0);
+  const int e = gend;
+  float acc = 0.0f, part = 0.0f;
+  // open row at chunk start: the non-empty row containing entry cb
+  auto open_row = [&](int cb) -> int {
+    const uint32_t m = __ballot_sync(FULL, rs <= cb && cb < re);
+    return m ? __ffs(m) - 1 : -1;
+  };
+  int o = open_row(s);
+  int oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
+  const uint32_t lane_mask_le = (lane == 31) ? FULL : ((2u << lane) - 1u);
+  for (int c0 = s; c0 < e; c0 += 32 * kStreamUnroll) {
+    int cc[kStreamUnroll];
+    float vv[kStreamUnroll], pp[kStreamUnroll];
+#pragma unroll
+    for (int u = 0; u < kStreamUnroll; ++u) {
+      const int k = c0 + 32 * u + lane;
+      const bool ok = k < e;
+      cc[u] = ok ? ld_stream(A.col + k, ps) : -1;
+      vv[u] = ok ? ld_stream(A.val + k, ps) : 0.0f;
+    }
+#pragma unroll
+    for (int u = 0; u < kStreamUnroll; ++u) pp[u] = cc[u] >= 0 ? vv[u] * ld_x(A.x + cc[u], px) : 0.0f;
+#pragma unroll
+    for (int u = 0; u < kStreamUnroll; ++u) {
+      const int cb = c0 + 32 * u;
+      if (cb >= e) break;
+      if (oe >= cb + 32) {   // whole chunk inside the open row
+        part += pp[u];
+        continue;
+      }
+      // fold the open row's per-lane partials
+      float P = part;
+#pragma unroll
+      for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
+      if (lane == o) acc += P;
+      part = 0.0f;
+      // segmented inclusive scan over the chunk
+      const uint32_t bit = (rs >= cb && rs < cb + 32 && rs < re) ? (1u << (rs - cb)) : 0u;
+      const uint32_t H = __reduce_or_sync(FULL, bit) | 1u;
+      const int seg_start = 31 - __clz(H & lane_mask_le);
+      float v = pp[u];
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const float t = __shfl_up_sync(FULL, v, d);
+        if (lane - d >= seg_start) v += t;
+      }
+      const int lo = max(rs, cb), hi = min(re, cb + 32);
+      const bool has = lo < hi;
+      const float got = __shfl_sync(FULL, v, has ? hi - 1 - cb : 0);
+      if (has) acc += got;
+      const int nb = cb + 32;
+      o = open_row(nb);
+      oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
+    }
+    if (Poll::active && poll()) break;
+  }
+  float P = part;
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
+  if (lane == o) acc += P;
+  if (lane < nr) out[w * 32 + lane] = acc;
 }
 
-__device__ __forceinline__ void run_unit_dyn(int vid, const SpmvDev &A, uint32_t j, float *out) {
+template <int VID, class Poll = NoPoll>
+__device__ __forceinline__ void run_unit(const SpmvDev &A, uint32_t j, float *out, const Poll &poll = Poll()) {
+  if constexpr (VID == 0) unit_csr_scalar(A, j, out, poll);
+  else if constexpr (VID == 1) unit_csr_vector(A, j, out, poll);
+  else if constexpr (VID == 2) unit_ell(A, j, out, poll);
+  else if constexpr (VID == 3) unit_jds(A, j, out, poll);
+  else unit_csr_stream(A, j, out, poll);
+}
+
+template <class Poll>
+__device__ __forceinline__ void run_unit_dyn(int vid, const SpmvDev &A, uint32_t j, float *out, const Poll &poll) {
   switch (vid) {
-    case 0: unit_csr_scalar(A, j, out); break;
-    case 1: unit_csr_vector(A, j, out); break;
-    case 2: unit_ell(A, j, out); break;
-    default: unit_jds(A, j, out); break;
+    case 0: unit_csr_scalar(A, j, out, poll); break;
+    case 1: unit_csr_vector(A, j, out, poll); break;
+    case 2: unit_ell(A, j, out, poll); break;
+    case 3: unit_jds(A, j, out, poll); break;
+    default: unit_csr_stream(A, j, out, poll); break;
   }
 }
 

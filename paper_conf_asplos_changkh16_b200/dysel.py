@@ -25,13 +25,16 @@ OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_NOMEM, ERR_CUDA, ERR_NOT_FOUND, ERR_NCCL =
 FULLY, HYBRID, SWAP, AUTO = 0, 1, 2, 3
 SYNC, ASYNC = 0, 4
 NO_PROFILE, HOST_ORCH, FORCE_PROFILE, CONTIGUOUS, SCORE_CYCLES = 8, 16, 32, 64, 128
+SCORE_MAKESPAN, NO_TAIL, NO_ABORT = 256, 512, 1024
 DEFAULT_MODE = FULLY | ASYNC
 V_ATOMICS, V_NONUNIFORM = 1, 2
 ROLE_PRODUCTIVE, ROLE_SANDBOX, ROLE_BATCH, ROLE_PRIVATE, ROLE_EAGER = range(5)
 MAX_VARIANTS = 16
-SPMV_CSR_SCALAR, SPMV_CSR_VECTOR, SPMV_ELL, SPMV_JDS = range(4)
-SPMV_NAMES = ["csr_scalar", "csr_vector", "ell", "jds"]
-FMT_ELL, FMT_JDS = 1, 2
+SPMV_CSR_SCALAR, SPMV_CSR_VECTOR, SPMV_ELL, SPMV_JDS, SPMV_CSR_STREAM = range(5)
+SPMV_NVARIANTS = 5
+SPMV_NAMES = ["csr_scalar", "csr_vector", "ell", "jds", "csr_stream"]
+FMT_ELL, FMT_JDS, FMT_STREAM = 1, 2, 4
+FMT_ALL = FMT_ELL | FMT_JDS | FMT_STREAM
 SGEMM_S64, SGEMM_S128, SGEMM_T128x64, SGEMM_T128x128 = range(4)
 SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"]
 
@@ -50,6 +53,7 @@ class Report(ctypes.Structure):
                 ("n_variants", ctypes.c_int32), ("c", c_u64), ("n_granules", c_u64),
                 ("score", c_u64 * MAX_VARIANTS), ("makespan_ns", c_u64 * MAX_VARIANTS),
                 ("units", c_u64 * MAX_VARIANTS), ("cycles", c_u64 * MAX_VARIANTS),
+                ("busy_ns", c_u64 * MAX_VARIANTS), ("aborted", c_u64 * MAX_VARIANTS), ("tail_units", c_u64),
                 ("eager_units", c_u64), ("host_ns", c_u64), ("slices", ctypes.POINTER(SliceRec)),
                 ("slices_cap", ctypes.c_int32), ("n_slices", ctypes.c_int32),
                 ("unit_variant", ctypes.POINTER(ctypes.c_uint8)), ("unit_variant_cap", c_u64)]
@@ -57,7 +61,7 @@ class Report(ctypes.Structure):
 
 class PlanInfo(ctypes.Structure):
     _fields_ = [("n_rows", c_i64), ("n_cols", c_i64), ("nnz", c_i64), ("n_variants", ctypes.c_int32),
-                ("variant_ids", ctypes.c_int32 * 4), ("ell_width", ctypes.c_int32), ("uniform", ctypes.c_int32),
+                ("variant_ids", ctypes.c_int32 * SPMV_NVARIANTS), ("ell_width", ctypes.c_int32), ("uniform", ctypes.c_int32),
                 ("max_row_len", ctypes.c_int32), ("prep_ns", c_u64), ("ell_bytes", c_u64), ("jds_bytes", c_u64)]
 
 
@@ -135,7 +139,8 @@ def report_dict(rep: Report, names=None, uv=None):
              c=rep.c, n_granules=rep.n_granules, eager_units=rep.eager_units, host_ns=rep.host_ns,
              score=list(rep.score[:MAX_VARIANTS]), makespan_ns=list(rep.makespan_ns[:MAX_VARIANTS]),
              units=list(rep.units[:MAX_VARIANTS]), cycles=list(rep.cycles[:MAX_VARIANTS]),
-             n_slices=rep.n_slices)
+             busy_ns=list(rep.busy_ns[:MAX_VARIANTS]), aborted=list(rep.aborted[:MAX_VARIANTS]),
+             tail_units=rep.tail_units, n_slices=rep.n_slices)
     if rep.slices and rep.slices_cap:
         d["slices"] = [dict(begin=rep.slices[i].granule_begin, count=rep.slices[i].granule_count,
                             stride=rep.slices[i].granule_stride, variant=rep.slices[i].variant,
@@ -239,7 +244,7 @@ class Context:
         return int(dysel_kernel_launches(self.h))
 
     # ------------------------------------------------------------- SpMV
-    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ELL | FMT_JDS, default=SPMV_CSR_VECTOR,
+    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ALL, default=SPMV_CSR_VECTOR,
                      stream=None) -> SpmvPlan:
         n = row_ptr.numel() - 1
         nnz = col.numel()

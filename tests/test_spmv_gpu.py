@@ -237,6 +237,54 @@ def test_edge_cases(ctx, D):
     assert e.value.status == D.ERR_UNSUPPORTED
 
 
+@pytest.mark.parametrize("asy", [False, True])
+def test_tail_launch_hands_off_remainder(ctx, D, asy):
+    """The winner's plain kernel runs the unclaimed remainder (CDP2 tail
+    launch); NO_TAIL keeps it inside the dispatcher.  Same output either way."""
+    import torch
+    A = MATS["powerlaw"]()
+    x = uniform_f32(11, A.n_cols)
+    plan = prepared(ctx, A)
+    mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0)
+    y1 = torch.empty(A.n_rows, device="cuda")
+    r1 = ctx.spmv(plan, vec(x), y1, f=0.05, mode=mode, report=True, unit_map=True)
+    if not asy:
+        assert r1["tail_units"] == plan.n_units - len(plan.variant_ids) * r1["c"]
+    assert spmv_err(A, x, y1) <= SPMV_TOL
+    y2 = torch.empty(A.n_rows, device="cuda")
+    r2 = ctx.spmv(plan, vec(x), y2, f=0.05, mode=mode | D.NO_TAIL, report=True)
+    assert r2["tail_units"] == 0
+    assert spmv_err(A, x, y2) <= SPMV_TOL
+    plan.destroy()
+
+
+def test_dominance_abort_is_exact(ctx, D):
+    """Hybrid sandbox units of a variant whose guaranteed busy time already
+    exceeds a completed variant's total stop early; the dominated variant gets
+    the maximal score and the winner is the busy-time argmin of the others."""
+    import torch
+    from workloads import csr_from_lengths
+    # a few very long rows make thread-per-row variants hopeless
+    L = np.full(40 * 256, 8)
+    L[::97] = 6000
+    A = csr_from_lengths(L, 20000, 21, 22)
+    x = uniform_f32(23, A.n_cols)
+    plan = prepared(ctx, A, default=1)
+    y = torch.empty(A.n_rows, device="cuda")
+    rep = ctx.spmv(plan, vec(x), y, f=0.5, mode=D.HYBRID | D.SYNC | D.FORCE_PROFILE, report=True)
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    ids = plan.variant_ids
+    cap = (1 << 56) - 1
+    live = [v for v in ids if rep["score"][v] != cap]
+    assert rep["selected"] == min(live, key=lambda v: (rep["score"][v], ids.index(v)))
+    assert sum(rep["aborted"][v] for v in ids) > 0          # someone was stopped
+    assert all(rep["score"][v] == cap for v in ids if rep["aborted"][v] > 0)
+    rep2 = ctx.spmv(plan, vec(x), y, f=0.5, mode=D.HYBRID | D.SYNC | D.FORCE_PROFILE | D.NO_ABORT, report=True)
+    assert sum(rep2["aborted"][v] for v in ids) == 0
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    plan.destroy()
+
+
 def test_long_rows_vector_path(ctx):
     """Rows >= 128 entries take CSR-V's 128-bit path (head / body / tail)."""
     import torch
