@@ -85,6 +85,8 @@ const char *dysel_status_str(dysel_status s);
 #define DYSEL_SCORE_MAKESPAN 256u /* score = latest CTA end - earliest CTA start (%globaltimer), Fig. 7b */
 #define DYSEL_NO_TAIL 512u      /* SpMV device path: run the remainder inside the dispatcher (no CDP2 tail launch) */
 #define DYSEL_NO_ABORT 1024u    /* SpMV device path: never stop dominated sandbox units early */
+#define DYSEL_SEQUENTIAL 2048u  /* SpMV device path: profile the variants one after another, each alone on the
+                                   GPU (default variant first), scored by makespan (reading A-23) */
 /* Default score: generic launcher = makespan (variants are separate concurrent
  * grids, Fig. 7b); SpMV dispatcher = mean per-unit busy time (%globaltimer end -
  * start of each profiled unit; all variants share one launch and occupancy). */

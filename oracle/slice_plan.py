@@ -94,8 +94,13 @@ def resolve_mode(mode, vflags):
     return base
 
 
-def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS) -> Plan:
-    """U: units per dim (3-tuple); wa: per-variant 3-tuples of units per CTA."""
+def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, wave_units=0) -> Plan:
+    """U: units per dim (3-tuple); wa: per-variant 3-tuples of units per CTA.
+
+    wave_units (reading A-3b, SpMV device path): profiling is also off when
+    the whole grid (G_n granules) fits in one wave of the default variant —
+    everything runs concurrently, so no remainder can benefit.
+    """
     K = len(wa)
     vflags = vflags or [0] * K
     if not (1 <= K <= 16) or not (0.0 <= f <= 1.0) or not (0 <= default_variant < K):
@@ -128,7 +133,7 @@ def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS) 
                 c = 1 if (Gn >= K if rmode == FULLY else Gn >= 1) else 0
             active = c >= 1
         else:
-            active = c >= 1 and default_ctas >= min_ctas
+            active = c >= 1 and default_ctas >= min_ctas and Gn > wave_units
     p = Plan(K, g, G, Gn, h, c if active else 0, active, rmode)
     if not active:
         p.remainder = list(range(Gn))

@@ -327,8 +327,12 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
   cudaDeviceGetAttribute(&ctx->n_sm, cudaDevAttrMultiProcessorCount, cuda_device);
   cudaDeviceGetAttribute(&v, cudaDevAttrL2CacheSize, cuda_device);
   ctx->l2_bytes = (uint64_t)v;
+  // profiling streams get the highest priority: profiling before eager work
+  int prio_lo = 0, prio_hi = 0;
+  cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
   for (int i = 0; i < DYSEL_MAX_VARIANTS; ++i) {
-    if (cudaStreamCreateWithFlags(&ctx->fork[i], cudaStreamNonBlocking) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+    if (cudaStreamCreateWithPriority(&ctx->fork[i], cudaStreamNonBlocking, prio_hi) != cudaSuccess)
+      return fail(DYSEL_ERR_CUDA);
     if (cudaEventCreateWithFlags(&ctx->ev_join[i], cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   }
   if (cudaStreamCreateWithFlags(&ctx->query, cudaStreamNonBlocking) != cudaSuccess) return fail(DYSEL_ERR_CUDA);

@@ -157,7 +157,7 @@ __device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, i
     s = __fmaf_rn(v1.y, y1, s);
     s = __fmaf_rn(v1.z, y2, s);
     s = __fmaf_rn(v1.w, y3, s);
-    if (Poll::active && poll()) return s;
+    if (Poll::active && __any_sync(0xffffffffu, poll())) return s;   // warp-uniform exit
   }
   for (; base < body_end; base += 128) {
     const int k0 = base + 4 * lane;
@@ -224,7 +224,7 @@ __device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, fl
 #pragma unroll
     for (int r = 0; r < kRowBatch; ++r)
       if (lane == i0 + r) mine = s[r];
-    if (Poll::active && poll()) break;
+    if (Poll::active && __any_sync(0xffffffffu, poll())) break;   // warp-uniform exit
   }
   if (lane < nr) out[w * 32 + lane] = mine;
 }
@@ -364,7 +364,7 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, fl
       o = open_row(nb);
       oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
     }
-    if (Poll::active && poll()) break;
+    if (Poll::active && __any_sync(FULL, poll())) break;   // warp-uniform exit
   }
   float P = part;
 #pragma unroll

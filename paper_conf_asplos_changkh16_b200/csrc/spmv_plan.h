@@ -1,0 +1,30 @@
+// dysel_spmv_plan: the SpMV variant pool for one CSR matrix (shared by
+// spmv_prep.cu — format preparation — and spmv.cu — dispatch).
+#pragma once
+
+#include <string>
+
+#include "internal.h"
+#include "spmv_kernels.cuh"
+
+struct dysel_spmv_plan {
+  dysel_ctx *ctx = nullptr;
+  dysel::SpmvDev dev{};
+  dysel_spmv_plan_info info{};
+  int32_t *ell_col = nullptr;
+  float *ell_val = nullptr;
+  int32_t *perm = nullptr, *jds_len = nullptr, *jd_ptr = nullptr, *jds_col = nullptr;
+  int64_t *blk_off = nullptr, *jd_off = nullptr;
+  float *jds_val = nullptr;
+  int K = 0;                          // pool size
+  int vids[DYSEL_SPMV_NVARIANTS] = {};  // pool index -> DYSEL_SPMV_* id
+  int def = 0;                        // pool index of the default (initial) variant
+  uint32_t n_units = 0;               // 256-row units
+  std::string sig;                    // generic-registry signature (host path)
+};
+
+namespace dysel {
+int spmv_pool_index(const dysel_spmv_plan *pl, int vid);
+// register the plan's pool with the generic launcher (host-orchestrated path)
+dysel_status spmv_register_pool(dysel_ctx *ctx, dysel_spmv_plan *pl);
+}  // namespace dysel

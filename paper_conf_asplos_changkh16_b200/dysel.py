@@ -25,7 +25,7 @@ OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_NOMEM, ERR_CUDA, ERR_NOT_FOUND, ERR_NCCL =
 FULLY, HYBRID, SWAP, AUTO = 0, 1, 2, 3
 SYNC, ASYNC = 0, 4
 NO_PROFILE, HOST_ORCH, FORCE_PROFILE, CONTIGUOUS, SCORE_CYCLES = 8, 16, 32, 64, 128
-SCORE_MAKESPAN, NO_TAIL, NO_ABORT = 256, 512, 1024
+SCORE_MAKESPAN, NO_TAIL, NO_ABORT, SEQUENTIAL = 256, 512, 1024, 2048
 DEFAULT_MODE = FULLY | ASYNC
 V_ATOMICS, V_NONUNIFORM = 1, 2
 ROLE_PRODUCTIVE, ROLE_SANDBOX, ROLE_BATCH, ROLE_PRIVATE, ROLE_EAGER = range(5)
@@ -244,7 +244,7 @@ class Context:
         return int(dysel_kernel_launches(self.h))
 
     # ------------------------------------------------------------- SpMV
-    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ALL, default=SPMV_CSR_VECTOR,
+    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ELL | FMT_JDS, default=SPMV_CSR_VECTOR,
                      stream=None) -> SpmvPlan:
         n = row_ptr.numel() - 1
         nnz = col.numel()

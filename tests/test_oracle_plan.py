@@ -64,6 +64,13 @@ def test_small_workload_deactivation():
     assert not p.active and p.remainder == list(range(128))
 
 
+def test_single_wave_deactivation_reading_a3b():
+    # D3: 574 units fit in one wave (8 CTAs/SM x 148 SMs) -> off; D4 does not
+    assert not P.plan((574,), [(1,)] * 4, 0.02, 148, 0, P.FULLY, wave_units=8 * 148).active
+    assert P.plan((574,), [(1,)] * 4, 0.02, 148, 0, P.FULLY | P.FORCE_PROFILE, wave_units=8 * 148).active
+    assert P.plan((39063,), [(1,)] * 3, 0.02, 148, 0, P.HYBRID, wave_units=4 * 148).active
+
+
 def test_survey_sgemm_d2m_numbers():
     # SGEMM medium 1024x992x1056, unit = 32x32 tile: U = (33, 32); tilings
     # 64x64 (2,2), 128x128 (4,4), 128x64 (N=64 -> 2, M=128 -> 4), 128x128.
