@@ -131,6 +131,7 @@ struct SandboxPoll {
 };
 
 // resident CTAs per SM each plain variant kernel is compiled for (register cap)
+// (CSR-V at 6/SM spills and measured slower on D4: 1.44 vs 1.35 ms)
 constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 6};
 
 // Plain kernel of one variant over a slice: the exhaustive oracle's pure
@@ -259,6 +260,8 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
   const unsigned long long fin = atomicAdd((unsigned long long *)&st->best, 0ull);
   atomicExch((unsigned long long *)&st->sel, fin);
   __threadfence();
+  // (measured: handing the remainder to the plain kernel beats letting the
+  // persistent eager kernel finish it even when the default won)
   if (p.tail) {
     const uint32_t old = p.async ? atomicAdd(&st->ticket, 1u << 30) : 0u;   // stop eager claims
     const uint64_t u0 = (uint64_t)p.p_end + old;

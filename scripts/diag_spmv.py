@@ -27,10 +27,11 @@ for v in plan.variant_ids:
 if only: sys.exit(0)
 ids = plan.variant_ids
 F = float(os.environ.get("F", "0.02"))
-for name, mode, f in [("auto_async", D.AUTO|D.ASYNC, F), ("auto_sync", D.AUTO, F), ("fully_async", D.FULLY|D.ASYNC, F),
+MODES = [(f"auto_async_f{f}", D.AUTO|D.ASYNC, f) for f in (0.002, 0.005, 0.01, 0.02, 0.05)] + [("auto_async", D.AUTO|D.ASYNC, F), ("auto_sync", D.AUTO, F), ("fully_async", D.FULLY|D.ASYNC, F),
                    ("hybrid_async_f.005", D.HYBRID|D.ASYNC, 0.005), ("hybrid_seq_f.1", D.HYBRID|D.SEQUENTIAL, 0.1),
                    ("hybrid_seq_f.05", D.HYBRID|D.SEQUENTIAL, 0.05), ("fully_seq_f.1", D.FULLY|D.SEQUENTIAL, 0.1),
-                   ("hybrid_sync_host", D.HYBRID|D.HOST_ORCH, F), ("no_profile", D.NO_PROFILE, F)]:
+                   ("hybrid_sync_host", D.HYBRID|D.HOST_ORCH, F), ("no_profile", D.NO_PROFILE, F)]
+for name, mode, f in MODES:
     t = ev_time(lambda: ctx.spmv(plan, x, y, f=f, mode=mode))
     r = ctx.spmv(plan, x, y, f=f, mode=mode, report=True)
     print(f"{name:22s} ms {t:8.4f} sel {r['selected_name']:10s} c {r['c']} eager {r['eager_units']} tail {r['tail_units']}",
