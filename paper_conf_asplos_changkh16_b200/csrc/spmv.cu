@@ -49,6 +49,7 @@ struct SpmvState {
 struct ProfParams {
   uint32_t K, c, n_units, p_end;   // p_end: first remainder unit
   uint32_t hybrid, async, contiguous, score_mode, def, tail, abort;
+  uint32_t eager_grid;   // ASYNC: CTAs of the eager kernel (launched by the default's first profiling CTA)
   int32_t vids[DYSEL_SPMV_NVARIANTS];
   uint32_t occ[DYSEL_SPMV_NVARIANTS];
   float *sandbox;        // (K-1) * c * 256 floats (hybrid)
@@ -173,6 +174,26 @@ __device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, ui
   }
 }
 
+template <int VID>
+__global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
+    spmv_eager_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, uint32_t p_end, uint32_t n_units, uint8_t *uv);
+
+// The eager grid is launched from the device (fire-and-forget child of the
+// default variant's first profiling CTA), so it can only start once profiling
+// CTAs are resident: a host launch becomes runnable at the same instant as the
+// profiling grids when calls are queued back to back, and the persistent
+// eager CTAs then take every SM first (measured: +30% step time).
+__device__ void eager_launch(int vid, const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p) {
+  const unsigned g = p.eager_grid;
+  switch (vid) {
+    case 0: spmv_eager_kernel<0><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
+    case 1: spmv_eager_kernel<1><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
+    case 2: spmv_eager_kernel<2><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
+    case 3: spmv_eager_kernel<3><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
+    default: spmv_eager_kernel<4><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
+  }
+}
+
 // Profiling copy of variant VID (pool index pv): one CTA per profiling unit.
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
@@ -184,6 +205,7 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
   const uint32_t j = p.hybrid ? b : (p.contiguous ? pv * p.c + b : pv + p.K * b);
   const bool productive = !p.hybrid || pv == p.def;
   const bool sandbox = !productive;
+  if (tid == 0 && b == 0 && pv == p.def && p.eager_grid) eager_launch(p.vids[p.def], A, y, st, p);
   if (tid == 0) {
     s_abort = 0;
     s_last = dysel_globaltimer();
@@ -531,6 +553,12 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   SpmvDev A = pl->dev;
   A.x = d_x;
   SpmvState *dst = cs->d_state;
+  if (p.async && p.p_end < p.n_units) {
+    const int dv = pl->vids[pl->def];
+    p.eager_grid =
+        (uint32_t)std::min<uint64_t>((uint64_t)std::max(1, cs->occ_eager[dv]) * ctx->n_sm, p.n_units - p.p_end);
+    ctx->launches++;   // device-side launch
+  }
   spmv_state_init_kernel<<<1, 32, 0, st>>>(dst, pl->K, pl->def);
   DYSEL_TRY(check_launch(ctx, "spmv_state_init_kernel"));
   DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_start, st));
@@ -550,12 +578,6 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       DYSEL_TRY(check_launch(ctx, "spmv_prof_kernel"));
       DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[i], ctx->fork[i]));
     }
-  }
-  if (p.async && p.p_end < p.n_units) {
-    const int dv = pl->vids[pl->def];
-    const int grid = (int)std::min<uint64_t>((uint64_t)std::max(1, cs->occ_eager[dv]) * ctx->n_sm, p.n_units - p.p_end);
-    kEager[dv](A, d_y, dst, p, grid, st);
-    DYSEL_TRY(check_launch(ctx, "spmv_eager_kernel"));
   }
   for (int i = 0; i < pl->K; ++i) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[i], 0));
   if (!p.tail && !p.async && p.p_end < p.n_units) {   // NO_TAIL: gated remainder copies of every variant

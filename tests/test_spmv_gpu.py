@@ -258,6 +258,30 @@ def test_tail_launch_hands_off_remainder(ctx, D, asy):
     plan.destroy()
 
 
+def test_tail_launch_is_stream_ordered(ctx, D):
+    """Work queued on the launching stream after dysel_spmv must see the
+    tail-launched remainder complete (the device-launched grid belongs to its
+    parent's completion), without any host synchronisation in between."""
+    import torch
+    A = d4_powerlaw(n=400_000, lmax=8000)
+    x = uniform_f32(12, A.n_cols)
+    plan = prepared(ctx, A)
+    xd = vec(x)
+    ref = torch.empty(A.n_rows, device="cuda")
+    ctx.spmv_variant(plan, 1, xd, ref)
+    torch.cuda.synchronize()
+    for mode in (D.HYBRID | D.SYNC, D.HYBRID | D.ASYNC, D.FULLY | D.SYNC):
+        for _ in range(3):
+            y = torch.full((A.n_rows,), float("nan"), device="cuda")
+            ctx.spmv(plan, xd, y, f=0.01, mode=mode | D.FORCE_PROFILE)
+            nan_count = torch.isnan(y).sum()          # same stream, no sync
+            snap = y.clone()
+            torch.cuda.synchronize()
+            assert nan_count.item() == 0, mode
+            assert spmv_err(A, x, snap) <= SPMV_TOL
+    plan.destroy()
+
+
 def test_dominance_abort_is_exact(ctx, D):
     """Hybrid sandbox units of a variant whose guaranteed busy time already
     exceeds a completed variant's total stop early; the dominated variant gets
