@@ -58,24 +58,33 @@ class ClockSampler:
         self._t = None
 
     def _run(self):
-        while not self._stop.is_set():
-            try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
-                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
-                                     timeout=5).stdout.strip()
-                if out:
-                    self.rows.append([c.strip() for c in out.split(",")])
-            except Exception:
-                pass
-            self._stop.wait(0.1)
+        # one long-lived `nvidia-smi -lms 20` reader (spawning a process per
+        # sample is too slow for a timed region of tens of ms)
+        try:
+            self._p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                        "--format=csv,noheader,nounits", "-lms", "20"],
+                                       stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            for line in self._p.stdout:
+                if line.strip():
+                    self.rows.append([c.strip() for c in line.split(",")])
+                if self._stop.is_set():
+                    break
+        except Exception:
+            pass
 
     def __enter__(self):
+        self._p = None
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
+        time.sleep(0.3)    # first samples before the timed region
+        self.rows.clear()
         return self
 
     def __exit__(self, *a):
+        time.sleep(0.05)
         self._stop.set()
+        if self._p is not None:
+            self._p.terminate()
         self._t.join(timeout=10)
 
     def summary(self):
