@@ -2,15 +2,63 @@
 // launcher (dysel_launch), so SGEMM exercises the same slice planner, device
 // timing and gated device-side remainder as user-registered kernels.
 // Unit = one 32x32 tile of C; wa = (tile_N/32, tile_M/32) (SURVEY §8 notation).
+#include <cudaTypedefs.h>
+
 #include <cstring>
 
 #include "internal.h"
 #include "sgemm_simt.cuh"
 #include "sgemm_tc.cuh"
+#include "sgemm_tma.cuh"
 
 namespace dysel {
 
 static const char *kSgemmSig = "dysel.sgemm";
+
+static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+    cudaGetLastError();
+  }
+  return fn;
+}
+
+// 2-D fp32 tensor map, 128-byte swizzle, zero fill out of bounds.
+static bool make_map(CUtensorMap *m, const float *base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
+                     uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz) {
+  auto enc = tensor_map_encoder();
+  if (!enc) return false;
+  const cuuint64_t dims[2] = {inner, outer};
+  const cuuint64_t strides[1] = {ld_elems * sizeof(float)};
+  const cuuint32_t box[2] = {box_inner, box_outer};
+  const cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)base, dims, strides, box, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// tcgen05 path: TMA pipeline when the operands allow TMA (16-byte aligned
+// bases, lda / ldb multiples of 4), else the register-staged kernel.
+template <int BN>
+static dysel_status launch_tc(const SgemmArgs &g, float *C, const dysel_slice &s, unsigned ctas, cudaStream_t st) {
+  const bool tma_ok = g.K > 0 && ((((uintptr_t)g.A) | ((uintptr_t)g.B)) & 15) == 0 && (g.lda % 4) == 0 &&
+                      (g.ldb % 4) == 0;
+  if (tma_ok) {
+    CUtensorMap ta, tb;
+    // A: K-major SW128 (16-byte granules); B: MN-major tf32 needs 32-byte atoms
+    if (make_map(&ta, g.A, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.lda, 32, 128, CU_TENSOR_MAP_SWIZZLE_128B) &&
+        make_map(&tb, g.B, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.ldb, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) {
+      sgemm_tma_kernel<BN><<<ctas, 192, TmaCfg<BN>::SMEM, st>>>(ta, tb, g, C, s);
+      return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
+    }
+  }
+  return launch_tc_sgemm<BN>(g, C, s, ctas, st);
+}
 
 template <int VID>
 static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
@@ -34,9 +82,9 @@ static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, vo
   } else if constexpr (VID == DYSEL_SGEMM_S128) {
     sgemm_simt_kernel<128, 128, 8, 8, 8><<<(unsigned)ctas, 256, 0, st>>>(g, C, *s);
   } else if constexpr (VID == DYSEL_SGEMM_T128x64) {
-    DYSEL_TRY(launch_tc_sgemm<64>(g, C, *s, (unsigned)ctas, st));
+    DYSEL_TRY(launch_tc<64>(g, C, *s, (unsigned)ctas, st));
   } else {
-    DYSEL_TRY(launch_tc_sgemm<128>(g, C, *s, (unsigned)ctas, st));
+    DYSEL_TRY(launch_tc<128>(g, C, *s, (unsigned)ctas, st));
   }
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
@@ -50,6 +98,11 @@ dysel_status sgemm_register(dysel_ctx *ctx) {
       {"tc3xtf32_128x128", sgemm_variant_fn<3>, {4, 4, 1}, sb, 1, 0, nullptr},
   };
   DYSEL_TRY(tc_sgemm_init());
+  if (cudaFuncSetAttribute(sgemm_tma_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, TmaCfg<64>::SMEM) !=
+          cudaSuccess ||
+      cudaFuncSetAttribute(sgemm_tma_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, TmaCfg<128>::SMEM) !=
+          cudaSuccess)
+    return DYSEL_ERR_CUDA;
   return dysel_register_variants(ctx, kSgemmSig, v, DYSEL_SGEMM_NVARIANTS, DYSEL_SGEMM_S64);
 }
 

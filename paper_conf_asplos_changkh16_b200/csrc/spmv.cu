@@ -407,16 +407,9 @@ template <int VID>
 static void launch_prof(const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p, uint32_t pv, cudaStream_t s) {
   spmv_prof_kernel<VID><<<p.c, kUnitRows, 0, s>>>(A, y, st, p, pv);
 }
-template <int VID>
-static void launch_eager(const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p, int grid, cudaStream_t s) {
-  spmv_eager_kernel<VID><<<grid, kUnitRows, 0, s>>>(A, y, st, p.p_end, p.n_units, p.unit_variant);
-}
 typedef void (*ProfLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, uint32_t, cudaStream_t);
-typedef void (*EagerLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, int, cudaStream_t);
 static const ProfLauncher kProf[DYSEL_SPMV_NVARIANTS] = {launch_prof<0>, launch_prof<1>, launch_prof<2>, launch_prof<3>,
                                                          launch_prof<4>};
-static const EagerLauncher kEager[DYSEL_SPMV_NVARIANTS] = {launch_eager<0>, launch_eager<1>, launch_eager<2>,
-                                                           launch_eager<3>, launch_eager<4>};
 
 }  // namespace dysel
 
@@ -585,9 +578,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       dysel_slice s = unit_slice(p.p_end, p.n_units - p.p_end, p.n_units, pl->vids[i]);
       s.gate = &dst->sel;
       s.variant = i;   // gate compares the pool index
-      SpmvDev Ax = A;
       void *args[2] = {d_y, (void *)d_x};
-      (void)Ax;
       DYSEL_TRY(kVariantFns[pl->vids[i]](&s, args, st, pl));
       DYSEL_TRY(check_launch(ctx, "spmv gated remainder"));
     }
