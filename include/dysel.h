@@ -156,6 +156,9 @@ typedef struct {
   uint32_t *variants_done;   /* completed variants; the last one copies *best into *sel */
   uint32_t n_variants;
   uint32_t score_cycles;     /* 1 => score by cycles/units */
+  uint32_t occupancy;        /* resident CTAs per SM of this variant (0 = unknown); when set and
+                                score_cycles == 0 the score is sum(CTA clock64 cycles) * 64 /
+                                (units * occupancy): time per unit per execution slot (A-6) */
   uint64_t *sel;             /* final packed selection (~0 until profiling completes) */
   /* gated batch: when non-NULL the copy runs only if (*gate & 0xff) == variant */
   const uint64_t *gate;
@@ -177,6 +180,9 @@ typedef struct {
   int n_sandbox_args;
   uint32_t flags;            /* DYSEL_V_* */
   void *user;                /* passed to fn */
+  uint64_t ctas_per_wave;    /* optional: CTAs of this variant resident at once on the device
+                                (occupancy x #SM); 0 = unknown.  When the default variant's full
+                                grid fits in one wave, profiling is off (reading A-3b). */
 } dysel_variant;
 
 /* Register K = n variants under kernel_sig (DySelAddKernel, Fig. 6a

@@ -128,7 +128,10 @@ __device__ __forceinline__ void dysel_prof_end(const dysel_slice &s, dysel_prof_
         const unsigned long long b = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
         const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
         const unsigned long long un = atomicAdd((unsigned long long *)&slot->units, 0ull);
-        unsigned long long score = s.score_cycles ? (un ? cy / un : (1ull << 56) - 1) : (b - a);
+        unsigned long long score =
+            s.score_cycles ? (un ? cy / un : (1ull << 56) - 1)
+            : s.occupancy  ? (un ? cy * 64ull / (un * (unsigned long long)s.occupancy) : (1ull << 56) - 1)
+                           : (b - a);
         if (score > (1ull << 56) - 1) score = (1ull << 56) - 1;
         atomicMin((unsigned long long *)s.best, (score << 8) | (unsigned)s.variant);
         __threadfence();

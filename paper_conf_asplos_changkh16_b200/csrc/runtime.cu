@@ -243,10 +243,22 @@ static dysel_slice base_slice(const Plan &p) {
   return s;
 }
 
-static uint64_t host_score(const dysel_timer_slot &t, bool cycles) {
+// same rule as dysel_prof_end (dysel_device.cuh)
+static uint64_t host_score(const dysel_timer_slot &t, bool cycles, uint32_t occupancy) {
   const uint64_t cap = (1ull << 56) - 1;
-  uint64_t s = cycles ? (t.units ? t.cycles / t.units : cap) : (t.t_end_max - t.t_start_min);
+  uint64_t s = cycles      ? (t.units ? t.cycles / t.units : cap)
+               : occupancy ? (t.units ? t.cycles * 64ull / (t.units * (uint64_t)occupancy) : cap)
+                           : (t.t_end_max - t.t_start_min);
   return std::min(s, cap);
+}
+
+// resident CTAs per SM of variant v, when every variant declares ctas_per_wave
+// (the occupancy-normalised score needs all of them), else 0 (makespan)
+static uint32_t variant_occupancy(const Registered &R, int v, uint32_t mode, int n_sm) {
+  if (mode & DYSEL_SCORE_MAKESPAN) return 0;
+  for (const auto &x : R.v)
+    if (x.ctas_per_wave == 0) return 0;
+  return (uint32_t)std::max<uint64_t>(1, R.v[v].ctas_per_wave / (uint64_t)std::max(1, n_sm));
 }
 
 static void fill_report_common(dysel_report *rep, const Plan &p, int mode_used, int profiled, int selected) {
@@ -498,6 +510,15 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
   Plan P;
   DYSEL_TRY(make_plan(ctx, ndrange_units, wa, K, f, ctx->n_sm, R.def, mode, vflags, &P));
   resolve_pending(ctx, nullptr);
+  if (P.active && !(mode & DYSEL_FORCE_PROFILE) && R.v[R.def].ctas_per_wave > 0) {
+    // reading A-3b: the default variant's whole grid runs in one wave
+    uint64_t def_ctas = 1;
+    for (int d = 0; d < 3; ++d) def_ctas *= (P.U[d] + wa[R.def][d] - 1) / wa[R.def][d];
+    if (def_ctas <= R.v[R.def].ctas_per_wave) {
+      P.active = false;
+      P.c = 0;
+    }
+  }
   cudaStream_t st = (cudaStream_t)stream_v;
   if (rep) rep->n_slices = 0;
   if (P.Gn == 0) {
@@ -584,6 +605,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
     s.variants_done = &ctx->d_prof->variants_done;
     s.n_variants = (uint32_t)K;
     s.score_cycles = score_cycles ? 1u : 0u;
+    s.occupancy = variant_occupancy(R, v, mode, ctx->n_sm);
     s.sel = &ctx->d_prof->sel;
     DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[v], ctx->ev_start, 0));
     DYSEL_TRY(R.v[v].fn(&s, vargs[v].data(), ctx->fork[v], R.v[v].user));
@@ -665,7 +687,9 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
         DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&ctx->h_prof->slot[v], &ctx->d_prof->slot[v], sizeof(dysel_timer_slot),
                                             cudaMemcpyDeviceToHost, ctx->query));
         DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(ctx->query));
-        uint64_t pk = (host_score(ctx->h_prof->slot[v], score_cycles) << 8) | (uint64_t)v;
+        uint64_t pk =
+            (host_score(ctx->h_prof->slot[v], score_cycles, variant_occupancy(R, v, mode, ctx->n_sm)) << 8) |
+            (uint64_t)v;
         if (pk < best_pack) {
           best_pack = pk;
           best_v = v;
@@ -742,7 +766,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
       rep->makespan_ns[v] = t.t_end_max - t.t_start_min;
       rep->units[v] = t.units;
       rep->cycles[v] = t.cycles;
-      rep->score[v] = host_score(t, score_cycles);
+      rep->score[v] = host_score(t, score_cycles, variant_occupancy(R, v, mode, ctx->n_sm));
     }
     rep->host_ns = now_ns() - t_host0;
   }

@@ -91,19 +91,28 @@ static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, vo
 
 dysel_status sgemm_register(dysel_ctx *ctx) {
   static const int sb[1] = {0};
-  dysel_variant v[DYSEL_SGEMM_NVARIANTS] = {
-      {"simt64x64", sgemm_variant_fn<0>, {2, 2, 1}, sb, 1, 0, nullptr},
-      {"simt128x128", sgemm_variant_fn<1>, {4, 4, 1}, sb, 1, 0, nullptr},
-      {"tc3xtf32_128x64", sgemm_variant_fn<2>, {2, 4, 1}, sb, 1, 0, nullptr},
-      {"tc3xtf32_128x128", sgemm_variant_fn<3>, {4, 4, 1}, sb, 1, 0, nullptr},
-  };
   DYSEL_TRY(tc_sgemm_init());
   if (cudaFuncSetAttribute(sgemm_tma_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, TmaCfg<64>::SMEM) !=
           cudaSuccess ||
       cudaFuncSetAttribute(sgemm_tma_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, TmaCfg<128>::SMEM) !=
           cudaSuccess)
     return DYSEL_ERR_CUDA;
-  return dysel_register_variants(ctx, kSgemmSig, v, DYSEL_SGEMM_NVARIANTS, DYSEL_SGEMM_S64);
+  // CTAs resident at once (reading A-3b: a grid within one wave is not profiled)
+  int o[4] = {0, 0, 0, 0};
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[0], sgemm_simt_kernel<64, 64, 16, 4, 4>, 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[1], sgemm_simt_kernel<128, 128, 8, 8, 8>, 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], sgemm_tma_kernel<64>, 192, TmaCfg<64>::SMEM);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[3], sgemm_tma_kernel<128>, 192, TmaCfg<128>::SMEM);
+  cudaGetLastError();
+  const uint64_t n = (uint64_t)ctx->n_sm;
+  dysel_variant v[DYSEL_SGEMM_NVARIANTS] = {
+      {"simt64x64", sgemm_variant_fn<0>, {2, 2, 1}, sb, 1, 0, nullptr, (uint64_t)o[0] * n},
+      {"simt128x128", sgemm_variant_fn<1>, {4, 4, 1}, sb, 1, 0, nullptr, (uint64_t)o[1] * n},
+      {"tc3xtf32_128x64", sgemm_variant_fn<2>, {2, 4, 1}, sb, 1, 0, nullptr, (uint64_t)o[2] * n},
+      {"tc3xtf32_128x128", sgemm_variant_fn<3>, {4, 4, 1}, sb, 1, 0, nullptr, (uint64_t)o[3] * n},
+  };
+  // initial ("default") version on B200: the tensor-core tiling (A-5)
+  return dysel_register_variants(ctx, kSgemmSig, v, DYSEL_SGEMM_NVARIANTS, DYSEL_SGEMM_T128x64);
 }
 
 static dysel_status check_args(dysel_ctx *ctx, int M, int N, int K, const float *A, int lda, const float *B, int ldb,

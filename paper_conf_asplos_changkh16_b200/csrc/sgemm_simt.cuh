@@ -114,7 +114,7 @@ __global__ void __launch_bounds__(256) sgemm_simt_kernel(SgemmArgs g, float *__r
   uint64_t u[3];
   const bool ok = dysel_cta_origin(s, wa, blockIdx.x, u);
   if (ok) simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32);
-  dysel_prof_end(s, psm, ok ? 1u : 0u);
+  dysel_prof_end(s, psm, ok ? wa[0] * wa[1] : 0u);   // units (32x32 tiles) this CTA covered
 }
 
 }  // namespace dysel

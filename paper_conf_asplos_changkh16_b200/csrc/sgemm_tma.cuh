@@ -288,7 +288,7 @@ __global__ void __launch_bounds__(192, 1)
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS));
   }
-  dysel_prof_end(s, psm, 1u);
+  dysel_prof_end(s, psm, wa[0] * wa[1]);   // units (32x32 tiles) this CTA covered
 }
 
 }  // namespace dysel
