@@ -367,6 +367,23 @@ def secondary_workloads(ctx, D, args, stream):
                       "warm_no_profile_us": round(ta * 1e6, 2),
                       "all_us": {k: round(v * 1e6, 2) for k, v in res.items()}}
     plan.destroy()
+    # D6: the paper's Case IV inputs — the scalar/vector flip
+    from workloads import d6_diag, d6_random
+    for name, A6 in (("d6_random_16k_1pct", d6_random()), ("d6_diagonal_2M", d6_diag())):
+        x6 = torch.from_numpy(uniform_f32(6, A6.n_cols)).cuda()
+        rp6, col6, val6 = (torch.from_numpy(a).cuda() for a in (A6.row_ptr, A6.col, A6.val))
+        plan6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_CSR_VECTOR)
+        y6 = torch.empty(A6.n_rows, device="cuda")
+        r6 = {D.SPMV_NAMES[v]: time_b2b(lambda: ctx.spmv_variant(plan6, v, x6, y6), 20, stream)
+              for v in plan6.variant_ids}
+        b6 = min(r6, key=r6.get)
+        t6 = time_b2b(lambda: ctx.spmv(plan6, x6, y6, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE), 20, stream)
+        rep6 = ctx.spmv(plan6, x6, y6, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE, report=True)
+        out[name] = {"best_variant": b6, "best_us": round(r6[b6] * 1e6, 2),
+                     "scalar_over_vector": round(r6["csr_scalar"] / r6["csr_vector"], 3),
+                     "dysel_forced_us": round(t6 * 1e6, 2), "selected": rep6["selected_name"],
+                     "all_us": {k: round(v * 1e6, 2) for k, v in r6.items()}}
+        plan6.destroy()
     # D2m: Parboil-medium SGEMM 1024 x 992 x 1056
     M, K, N = 1024, 992, 1056
     Ah, Bh, _ = sgemm_inputs(M, K, N)

@@ -100,7 +100,8 @@ struct dysel_ctx {
   dysel::ScratchBuf sandbox[2 * DYSEL_MAX_VARIANTS];
   dysel::ScratchBuf unit_variant;    // device bytes, one per granule
   dysel::PendingSel pending[dysel::kPendingRing];
-  uint64_t *h_pending_sel = nullptr;   // pinned, kPendingRing words
+  uint64_t *h_pending_sel = nullptr;   // pinned + mapped, kPendingRing words
+  uint64_t *d_pending_sel = nullptr;   // device alias of h_pending_sel
   int pending_head = 0;
   uint64_t launches = 0;
   uint64_t plan_serial = 0;
@@ -116,6 +117,10 @@ dysel_status scratch(dysel_ctx *ctx, ScratchBuf &b, size_t bytes);
 uint64_t now_ns();
 // enqueue a D2H copy of *d_sel for `sig` on `st`; cache updated when it lands
 dysel_status push_pending_sel(dysel_ctx *ctx, const std::string &sig, const uint64_t *d_sel, cudaStream_t st);
+// device-written variant: reserve a ring slot (its mapped device pointer is
+// handed to the kernel that publishes the selection), then commit after launch
+int reserve_pending_sel(dysel_ctx *ctx, uint64_t **d_slot);
+dysel_status commit_pending_sel(dysel_ctx *ctx, int slot, const std::string &sig, cudaStream_t st);
 // move landed selections into the cache; block_sig != NULL waits for that sig
 void resolve_pending(dysel_ctx *ctx, const char *block_sig);
 // spmv.cu

@@ -54,19 +54,31 @@ uint64_t now_ns() {
       .count();
 }
 
-dysel_status push_pending_sel(dysel_ctx *ctx, const std::string &sig, const uint64_t *d_sel, cudaStream_t st) {
+int reserve_pending_sel(dysel_ctx *ctx, uint64_t **d_slot) {
   int i = ctx->pending_head;
   PendingSel &p = ctx->pending[i];
   if (p.used) {   // ring full: retire the oldest entry first
     cudaEventSynchronize(p.ev);
     resolve_pending(ctx, nullptr);
   }
-  DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&ctx->h_pending_sel[i], d_sel, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  ctx->h_pending_sel[i] = ~0ull;
+  if (d_slot) *d_slot = ctx->d_pending_sel + i;
+  return i;
+}
+
+dysel_status commit_pending_sel(dysel_ctx *ctx, int i, const std::string &sig, cudaStream_t st) {
+  PendingSel &p = ctx->pending[i];
   DYSEL_CUDA_TRY(ctx, cudaEventRecord(p.ev, st));
   p.sig = sig;
   p.used = true;
   ctx->pending_head = (i + 1) % kPendingRing;
   return DYSEL_OK;
+}
+
+dysel_status push_pending_sel(dysel_ctx *ctx, const std::string &sig, const uint64_t *d_sel, cudaStream_t st) {
+  const int i = reserve_pending_sel(ctx, nullptr);
+  DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&ctx->h_pending_sel[i], d_sel, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+  return commit_pending_sel(ctx, i, sig, st);
 }
 
 void resolve_pending(dysel_ctx *ctx, const char *block_sig) {
@@ -352,7 +364,9 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
   if (cudaEventCreateWithFlags(&ctx->ev_fork2, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (cudaMalloc(&ctx->d_prof, sizeof(DevProf)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
   if (cudaMallocHost(&ctx->h_prof, sizeof(DevProf)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
-  if (cudaMallocHost(&ctx->h_pending_sel, kPendingRing * sizeof(uint64_t)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+  if (cudaHostAlloc((void **)&ctx->h_pending_sel, kPendingRing * sizeof(uint64_t), cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostGetDevicePointer((void **)&ctx->d_pending_sel, ctx->h_pending_sel, 0) != cudaSuccess)
+    return fail(DYSEL_ERR_NOMEM);
   for (int i = 0; i < kPendingRing; ++i)
     if (cudaEventCreateWithFlags(&ctx->pending[i].ev, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (spmv_ctx_init(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);

@@ -50,6 +50,7 @@ struct ProfParams {
   uint32_t K, c, n_units, p_end;   // p_end: first remainder unit
   uint32_t hybrid, async, contiguous, score_mode, def, tail, abort;
   uint32_t eager_grid;   // ASYNC: CTAs of the eager kernel (launched by the default's first profiling CTA)
+  uint64_t *host_sel;    // mapped pinned word: the publishing CTA writes the selection here (cache)
   int32_t vids[DYSEL_SPMV_NVARIANTS];
   uint32_t occ[DYSEL_SPMV_NVARIANTS];
   float *sandbox;        // (K-1) * c * 256 floats (hybrid)
@@ -165,12 +166,18 @@ __device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, ui
   s.role = DYSEL_ROLE_BATCH;
   s.variant = vid;
   const unsigned grid = (unsigned)(n_units - u0);
+  // Fire-and-forget, not a tail launch: the remainder depends only on the
+  // selection, so it starts at once, overlapping the drain of the eager CTAs
+  // and of the last profiling CTAs (a tail launch would wait for the whole
+  // parent grid, including its fire-and-forget eager child).  Stream order is
+  // kept: a grid completes only with all its device-launched children.
+  const cudaStream_t ff = cudaStreamFireAndForget;
   switch (vid) {
-    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
-    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
-    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
-    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
-    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, cudaStreamTailLaunch>>>(A, y, s, uv); break;
+    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
+    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
+    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
+    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
+    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
   }
 }
 
@@ -194,14 +201,14 @@ __device__ void eager_launch(int vid, const SpmvDev &A, float *y, SpmvState *st,
   }
 }
 
-// Profiling copy of variant VID (pool index pv): one CTA per profiling unit.
+// One profiling unit of variant VID (pool index pv): the b-th unit of its slice.
 template <int VID>
-__global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
-    spmv_prof_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
+__device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ y, SpmvState *st,
+                                          const ProfParams &p, uint32_t pv, uint32_t b) {
   __shared__ unsigned long long s_last;
   __shared__ int s_abort, s_skip;
   __shared__ dysel_prof_smem psm;
-  const uint32_t tid = threadIdx.x, b = blockIdx.x;
+  const uint32_t tid = threadIdx.x;
   const uint32_t j = p.hybrid ? b : (p.contiguous ? pv * p.c + b : pv + p.K * b);
   const bool productive = !p.hybrid || pv == p.def;
   const bool sandbox = !productive;
@@ -281,6 +288,7 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
   __threadfence();
   const unsigned long long fin = atomicAdd((unsigned long long *)&st->best, 0ull);
   atomicExch((unsigned long long *)&st->sel, fin);
+  if (p.host_sel) *(volatile uint64_t *)p.host_sel = fin;   // activation-flag cache, no D2H copy
   __threadfence();
   // (measured: handing the remainder to the plain kernel beats letting the
   // persistent eager kernel finish it even when the default won)
@@ -292,6 +300,50 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
       tail_launch(p.vids[fin & 0xff], A, y, u0, p.n_units, p.unit_variant);
     }
   }
+}
+
+// Profiling copy of one variant (sequential profiling: one launch per variant).
+template <int VID>
+__global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
+    spmv_prof_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
+  prof_unit<VID>(A, y, st, p, pv, blockIdx.x);
+}
+
+// All K profiling slices in ONE launch (no forked streams / joins): CTA b runs
+// unit b / K of pool variant b mod K (interleaved start order).  The register
+// cap is generous (1 CTA/SM guaranteed) so each variant's code is compiled as
+// in its own kernel; its slice is far below one wave, so occupancy does not
+// shape the measured per-unit time, and the score is normalised by the plain
+// kernel's occupancy anyway.
+__global__ void __launch_bounds__(kUnitRows, 1)
+    spmv_prof_all_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p) {
+  const uint32_t pv = blockIdx.x % p.K, b = blockIdx.x / p.K;
+  switch (p.vids[pv]) {
+    case 0: prof_unit<0>(A, y, st, p, pv, b); break;
+    case 1: prof_unit<1>(A, y, st, p, pv, b); break;
+    case 2: prof_unit<2>(A, y, st, p, pv, b); break;
+    case 3: prof_unit<3>(A, y, st, p, pv, b); break;
+    default: prof_unit<4>(A, y, st, p, pv, b); break;
+  }
+}
+
+// Remainder without a device launch (DYSEL_NO_TAIL, sync): launched by the
+// host right after the profiling kernel on the same stream; every CTA reads
+// the published selection and runs that variant's unit code.
+__global__ void __launch_bounds__(kUnitRows, 4)
+    spmv_remainder_switch_kernel(SpmvDev A, float *__restrict__ y, const SpmvState *st, ProfParams p) {
+  __shared__ int s_vid;
+  if (threadIdx.x == 0) s_vid = p.vids[dysel_ld_acquire_u64(&st->sel) & 0xff];
+  __syncthreads();
+  const uint32_t u = p.p_end + blockIdx.x;
+  switch (s_vid) {
+    case 0: run_unit<0>(A, u, y + (size_t)u * kUnitRows); break;
+    case 1: run_unit<1>(A, u, y + (size_t)u * kUnitRows); break;
+    case 2: run_unit<2>(A, u, y + (size_t)u * kUnitRows); break;
+    case 3: run_unit<3>(A, u, y + (size_t)u * kUnitRows); break;
+    default: run_unit<4>(A, u, y + (size_t)u * kUnitRows); break;
+  }
+  if (p.unit_variant && threadIdx.x == 0) p.unit_variant[u] = (uint8_t)s_vid;
 }
 
 // Eager copy of the default variant (ASYNC): persistent CTAs claim remainder
@@ -552,38 +604,24 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
         (uint32_t)std::min<uint64_t>((uint64_t)std::max(1, cs->occ_eager[dv]) * ctx->n_sm, p.n_units - p.p_end);
     ctx->launches++;   // device-side launch
   }
+  const int pend = reserve_pending_sel(ctx, &p.host_sel);
   spmv_state_init_kernel<<<1, 32, 0, st>>>(dst, pl->K, pl->def);
   DYSEL_TRY(check_launch(ctx, "spmv_state_init_kernel"));
-  DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_start, st));
-  if (sequential) {   // one after another on one profiling stream, default first
-    DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[0], ctx->ev_start, 0));
+  if (sequential) {   // one launch per variant, back to back on the stream, default first
     for (int k = 0; k < pl->K; ++k) {
       const int i = k == 0 ? pl->def : (k <= pl->def ? k - 1 : k);
-      kProf[pl->vids[i]](A, d_y, dst, p, (uint32_t)i, ctx->fork[0]);
+      kProf[pl->vids[i]](A, d_y, dst, p, (uint32_t)i, st);
       DYSEL_TRY(check_launch(ctx, "spmv_prof_kernel"));
     }
-    DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[0], ctx->fork[0]));
-    for (int i = 1; i < pl->K; ++i) DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[i], ctx->fork[0]));
-  } else {
-    for (int i = 0; i < pl->K; ++i) {   // profiling copies first: they get the SMs (and high priority)
-      DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[i], ctx->ev_start, 0));
-      kProf[pl->vids[i]](A, d_y, dst, p, (uint32_t)i, ctx->fork[i]);
-      DYSEL_TRY(check_launch(ctx, "spmv_prof_kernel"));
-      DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[i], ctx->fork[i]));
-    }
+  } else {   // all K profiling slices in one launch on the stream
+    spmv_prof_all_kernel<<<p.K * p.c, kUnitRows, 0, st>>>(A, d_y, dst, p);
+    DYSEL_TRY(check_launch(ctx, "spmv_prof_all_kernel"));
   }
-  for (int i = 0; i < pl->K; ++i) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[i], 0));
-  if (!p.tail && !p.async && p.p_end < p.n_units) {   // NO_TAIL: gated remainder copies of every variant
-    for (int i = 0; i < pl->K; ++i) {
-      dysel_slice s = unit_slice(p.p_end, p.n_units - p.p_end, p.n_units, pl->vids[i]);
-      s.gate = &dst->sel;
-      s.variant = i;   // gate compares the pool index
-      void *args[2] = {d_y, (void *)d_x};
-      DYSEL_TRY(kVariantFns[pl->vids[i]](&s, args, st, pl));
-      DYSEL_TRY(check_launch(ctx, "spmv gated remainder"));
-    }
+  if (!p.tail && !p.async && p.p_end < p.n_units) {   // NO_TAIL: host-launched switch remainder
+    spmv_remainder_switch_kernel<<<p.n_units - p.p_end, kUnitRows, 0, st>>>(A, d_y, dst, p);
+    DYSEL_TRY(check_launch(ctx, "spmv_remainder_switch_kernel"));
   }
-  DYSEL_TRY(push_pending_sel(ctx, pl->sig, &dst->sel, st));
+  DYSEL_TRY(commit_pending_sel(ctx, pend, pl->sig, st));
   if (rep) {
     SpmvState *h = cs->h_state;
     DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(h, dst, sizeof(SpmvState), cudaMemcpyDeviceToHost, st));
