@@ -43,11 +43,13 @@ struct SpmvState {
   uint64_t busy[DYSEL_MAX_VARIANTS];      // sum of unit busy times (ns)
   uint64_t lb[DYSEL_MAX_VARIANTS];        // lower bound of the final busy sum (ns)
   uint64_t aborted[DYSEL_MAX_VARIANTS];   // sandbox units stopped / skipped by dominance
+  uint64_t max_busy[DYSEL_MAX_VARIANTS];  // longest profiled unit (ns)
   dysel_timer_slot slot[DYSEL_MAX_VARIANTS];
 };
 
 struct ProfParams {
   uint32_t K, c, n_units, p_end;   // p_end: first remainder unit
+  uint32_t n_sm;
   uint32_t hybrid, async, contiguous, score_mode, def, tail, abort;
   uint32_t eager_grid;   // ASYNC: CTAs of the eager kernel (launched by the default's first profiling CTA)
   uint64_t *host_sel;    // mapped pinned word: the publishing CTA writes the selection here (cache)
@@ -65,6 +67,7 @@ __global__ void spmv_state_init_kernel(SpmvState *s, int K, int def) {
     s->busy[v] = 0;
     s->lb[v] = 0;
     s->aborted[v] = 0;
+    s->max_busy[v] = 0;
     s->slot[v].t_start_min = ~0ull;
     s->slot[v].t_end_max = 0;
     s->slot[v].units = 0;
@@ -108,21 +111,41 @@ constexpr uint64_t kPollNs = 2000;
 struct SandboxPoll {
   static constexpr bool active = true;
   unsigned long long *s_last;   // smem: last report time
+  const unsigned long long *s_start;   // smem: this unit's start time
   volatile int *s_abort;        // smem
   unsigned long long *lb;
   const uint64_t *best_total;
   uint32_t *dominated;
   const uint64_t *t_start;      // makespan mode: the variant's earliest CTA start
-  uint32_t occ;                 // busy mode: resident CTAs / SM of the variant
+  uint64_t scale_num;           // busy mode: lower bound of the predicted time = lb * num / den
+  uint64_t scale_den;
   uint32_t makespan;
+  // thread-per-row loops: every thread polls (its own loop); warp loops: warp()
   __device__ __forceinline__ bool operator()() const {
     if (*s_abort) return true;
+    return report();
+  }
+  // warp-cooperative loops: only lane 0 reads the timer (cheap for the other
+  // lanes; the caller combines with __any_sync)
+  __device__ __forceinline__ bool warp() const {
+    if (*s_abort) return true;
+    if ((threadIdx.x & 31) != 0) return false;
+    return report();
+  }
+  __device__ __forceinline__ bool report() const {
     const unsigned long long now = dysel_globaltimer();
     const unsigned long long last = *(volatile unsigned long long *)s_last;
     if (now - last < kPollNs) return false;
     if (atomicCAS(s_last, last, now) != last) return *s_abort != 0;   // another thread reports
     const unsigned long long l = atomicAdd(lb, now - last) + (now - last);
-    const unsigned long long cost = makespan ? now - ld_relaxed_u64(t_start) : l * 1024ull / occ;
+    unsigned long long cost;
+    if (makespan) {
+      cost = now - ld_relaxed_u64(t_start);
+    } else {   // predicted full-grid time >= max(throughput bound, this unit's elapsed time)
+      const unsigned long long thr = l * scale_num / scale_den;
+      const unsigned long long el = now - *(volatile const unsigned long long *)s_start;
+      cost = thr > el ? thr : el;
+    }
     if (cost > ld_relaxed_u64(best_total) || ld_relaxed_u32(dominated) != 0) {
       *s_abort = 1;
       atomicExch(dominated, 1u);
@@ -205,10 +228,13 @@ __device__ void eager_launch(int vid, const SpmvDev &A, float *y, SpmvState *st,
 template <int VID>
 __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ y, SpmvState *st,
                                           const ProfParams &p, uint32_t pv, uint32_t b) {
-  __shared__ unsigned long long s_last;
+  __shared__ unsigned long long s_last, s_start;
   __shared__ int s_abort, s_skip;
   __shared__ dysel_prof_smem psm;
   const uint32_t tid = threadIdx.x;
+  // predicted full-grid time of a variant (A-6): max(throughput bound, longest
+  // unit); throughput bound = busy_sum * G_n / (c * occupancy * #SM)
+  const uint64_t thr_den = (uint64_t)p.c * max(1u, p.occ[pv]) * max(1u, p.n_sm);
   const uint32_t j = p.hybrid ? b : (p.contiguous ? pv * p.c + b : pv + p.K * b);
   const bool productive = !p.hybrid || pv == p.def;
   const bool sandbox = !productive;
@@ -216,7 +242,8 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
   if (tid == 0) {
     s_abort = 0;
     s_last = dysel_globaltimer();
-    s_skip = (sandbox && p.abort && ld_relaxed_u32(&st->dominated[pv]) != 0) ? 1 : 0;
+    s_start = s_last;
+    s_skip =(sandbox && p.abort && ld_relaxed_u32(&st->dominated[pv]) != 0) ? 1 : 0;
     if (!s_skip) atomicMin((unsigned long long *)&st->slot[pv].t_start_min, s_last);   // variant start (makespan)
   }
   __syncthreads();
@@ -230,8 +257,9 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     }
     if (sandbox && p.abort)
       run_unit<VID>(A, j, out,
-                    SandboxPoll{&s_last, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total, &st->dominated[pv],
-                                &st->slot[pv].t_start_min, p.occ[pv], p.score_mode == 2 ? 1u : 0u});
+                    SandboxPoll{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
+                                &st->dominated[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
+                                p.score_mode == 2 ? 1u : 0u});
     else
       run_unit<VID>(A, j, out, NoPoll());
     if ((tid & 31) == 0) {
@@ -259,6 +287,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     atomicAdd((unsigned long long *)&slot->cycles, c1 - c0);
     atomicAdd((unsigned long long *)&st->busy[pv], t1 - t0);
     atomicAdd((unsigned long long *)&st->lb[pv], t1 - s_last);   // the rest of this unit's time
+    atomicMax((unsigned long long *)&st->max_busy[pv], t1 - t0);
   }
   if (skipped || s_abort) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
   atomicAdd((unsigned long long *)&slot->units, 1ull);
@@ -272,14 +301,14 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
   const unsigned long long e = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
   const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
   const unsigned long long bz = atomicAdd((unsigned long long *)&st->busy[pv], 0ull);
+  const unsigned long long mb = atomicAdd((unsigned long long *)&st->max_busy[pv], 0ull);
   const bool dom = ld_relaxed_u32(&st->dominated[pv]) != 0;
   const unsigned long long cap = (1ull << 56) - 1;
-  unsigned long long score = p.score_mode == 1 ? cy / p.c
-                             : p.score_mode == 2 ? e - a
-                                                 : bz / ((unsigned long long)p.c * max(1u, p.occ[pv]));
+  const unsigned long long thr = bz * (unsigned long long)p.n_units / thr_den;
+  const unsigned long long pred = thr > mb ? thr : mb;   // predicted full-grid time (ns)
+  unsigned long long score = p.score_mode == 1 ? cy / p.c : p.score_mode == 2 ? e - a : pred;
   if (dom || score > cap) score = cap;
-  if (!dom) atomicMin((unsigned long long *)&st->best_total,
-                      p.score_mode == 2 ? e - a : bz * 1024ull / max(1u, p.occ[pv]));   // dominance units
+  if (!dom) atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
   atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
   __threadfence();
   const uint32_t vd = atomicAdd(&st->variants_done, 1u) + 1u;
@@ -576,6 +605,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.K = (uint32_t)pl->K;
   p.c = (uint32_t)P.c;
   p.n_units = pl->n_units;
+  p.n_sm = (uint32_t)ctx->n_sm;
   p.hybrid = P.mode == DYSEL_HYBRID;
   p.p_end = p.hybrid ? p.c : p.K * p.c;
   p.async = async;
@@ -645,7 +675,9 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       rep->score[id] = h->dominated[v] ? cap
                        : p.score_mode == 1 ? (t.units ? t.cycles / t.units : cap)
                        : p.score_mode == 2 ? rep->makespan_ns[id]
-                                           : (t.units ? h->busy[v] / (t.units * p.occ[v]) : cap);
+                                           : std::max<uint64_t>(h->busy[v] * p.n_units /
+                                                                    ((uint64_t)p.c * p.occ[v] * p.n_sm),
+                                                                h->max_busy[v]);
     }
     if (sel_pool < pl->K) ctx->sel_cache[pl->sig] = sel_pool;
     rep->host_ns = now_ns() - t_host0;

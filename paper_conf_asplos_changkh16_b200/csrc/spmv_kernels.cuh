@@ -60,6 +60,7 @@ struct SpmvDev {
 struct NoPoll {
   static constexpr bool active = false;
   __device__ __forceinline__ bool operator()() const { return false; }
+  __device__ __forceinline__ bool warp() const { return false; }
 };
 
 // ------------------------------------------------------------ load helpers
@@ -157,7 +158,7 @@ __device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, i
     s = __fmaf_rn(v1.y, y1, s);
     s = __fmaf_rn(v1.z, y2, s);
     s = __fmaf_rn(v1.w, y3, s);
-    if (Poll::active && __any_sync(0xffffffffu, poll())) return s;   // warp-uniform exit
+    if (Poll::active && __any_sync(0xffffffffu, poll.warp())) return s;   // warp-uniform exit
   }
   for (; base < body_end; base += 128) {
     const int k0 = base + 4 * lane;
@@ -224,7 +225,7 @@ __device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, fl
 #pragma unroll
     for (int r = 0; r < kRowBatch; ++r)
       if (lane == i0 + r) mine = s[r];
-    if (Poll::active && __any_sync(0xffffffffu, poll())) break;   // warp-uniform exit
+    if (Poll::active && __any_sync(0xffffffffu, poll.warp())) break;   // warp-uniform exit
   }
   if (lane < nr) out[w * 32 + lane] = mine;
 }
@@ -364,7 +365,7 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, fl
       o = open_row(nb);
       oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
     }
-    if (Poll::active && __any_sync(FULL, poll())) break;   // warp-uniform exit
+    if (Poll::active && __any_sync(FULL, poll.warp())) break;   // warp-uniform exit
   }
   float P = part;
 #pragma unroll
