@@ -108,6 +108,8 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
 // (sequential profiling: the variant runs alone) -> time since the variant's
 // first CTA started vs the best completed makespan.
 constexpr uint64_t kPollNs = 2000;
+constexpr long long kPollCycles = 2048;   // ~1 us at 1.9 GHz
+constexpr uint32_t kWarpPollEvery = 4;
 struct SandboxPoll {
   static constexpr bool active = true;
   unsigned long long *s_last;   // smem: last report time
@@ -120,44 +122,71 @@ struct SandboxPoll {
   uint64_t scale_num;           // busy mode: lower bound of the predicted time = lb * num / den
   uint64_t scale_den;
   uint32_t makespan;
+  // %globaltimer reads are slow (measured: polling it every loop step doubled
+  // the per-unit time of CSR-V / CSR-W sandboxes); the per-SM cycle counter
+  // (CS2R) gates them to one per kPollCycles per thread.
+  mutable long long next_clk = 0;
+  __device__ __forceinline__ bool due() const {
+    const long long c = clock64();
+    if (c < next_clk) return false;
+    next_clk = c + kPollCycles;
+    return true;
+  }
   // thread-per-row loops: every thread polls (its own loop); warp loops: warp()
   __device__ __forceinline__ bool operator()() const {
     if (*s_abort) return true;
-    return report();
+    return due() && report();
   }
   // warp-cooperative loops: only lane 0 reads the timer (cheap for the other
   // lanes; the caller combines with __any_sync)
+  // Warp loops call this once per step (~one L2 round trip of work): checking
+  // only every kWarpPollEvery-th step keeps the sandbox's per-unit time close
+  // to the plain kernel's (measured).
+  mutable uint32_t tick = 0;
   __device__ __forceinline__ bool warp() const {
+    if ((++tick & (kWarpPollEvery - 1)) != 0) return false;   // warp-uniform
     if (*s_abort) return true;
     if ((threadIdx.x & 31) != 0) return false;
-    return report();
+    return due() && report();
   }
+  // Global values read by this thread's previous report, issued without waiting
+  // (a blocking global atomic / load per report stalled the polling warp for
+  // ~3 L2 round trips and doubled sandbox unit times).  Stale values stay
+  // safe: lb only grows (a stale lb is still a lower bound) and best_total
+  // only shrinks (a stale best aborts later, never wrongly).
+  mutable unsigned long long lb_seen = 0, best_seen = ~0ull, t0_seen = ~0ull;
+  mutable uint32_t dom_seen = 0;
   __device__ __forceinline__ bool report() const {
     const unsigned long long now = dysel_globaltimer();
     const unsigned long long last = *(volatile unsigned long long *)s_last;
     if (now - last < kPollNs) return false;
     if (atomicCAS(s_last, last, now) != last) return *s_abort != 0;   // another thread reports
-    const unsigned long long l = atomicAdd(lb, now - last) + (now - last);
+    atomicAdd(lb, now - last);   // no return value: a fire-and-forget RED
+    const unsigned long long l = lb_seen + (now - last);
     unsigned long long cost;
     if (makespan) {
-      cost = now - ld_relaxed_u64(t_start);
+      cost = t0_seen == ~0ull ? 0ull : now - t0_seen;
     } else {   // predicted full-grid time >= max(throughput bound, this unit's elapsed time)
       const unsigned long long thr = l * scale_num / scale_den;
       const unsigned long long el = now - *(volatile const unsigned long long *)s_start;
       cost = thr > el ? thr : el;
     }
-    if (cost > ld_relaxed_u64(best_total) || ld_relaxed_u32(dominated) != 0) {
+    if (cost > best_seen || dom_seen != 0) {
       *s_abort = 1;
       atomicExch(dominated, 1u);
       return true;
     }
+    lb_seen = ld_relaxed_u64((const uint64_t *)lb);
+    best_seen = ld_relaxed_u64(best_total);
+    dom_seen = ld_relaxed_u32(dominated);
+    if (makespan) t0_seen = ld_relaxed_u64(t_start);
     return false;
   }
 };
 
 // resident CTAs per SM each plain variant kernel is compiled for (register cap)
 // (CSR-V at 6/SM spills and measured slower on D4: 1.44 vs 1.35 ms)
-constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 6};
+constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 5};
 
 // Plain kernel of one variant over a slice: the exhaustive oracle's pure
 // version, the activation-flag-off path, the tail-launched remainder, the

@@ -34,6 +34,7 @@ constexpr int kUnitRows = 256;
 constexpr int kVecMin = 128;   // CSR-V: rows at least this long use 128-bit loads
 constexpr int kRowBatch = 4;   // CSR-V: rows in flight per warp
 constexpr int kStreamUnroll = 4;   // CSR-W: 32-entry chunks in flight per warp
+constexpr int kStreamLong = 512;   // CSR-W: open-row stretch that switches to 128-bit loads
 
 struct SpmvDev {
   int32_t n_rows, n_cols;
@@ -322,6 +323,38 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, fl
   int oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
   const uint32_t lane_mask_le = (lane == 31) ? FULL : ((2u << lane) - 1u);
   for (int c0 = s; c0 < e; c0 += 32 * kStreamUnroll) {
+    // long stretch of the open row ahead: 128-bit loads, 256 entries per step
+    // (o, oe unchanged: the stretch ends inside the open row)
+    if (A.vec_ok && oe - c0 >= kStreamLong) {
+      const int a = (c0 + 3) & ~3;
+      if (c0 + lane < a) part += ld_stream(A.val + c0 + lane, ps) * ld_x(A.x + ld_stream(A.col + c0 + lane, ps), px);
+      const int body_end = a + ((oe - a) & ~255);
+      bool stop = false;
+      for (int base = a; base < body_end; base += 256) {
+        const int k0 = base + 4 * lane, k1 = k0 + 128;
+        const int4 q0 = ld_stream4(A.col + k0, ps), q1 = ld_stream4(A.col + k1, ps);
+        const float4 v0 = ld_stream4(A.val + k0, ps), v1 = ld_stream4(A.val + k1, ps);
+        const float x0 = ld_x(A.x + q0.x, px), x1 = ld_x(A.x + q0.y, px), x2 = ld_x(A.x + q0.z, px),
+                    x3 = ld_x(A.x + q0.w, px);
+        const float z0 = ld_x(A.x + q1.x, px), z1 = ld_x(A.x + q1.y, px), z2 = ld_x(A.x + q1.z, px),
+                    z3 = ld_x(A.x + q1.w, px);
+        part = __fmaf_rn(v0.x, x0, part);
+        part = __fmaf_rn(v0.y, x1, part);
+        part = __fmaf_rn(v0.z, x2, part);
+        part = __fmaf_rn(v0.w, x3, part);
+        part = __fmaf_rn(v1.x, z0, part);
+        part = __fmaf_rn(v1.y, z1, part);
+        part = __fmaf_rn(v1.z, z2, part);
+        part = __fmaf_rn(v1.w, z3, part);
+        if (Poll::active && __any_sync(FULL, poll.warp())) {
+          stop = true;
+          break;
+        }
+      }
+      if (stop) break;
+      c0 = body_end;
+      if (c0 >= e) break;
+    }
     int cc[kStreamUnroll];
     float vv[kStreamUnroll], pp[kStreamUnroll];
 #pragma unroll

@@ -14,7 +14,8 @@ import weakref
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdysel.so")
+# DYSEL_LIB: an experimental build of the same library (scripts/build_exp.py)
+LIB_PATH = os.environ.get("DYSEL_LIB") or os.path.join(_HERE, "libdysel.so")
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built: run `python -m paper_conf_asplos_changkh16_b200.build` "
                       "(or __graft_entry__.build()); there is no fallback path")
@@ -244,7 +245,7 @@ class Context:
         return int(dysel_kernel_launches(self.h))
 
     # ------------------------------------------------------------- SpMV
-    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ELL | FMT_JDS, default=SPMV_CSR_VECTOR,
+    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ALL, default=SPMV_CSR_VECTOR,
                      stream=None) -> SpmvPlan:
         n = row_ptr.numel() - 1
         nnz = col.numel()
