@@ -153,7 +153,8 @@ METRIC = "DySel SpMV GB/s (power-law 1e7 rows, profiling on every call) + overhe
 def config(A, world):
     return {"workload": "D4 power-law SpMV: 10^7 rows, p(L)~L^-1.761 on [1,16384], uniform cols, fp32 CSR",
             "n_rows": int(A.n_rows), "nnz": int(A.nnz), "parallelism": f"row-shard{world}",
-            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": "AUTO|ASYNC (hybrid), f=0.005"}
+            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": "AUTO|ASYNC (hybrid), f=0.005",
+            "default_variant": "DYSEL_SPMV_DEFAULT_AUTO (A-30)"}
 
 
 # ------------------------------------------------------------------ timing
@@ -193,7 +194,8 @@ def dysel_arm(args, world, rank, local_rank):
     xd = torch.from_numpy(x).to(dev)
     y = torch.empty(A.n_rows, device=dev)
     stream = torch.cuda.current_stream()
-    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_CSR_VECTOR)
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO)
+    default_name = D.SPMV_NAMES[plan.info.default_variant]
     mode = D.AUTO | D.ASYNC
     f = args.f
 
@@ -253,6 +255,20 @@ def dysel_arm(args, world, rank, local_rank):
             ctx.spmv(plan, xd, yl, mode=D.NO_PROFILE)
     ta = float(np.median(time_events(amort, 3, stream))) / I
     # ---- e2e through the public API with host buffers: x H2D, y D2H per step
+    # ---- ablations (rank 0, 1 GPU): sync mode, a non-best default, f
+    ablation = {}
+    if world == 1 and not args.no_secondary:
+        ablation["sync_overhead_pct"] = round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=D.AUTO), 10, stream)
+                                               / T_star - 1) * 100, 2)
+        ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10, stream)
+                                                      / T_star - 1) * 100, 2) for ff in (0.001, 0.002, 0.01, 0.02)}
+        for dname, dv in (("csr_vector", D.SPMV_CSR_VECTOR), ("jds", D.SPMV_JDS)):
+            pd = ctx.spmv_prepare(rp, col, val, A.n_cols, default=dv)
+            td = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode), 10, stream)
+            rd = ctx.spmv(pd, xd, yl, f=f, mode=mode, report=True)
+            ablation[f"default_{dname}"] = {"overhead_pct": round((td / T_star - 1) * 100, 2),
+                                            "selected": rd["selected_name"], "eager_units": rd["eager_units"]}
+            pd.destroy()
     xh = torch.from_numpy(x).pin_memory()
     yh = torch.empty(r1 - r0, dtype=torch.float32).pin_memory()
     def e2e_step():
@@ -295,6 +311,7 @@ def dysel_arm(args, world, rank, local_rank):
             "warmup": args.warmup, "ms_per_step": round(T_step * 1e3, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": config(A, world),
+            "default_variant": default_name,
             "overhead_pct_vs_best_variant": round((T_step - T_star) / T_star * 100, 3) if world == 1 else None,
             "best_variant_oracle": {"variant": best_name, "ms": round(T_star * 1e3, 4),
                                     "gbs": round(nbytes_total / T_star / 1e9, 2),
@@ -302,7 +319,7 @@ def dysel_arm(args, world, rank, local_rank):
             "selected": rep["selected_name"], "selection_matches_oracle": rep["selected_name"] == best_name,
             "mode_used": rep["mode_used"], "profiled_units_per_variant": rep["c"],
             "amortized_overhead_pct": round((ta - T_star) / T_star * 100, 3) if world == 1 else None,
-            "amortized_iters": I,
+            "amortized_iters": I, "ablation": ablation,
             "e2e": {"value": round(nbytes_total / T_e2e / 1e9, 3), "unit": "GB/s",
                     "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int((r1 - r0) * 4),
                     "ms_per_step": round(T_e2e * 1e3, 4)},
@@ -310,10 +327,11 @@ def dysel_arm(args, world, rank, local_rank):
                      "aborted_sandbox_units": {D.SPMV_NAMES[v]: rep["aborted"][v] for v in plan.variant_ids},
                      "busy_us_per_unit": {D.SPMV_NAMES[v]: round(rep["busy_ns"][v] / max(1, rep["units"][v]) / 1e3, 2)
                                           for v in plan.variant_ids},
-                     "kernels": "init + K profiling kernels + eager(default) + tail-launched remainder"},
+                     "kernels": "init + one profiling kernel (K variants) + K claim kernels (PDL-chained, "
+                                "default first: eager, then the winner's remainder)"},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": pk["hbm_gbs"], "unit": "GB/s",
                          "frac": round(achieved / pk["hbm_gbs"], 4), "traffic": traffic,
-                         "kernel": f"dysel::spmv_slice_kernel<{sel_name}> (full grid, event-timed)",
+                         "kernel": f"dysel::spmv_claim_kernel<{sel_name}> (pure full grid, event-timed back to back)",
                          "peak_source": src,
                          "note": "D4 gathers x at uniform-random columns: bound in practice by the L1TEX/L2 "
                                  "random-sector rate (DESIGN.md §Roofline), not HBM"},
@@ -333,7 +351,7 @@ def secondary_workloads(ctx, D, args, stream):
     A = d3_fem()
     x = torch.from_numpy(uniform_f32(384, A.n_cols)).cuda()
     rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
-    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_CSR_VECTOR)
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO)
     y = torch.empty(A.n_rows, device="cuda")
     nb = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -364,6 +382,7 @@ def secondary_workloads(ctx, D, args, stream):
                       "best_gbs": round(nb / res[best] / 1e9, 1), "dysel_us": round(td * 1e6, 2),
                       "dysel_gbs": round(nb / td / 1e9, 1), "overhead_pct": round((td / res[best] - 1) * 100, 2),
                       "selected": rep["selected_name"], "profiled": rep["profiled"],
+                      "default_variant": D.SPMV_NAMES[plan.info.default_variant],
                       "warm_no_profile_us": round(ta * 1e6, 2),
                       "all_us": {k: round(v * 1e6, 2) for k, v in res.items()}}
     plan.destroy()
@@ -372,7 +391,7 @@ def secondary_workloads(ctx, D, args, stream):
     for name, A6 in (("d6_random_16k_1pct", d6_random()), ("d6_diagonal_2M", d6_diag())):
         x6 = torch.from_numpy(uniform_f32(6, A6.n_cols)).cuda()
         rp6, col6, val6 = (torch.from_numpy(a).cuda() for a in (A6.row_ptr, A6.col, A6.val))
-        plan6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_CSR_VECTOR)
+        plan6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_DEFAULT_AUTO)
         y6 = torch.empty(A6.n_rows, device="cuda")
         r6 = {D.SPMV_NAMES[v]: time_b2b(lambda: ctx.spmv_variant(plan6, v, x6, y6), 20, stream)
               for v in plan6.variant_ids}

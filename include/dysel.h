@@ -83,10 +83,14 @@ const char *dysel_status_str(dysel_status s);
 #define DYSEL_CONTIGUOUS 64u    /* fully mode: contiguous per-variant slices instead of interleaved granules (A-24) */
 #define DYSEL_SCORE_CYCLES 128u /* score = sum of per-CTA clock64 cycles / units (A-6) */
 #define DYSEL_SCORE_MAKESPAN 256u /* score = latest CTA end - earliest CTA start (%globaltimer), Fig. 7b */
-#define DYSEL_NO_TAIL 512u      /* SpMV device path: run the remainder inside the dispatcher (no CDP2 tail launch) */
+#define DYSEL_NO_TAIL 512u      /* SpMV device path: the remainder kernel waits for the profiling kernel to
+                                   complete (stream order) instead of starting beside it (PDL) / no CDP2 tail */
 #define DYSEL_NO_ABORT 1024u    /* SpMV device path: never stop dominated sandbox units early */
 #define DYSEL_SEQUENTIAL 2048u  /* SpMV device path: profile the variants one after another, each alone on the
                                    GPU (default variant first), scored by makespan (reading A-23) */
+#define DYSEL_DEVICE_LAUNCH 4096u /* SpMV device path, round-1 scheme (ablation): eager kernel and remainder
+                                     launched from the device (CDP2 fire-and-forget) instead of the
+                                     host-launched PDL work kernel */
 /* Default score: generic launcher = makespan (variants are separate concurrent
  * grids, Fig. 7b); SpMV dispatcher = mean per-unit busy time (%globaltimer end -
  * start of each profiled unit; all variants share one launch and occupancy). */
@@ -219,6 +223,12 @@ typedef struct {
   uint8_t *unit_variant;    /* optional caller HOST array, one byte per granule: variant that
                                productively computed it (debug / c-6 tests; costs a D2H copy + sync) */
   uint64_t unit_variant_cap;
+  /* SpMV device path, filled only when a report is requested (diagnostics):
+   * ns since the first profiling CTA started — [0] 0, [1] selection
+   * published, [2] last profiling CTA ended, [3] first eager CTA started,
+   * [4] last eager CTA ended, [5] first remainder CTA started, [6] last
+   * remainder CTA ended, [7] longest profiling unit (ns); ~0 = did not happen. */
+  uint64_t timeline_ns[8];
 } dysel_report;
 
 /* Launch kernel_sig over an NDRange of ndrange_units[3] units
@@ -249,6 +259,11 @@ dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key); /* NULL key
  * (warp-streaming CSR with a warp-level segmented reduction; B200 addition). */
 enum { DYSEL_SPMV_CSR_SCALAR = 0, DYSEL_SPMV_CSR_VECTOR = 1, DYSEL_SPMV_ELL = 2, DYSEL_SPMV_JDS = 3,
        DYSEL_SPMV_CSR_STREAM = 4, DYSEL_SPMV_NVARIANTS = 5 };
+/* default_variant = DYSEL_SPMV_DEFAULT_AUTO: the library picks the initial
+ * version from the prepare-time row statistics (reading A-30): uniform rows
+ * (A-13) -> ELL when in the pool; otherwise CSR-W when in the pool, else
+ * CSR-V.  The choice is visible in dysel_spmv_plan_info.default_variant. */
+#define DYSEL_SPMV_DEFAULT_AUTO (-1)
 #define DYSEL_FMT_STREAM 4u   /* include CSR-W in the pool (reads the CSR arrays directly) */
 #define DYSEL_FMT_ELL 1u
 #define DYSEL_FMT_JDS 2u
@@ -264,6 +279,7 @@ typedef struct {
   int32_t max_row_len;
   uint64_t prep_ns;              /* device time of format preparation (a-1) */
   uint64_t ell_bytes, jds_bytes; /* extra device memory held by the plan */
+  int32_t default_variant;       /* DYSEL_SPMV_* id of the initial version (resolved when AUTO) */
 } dysel_spmv_plan_info;
 
 /* Build the variant pool for one CSR matrix: CSR -> ELL and CSR -> block JDS
@@ -271,7 +287,8 @@ typedef struct {
  * [nnz] (sorted or not), d_val fp32 [nnz]; nnz < 2^31.  formats_mask selects
  * which extra formats to build (DYSEL_FMT_*); ELL is skipped (and absent from
  * the pool) when W * n_rows > 4 * nnz.  default_variant is a DYSEL_SPMV_* id
- * (must be in the pool).  Blocks on `stream` (reads back sizes). */
+ * (must be in the pool) or DYSEL_SPMV_DEFAULT_AUTO.  Blocks on `stream` (reads
+ * back sizes). */
 dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, int64_t nnz,
                                 const int32_t *d_row_ptr, const int32_t *d_col, const float *d_val,
                                 uint32_t formats_mask, int default_variant, void *stream,
@@ -356,6 +373,14 @@ dysel_status dysel_timer_calibrate(dysel_ctx *ctx, uint64_t samples, uint64_t sp
 /* Known-cost test variants (c-8): registers sig with n variants whose CTAs
  * spin cost_ns[v] per unit (wa = 1) and write out[u] = v+1 for each unit u
  * (args[0] = uint32_t* out).  Used to check selection end to end. */
+/* Launch-path experiment: the full grid of one SpMV pool variant launched
+ * from the host (how = 0), from the device fire-and-forget (1) or as a device
+ * tail launch (2) by a one-thread parent kernel, stream-ordered on `stream`.
+ * h_resident_max (nullable, n_sm entries, HOST): the maximum number of CTAs
+ * resident at once on each SM (measured with %smid counters; blocks). */
+dysel_status dysel_debug_spmv_device_launch(dysel_ctx *ctx, dysel_spmv_plan *plan, int variant_id,
+                                            const float *d_x, float *d_y, int how, void *stream,
+                                            uint32_t *h_resident_max, int n_sm);
 dysel_status dysel_register_spin_variants(dysel_ctx *ctx, const char *sig, const uint32_t *cost_ns, int n,
                                           int default_variant);
 

@@ -18,6 +18,7 @@
 //      the tail launch, so eager work stops and the winner takes over.
 // Hybrid sandbox units of a provably losing variant stop early (dominance).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "dysel_device.cuh"
@@ -31,7 +32,12 @@ namespace dysel {
 // will run the remainder.  DYSEL_SCORE_CYCLES: sum clock64 / units.
 // DYSEL_SCORE_MAKESPAN: the paper's earliest start .. latest end (Fig. 7b).
 struct SpmvState {
-  uint32_t ticket;          // eager / remainder tickets
+  uint32_t ticket;          // CDP scheme: eager / remainder tickets (units)
+  uint32_t c2;              // claim kernels: remainder slot tickets after the selection (slot S + c2)
+  uint64_t c1;              // claim kernels: eager slot tickets (low 32 bits) | published (bit 32)
+  uint64_t sw;              // claim kernels: (S << 8) | selected pool index, ~0 until published
+  uint64_t pure_ctr;        // pure full-grid runs: slot tickets; the last warp of a run resets both
+  uint32_t pure_done;       // pure full-grid runs: warps finished
   uint32_t variants_done;
   uint64_t best;            // (score << 8) | pool variant
   uint64_t sel;             // final packed selection, ~0 until published
@@ -45,6 +51,10 @@ struct SpmvState {
   uint64_t aborted[DYSEL_MAX_VARIANTS];   // sandbox units stopped / skipped by dominance
   uint64_t max_busy[DYSEL_MAX_VARIANTS];  // longest profiled unit (ns)
   dysel_timer_slot slot[DYSEL_MAX_VARIANTS];
+  // diagnostics timeline (absolute %globaltimer ns; dysel_report.timeline_ns):
+  // 0 prof start (min), 1 publish, 2 prof end (max), 3/4 eager start/end,
+  // 5/6 remainder start/end, 7 longest profiling unit
+  uint64_t tl[8];
 };
 
 struct ProfParams {
@@ -56,7 +66,10 @@ struct ProfParams {
   int32_t vids[DYSEL_SPMV_NVARIANTS];
   uint32_t occ[DYSEL_SPMV_NVARIANTS];
   float *sandbox;        // (K-1) * c * 256 floats (hybrid)
+  uint64_t *tl;          // SpmvState::tl when a report is requested, else nullptr (no timeline atomics)
   uint8_t *unit_variant; // optional debug map (variant id per unit)
+  uint32_t pure;         // pure full-grid run of one variant (self-resetting counters, no init kernel)
+  uint32_t k_claim;      // claim kernels: max slots per claim (~kClaimNnz nonzeros of work)
 };
 
 __global__ void spmv_state_init_kernel(SpmvState *s, int K, int def) {
@@ -73,8 +86,12 @@ __global__ void spmv_state_init_kernel(SpmvState *s, int K, int def) {
     s->slot[v].units = 0;
     s->slot[v].cycles = 0;
   }
+  if (v < 8) s->tl[v] = (v == 0 || v == 3 || v == 5) ? ~0ull : 0ull;
   if (v == 0) {
     s->ticket = 0;
+    s->c2 = 0;
+    s->c1 = 0;
+    s->sw = ~0ull;
     s->variants_done = 0;
     s->best = (((1ull << 56) - 1) << 8) | (uint64_t)def;
     s->sel = ~0ull;
@@ -187,24 +204,65 @@ struct SandboxPoll {
 // resident CTAs per SM each plain variant kernel is compiled for (register cap)
 // (CSR-V at 6/SM spills and measured slower on D4: 1.44 vs 1.35 ms)
 constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 5};
+constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
+// claim kernels: CTAs per SM (CSR-S / ELL at 8 spilled ~200 B in the claim loop)
+constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {6, 4, 6, 6, 5};
 
 // Plain kernel of one variant over a slice: the exhaustive oracle's pure
 // version, the activation-flag-off path, the tail-launched remainder, the
 // gated remainder (NO_TAIL) and the host path's copies (dysel_device.cuh
 // timing / gating).
+//
+// No static shared memory: the kernel's occupancy must not depend on the
+// L1 / shared-memory carveout.  Measured on D4: with the 1 KB timing buffer
+// in this kernel, the smallest carveout (which device-side launches get, and
+// cudaSharedmemCarveoutMaxL1 asks for) cut CSR-W's resident CTAs and ran
+// 1.52 ms instead of 0.93 ms; a large carveout shrinks L1 (fewer gathers in
+// flight) and ran 2.25 ms.  Timed copies (host path) use spmv_slice_timed_kernel.
+// diagnostics: resident CTAs per SM (current, max) of timeline-instrumented launches
+__device__ uint32_t g_resident[2][1024];
+
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
-    spmv_slice_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s, uint8_t *uv) {
+    spmv_slice_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s, uint8_t *uv, uint64_t *tl) {
+  if (!dysel_gate_open(s)) return;
+  if (tl && threadIdx.x == 0) {
+    atomicMin((unsigned long long *)&tl[5], (unsigned long long)dysel_globaltimer());
+    const uint32_t sm = smid() & 1023;
+    atomicMax(&g_resident[1][sm], atomicAdd(&g_resident[0][sm], 1u) + 1u);
+  }
+  const uint32_t j = (uint32_t)(s.granule_begin + (uint64_t)blockIdx.x * s.granule_stride);
+  run_unit<VID>(A, j, y + (size_t)j * kUnitRows);
+  if (uv && threadIdx.x == 0) uv[j] = (uint8_t)VID;
+  if (tl) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      atomicMax((unsigned long long *)&tl[6], (unsigned long long)dysel_globaltimer());
+      atomicSub(&g_resident[0][smid() & 1023], 1u);
+    }
+  }
+}
+
+// Timed copy (generic launcher / paper host path: s.timer set, Fig. 7b).
+template <int VID>
+__global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
+    spmv_slice_timed_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s) {
   __shared__ dysel_prof_smem psm;
   if (!dysel_gate_open(s)) return;
   dysel_prof_begin(s, psm);
   const uint32_t j = (uint32_t)(s.granule_begin + (uint64_t)blockIdx.x * s.granule_stride);
   run_unit<VID>(A, j, y + (size_t)j * kUnitRows);
-  if (uv && threadIdx.x == 0) uv[j] = (uint8_t)VID;
   dysel_prof_end(s, psm, 1u);
 }
 
-__device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, uint64_t n_units, uint8_t *uv) {
+__device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, uint64_t n_units, uint8_t *uv,
+                            uint64_t *tl) {
   dysel_slice s;
   memset(&s, 0, sizeof(s));
   s.granule_begin = u0;
@@ -225,17 +283,47 @@ __device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, ui
   // kept: a grid completes only with all its device-launched children.
   const cudaStream_t ff = cudaStreamFireAndForget;
   switch (vid) {
-    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
-    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
-    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
-    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
-    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv); break;
+    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
+    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
+    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
+    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
+    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
   }
 }
 
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
-    spmv_eager_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, uint32_t p_end, uint32_t n_units, uint8_t *uv);
+    spmv_eager_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, uint32_t p_end, uint32_t n_units, uint8_t *uv,
+                      uint64_t *tl);
+
+// Debug (dysel_debug_spmv_device_launch): one thread launches the full grid of
+// a variant from the device, fire-and-forget (how = 1) or as a tail launch (2).
+__global__ void spmv_device_launch_kernel(SpmvDev A, float *y, int vid, uint64_t n_units, int how, uint64_t *tl) {
+  if (how == 1) {
+    tail_launch(vid, A, y, 0, n_units, nullptr, tl);
+    return;
+  }
+  dysel_slice s;
+  memset(&s, 0, sizeof(s));
+  s.granule_count = n_units;
+  s.granule_stride = 1;
+  s.g[0] = s.g[1] = s.g[2] = 1;
+  s.G[0] = (uint32_t)n_units;
+  s.G[1] = s.G[2] = 1;
+  s.U[0] = n_units;
+  s.U[1] = s.U[2] = 1;
+  s.role = DYSEL_ROLE_BATCH;
+  s.variant = vid;
+  const unsigned grid = (unsigned)n_units;
+  const cudaStream_t ts = cudaStreamTailLaunch;
+  switch (vid) {
+    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
+    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
+    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
+    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
+    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
+  }
+}
 
 // The eager grid is launched from the device (fire-and-forget child of the
 // default variant's first profiling CTA), so it can only start once profiling
@@ -245,16 +333,20 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
 __device__ void eager_launch(int vid, const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p) {
   const unsigned g = p.eager_grid;
   switch (vid) {
-    case 0: spmv_eager_kernel<0><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
-    case 1: spmv_eager_kernel<1><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
-    case 2: spmv_eager_kernel<2><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
-    case 3: spmv_eager_kernel<3><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
-    default: spmv_eager_kernel<4><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant); break;
+    case 0: spmv_eager_kernel<0><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 1: spmv_eager_kernel<1><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 2: spmv_eager_kernel<2><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 3: spmv_eager_kernel<3><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    default: spmv_eager_kernel<4><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
   }
 }
 
 // One profiling unit of variant VID (pool index pv): the b-th unit of its slice.
-template <int VID>
+// CDP: the round-1 scheme (DYSEL_DEVICE_LAUNCH) whose eager kernel and
+// remainder are launched from here; the default instantiation contains no
+// device-side launch (a grid that can launch children does not release
+// programmatic dependents early: measured, the PDL remainder waited for it).
+template <int VID, bool CDP>
 __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ y, SpmvState *st,
                                           const ProfParams &p, uint32_t pv, uint32_t b) {
   __shared__ unsigned long long s_last, s_start;
@@ -265,26 +357,36 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
   // unit); throughput bound = busy_sum * G_n / (c * occupancy * #SM)
   const uint64_t thr_den = (uint64_t)p.c * max(1u, p.occ[pv]) * max(1u, p.n_sm);
   const uint32_t j = p.hybrid ? b : (p.contiguous ? pv * p.c + b : pv + p.K * b);
-  const bool productive = !p.hybrid || pv == p.def;
+  // hybrid (reading A-4'): every variant runs the shared units into its own
+  // sandbox and may be stopped by dominance; the winner's sandbox is copied
+  // into y when the selection is published, so its profiled work is the
+  // productive one (never recomputed) whichever variant wins
+  const bool productive = !p.hybrid;
   const bool sandbox = !productive;
-  if (tid == 0 && b == 0 && pv == p.def && p.eager_grid) eager_launch(p.vids[p.def], A, y, st, p);
+  if constexpr (CDP)
+    if (tid == 0 && b == 0 && pv == p.def && p.eager_grid) eager_launch(p.vids[p.def], A, y, st, p);
   if (tid == 0) {
     s_abort = 0;
     s_last = dysel_globaltimer();
     s_start = s_last;
     s_skip =(sandbox && p.abort && ld_relaxed_u32(&st->dominated[pv]) != 0) ? 1 : 0;
     if (!s_skip) atomicMin((unsigned long long *)&st->slot[pv].t_start_min, s_last);   // variant start (makespan)
+    if (p.tl) atomicMin((unsigned long long *)&p.tl[0], s_last);
   }
   __syncthreads();
   const bool skipped = s_skip != 0;
-  float *out = productive ? y + (size_t)j * kUnitRows
-                          : p.sandbox + ((size_t)(pv < p.def ? pv : pv - 1) * p.c + b) * kUnitRows;
+  float *out = productive ? y + (size_t)j * kUnitRows : p.sandbox + ((size_t)pv * p.c + b) * kUnitRows;
   if (!skipped) {
     if ((tid & 31) == 0) {
       psm.c0[tid >> 5] = dysel_clock64();
       psm.t0[tid >> 5] = dysel_globaltimer();
     }
-    if (sandbox && p.abort)
+    // Dominance polling only in the thread-per-row variants (a single long
+    // row makes their units take milliseconds); the warp-cooperative ones
+    // (CSR-V, CSR-W) finish any unit in tens of us, and polling inside their
+    // loops measured +60% per-unit time on D4 (CSR-W 15 -> 24.6 us).
+    constexpr bool kPolled = VID == 0 || VID == 2 || VID == 3;
+    if (kPolled && sandbox && p.abort)
       run_unit<VID>(A, j, out,
                     SandboxPoll{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
                                 &st->dominated[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
@@ -308,54 +410,84 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     c0 = min(c0, __shfl_xor_sync(0xffffffffu, c0, o));
     c1 = max(c1, __shfl_xor_sync(0xffffffffu, c1, o));
   }
-  if (tid != 0) return;
-  dysel_timer_slot *slot = &st->slot[pv];
-  if (!skipped) {
-    atomicMin((unsigned long long *)&slot->t_start_min, t0);
-    atomicMax((unsigned long long *)&slot->t_end_max, t1);
-    atomicAdd((unsigned long long *)&slot->cycles, c1 - c0);
-    atomicAdd((unsigned long long *)&st->busy[pv], t1 - t0);
-    atomicAdd((unsigned long long *)&st->lb[pv], t1 - s_last);   // the rest of this unit's time
-    atomicMax((unsigned long long *)&st->max_busy[pv], t1 - t0);
+  bool publish = false;
+  unsigned long long fin = 0;
+  if (tid == 0) {
+    dysel_timer_slot *slot = &st->slot[pv];
+    if (!skipped) {
+      atomicMin((unsigned long long *)&slot->t_start_min, t0);
+      atomicMax((unsigned long long *)&slot->t_end_max, t1);
+      atomicAdd((unsigned long long *)&slot->cycles, c1 - c0);
+      atomicAdd((unsigned long long *)&st->busy[pv], t1 - t0);
+      atomicAdd((unsigned long long *)&st->lb[pv], t1 - s_last);   // the rest of this unit's time
+      atomicMax((unsigned long long *)&st->max_busy[pv], t1 - t0);
+      if (p.tl) atomicMax((unsigned long long *)&p.tl[7], t1 - t0);
+    }
+    if (p.tl) atomicMax((unsigned long long *)&p.tl[2], dysel_globaltimer());
+    if (skipped || s_abort) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
+    atomicAdd((unsigned long long *)&slot->units, 1ull);
+    if (productive && p.unit_variant) p.unit_variant[j] = (uint8_t)VID;
+    __threadfence();
+    const uint32_t done = atomicAdd(&st->ctas_done[pv], 1u) + 1u;
+    if (done == p.c) {
+      // ---- variant complete: score, packed atomicMin (A-7, A-8)
+      __threadfence();
+      const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
+      const unsigned long long e = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
+      const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
+      const unsigned long long bz = atomicAdd((unsigned long long *)&st->busy[pv], 0ull);
+      const unsigned long long mb = atomicAdd((unsigned long long *)&st->max_busy[pv], 0ull);
+      const bool dom = ld_relaxed_u32(&st->dominated[pv]) != 0;
+      const unsigned long long cap = (1ull << 56) - 1;
+      const unsigned long long thr = bz * (unsigned long long)p.n_units / thr_den;
+      const unsigned long long pred = thr > mb ? thr : mb;   // predicted full-grid time (ns)
+      unsigned long long score = p.score_mode == 1 ? cy / p.c : p.score_mode == 2 ? e - a : pred;
+      if (dom || score > cap) score = cap;
+      if (!dom) atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
+      atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
+      __threadfence();
+      const uint32_t vd = atomicAdd(&st->variants_done, 1u) + 1u;
+      if (vd == p.K) {
+        // ---- last variant: publish the selection, hand the remainder to the winner
+        __threadfence();
+        fin = atomicAdd((unsigned long long *)&st->best, 0ull);
+        publish = true;
+      }
+    }
   }
-  if (skipped || s_abort) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
-  atomicAdd((unsigned long long *)&slot->units, 1ull);
-  if (productive && p.unit_variant) p.unit_variant[j] = (uint8_t)VID;
-  __threadfence();
-  const uint32_t done = atomicAdd(&st->ctas_done[pv], 1u) + 1u;
-  if (done != p.c) return;
-  // ---- variant complete: score, packed atomicMin (A-7, A-8)
-  __threadfence();
-  const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
-  const unsigned long long e = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
-  const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
-  const unsigned long long bz = atomicAdd((unsigned long long *)&st->busy[pv], 0ull);
-  const unsigned long long mb = atomicAdd((unsigned long long *)&st->max_busy[pv], 0ull);
-  const bool dom = ld_relaxed_u32(&st->dominated[pv]) != 0;
-  const unsigned long long cap = (1ull << 56) - 1;
-  const unsigned long long thr = bz * (unsigned long long)p.n_units / thr_den;
-  const unsigned long long pred = thr > mb ? thr : mb;   // predicted full-grid time (ns)
-  unsigned long long score = p.score_mode == 1 ? cy / p.c : p.score_mode == 2 ? e - a : pred;
-  if (dom || score > cap) score = cap;
-  if (!dom) atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
-  atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
-  __threadfence();
-  const uint32_t vd = atomicAdd(&st->variants_done, 1u) + 1u;
-  if (vd != p.K) return;
-  // ---- last variant: publish the selection, hand the remainder to the winner
-  __threadfence();
-  const unsigned long long fin = atomicAdd((unsigned long long *)&st->best, 0ull);
+  publish = __shfl_sync(0xffffffffu, publish ? 1 : 0, 0) != 0;
+  if (!publish) return;
+  fin = __shfl_sync(0xffffffffu, fin, 0);
+  const uint32_t win = (uint32_t)(fin & 0xff);
+  if (p.hybrid) {   // the winner's profiled units become the productive ones (warp 0 copies)
+    const size_t n = min((size_t)p.c * kUnitRows, (size_t)A.n_rows);
+    const float *src = p.sandbox + (size_t)win * p.c * kUnitRows;
+    const size_t n4 = n / 4;
+    for (size_t q = tid; q < n4; q += 32) reinterpret_cast<float4 *>(y)[q] = reinterpret_cast<const float4 *>(src)[q];
+    for (size_t q = n4 * 4 + tid; q < n; q += 32) y[q] = src[q];
+    if (p.unit_variant)
+      for (uint32_t u = tid; u < p.c; u += 32) p.unit_variant[u] = (uint8_t)p.vids[win];
+    __syncwarp();
+    __threadfence();
+  }
+  if (tid != 0) return;
   atomicExch((unsigned long long *)&st->sel, fin);
+  {   // claim kernels: close the eager ticket range; the default keeps whole
+      // units only, so the switch point S is rounded up to a unit boundary
+    const uint64_t old = atomicOr((unsigned long long *)&st->c1, 1ull << 32);
+    const uint64_t n_slots = (uint64_t)(p.n_units - p.p_end) * kSlots;
+    const uint64_t S = min(((uint64_t)(uint32_t)old + kSlots - 1) / kSlots * kSlots, n_slots);
+    atomicExch((unsigned long long *)&st->sw, (S << 8) | win);
+  }
   if (p.host_sel) *(volatile uint64_t *)p.host_sel = fin;   // activation-flag cache, no D2H copy
+  if (p.tl) p.tl[1] = dysel_globaltimer();
   __threadfence();
-  // (measured: handing the remainder to the plain kernel beats letting the
-  // persistent eager kernel finish it even when the default won)
-  if (p.tail) {
+  if (CDP && p.tail) {
     const uint32_t old = p.async ? atomicAdd(&st->ticket, 1u << 30) : 0u;   // stop eager claims
     const uint64_t u0 = (uint64_t)p.p_end + old;
     if (u0 < p.n_units) {
       st->tail_begin = u0;
-      tail_launch(p.vids[fin & 0xff], A, y, u0, p.n_units, p.unit_variant);
+      if constexpr (CDP) tail_launch(p.vids[win], A, y, u0, p.n_units, p.unit_variant, p.tl);
     }
   }
 }
@@ -364,7 +496,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     spmv_prof_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
-  prof_unit<VID>(A, y, st, p, pv, blockIdx.x);
+  prof_unit<VID, false>(A, y, st, p, pv, blockIdx.x);
 }
 
 // All K profiling slices in ONE launch (no forked streams / joins): CTA b runs
@@ -373,43 +505,189 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
 // in its own kernel; its slice is far below one wave, so occupancy does not
 // shape the measured per-unit time, and the score is normalised by the plain
 // kernel's occupancy anyway.
-__global__ void __launch_bounds__(kUnitRows, 1)
+#ifndef DYSEL_PROF_MINB
+#define DYSEL_PROF_MINB 1
+#endif
+template <bool CDP>
+__global__ void __launch_bounds__(kUnitRows, DYSEL_PROF_MINB)
     spmv_prof_all_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p) {
+  // programmatic dependent launch: the claim kernels queued behind this one
+  // may start as soon as every profiling CTA is resident
+  if constexpr (!CDP) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const uint32_t pv = blockIdx.x % p.K, b = blockIdx.x / p.K;
   switch (p.vids[pv]) {
-    case 0: prof_unit<0>(A, y, st, p, pv, b); break;
-    case 1: prof_unit<1>(A, y, st, p, pv, b); break;
-    case 2: prof_unit<2>(A, y, st, p, pv, b); break;
-    case 3: prof_unit<3>(A, y, st, p, pv, b); break;
-    default: prof_unit<4>(A, y, st, p, pv, b); break;
+    case 0: prof_unit<0, CDP>(A, y, st, p, pv, b); break;
+    case 1: prof_unit<1, CDP>(A, y, st, p, pv, b); break;
+    case 2: prof_unit<2, CDP>(A, y, st, p, pv, b); break;
+    case 3: prof_unit<3, CDP>(A, y, st, p, pv, b); break;
+    default: prof_unit<4, CDP>(A, y, st, p, pv, b); break;
   }
 }
 
-// Remainder without a device launch (DYSEL_NO_TAIL, sync): launched by the
-// host right after the profiling kernel on the same stream; every CTA reads
-// the published selection and runs that variant's unit code.
-__global__ void __launch_bounds__(kUnitRows, 4)
-    spmv_remainder_switch_kernel(SpmvDev A, float *__restrict__ y, const SpmvState *st, ProfParams p) {
-  __shared__ int s_vid;
-  if (threadIdx.x == 0) s_vid = p.vids[dysel_ld_acquire_u64(&st->sel) & 0xff];
-  __syncthreads();
-  const uint32_t u = p.p_end + blockIdx.x;
-  switch (s_vid) {
-    case 0: run_unit<0>(A, u, y + (size_t)u * kUnitRows); break;
-    case 1: run_unit<1>(A, u, y + (size_t)u * kUnitRows); break;
-    case 2: run_unit<2>(A, u, y + (size_t)u * kUnitRows); break;
-    case 3: run_unit<3>(A, u, y + (size_t)u * kUnitRows); break;
-    default: run_unit<4>(A, u, y + (size_t)u * kUnitRows); break;
+// Remainder / eager claim kernels (default device path, readings A-27/A-28).
+// The HOST launches, right behind the profiling kernel and chained by
+// programmatic dependent launch, one persistent kernel per pool variant —
+// default first — each the variant's own code at its own occupancy.  Work is
+// claimed per WARP, one 32-row slot (unit u, slot w) per ticket, with no
+// CTA-wide barrier: measured on D4, a CTA-per-unit persistent loop ran CSR-W
+// 1.42 ms vs 0.94 ms for the plain grid (warps idled at the per-unit barrier
+// behind the unit's longest row, while a plain grid's finished warps free
+// their slots for new CTAs).
+//   * Eager (ASYNC, the default's kernel): slot tickets from c1
+//     until the selection is published.  Publishing sets c1's bit 32; the
+//     claim count T_p at that instant, rounded up to a whole unit, is the
+//     switch point S: slots [0, S) belong to the default (a unit is never
+//     split between two variants — JDS slots of a unit permute its rows).
+//   * Remainder: the selected variant's kernel claims slots S + c2.  Every
+//     other kernel exits once it sees the selection (SYNC: everyone waits
+//     for it, and S = 0).
+// Every slot is computed exactly once.  No device-side launch: device-launched
+// grids of the same kernels measured 7% slower on D4 (0.99 vs 0.93 ms), and
+// the round-1 tail launch added ~17 us of launch latency after the selection.
+// lane-0 poll of the published switch word (relaxed: only the word itself is consumed)
+__device__ __forceinline__ uint64_t wait_published(const uint64_t *sw_p) {
+  uint64_t sw = ld_relaxed_u64(sw_p);
+  for (uint32_t ns = 32; sw == ~0ull; ns = ns < 1024 ? 2 * ns : ns) {
+    __nanosleep(ns);
+    sw = ld_relaxed_u64(sw_p);
   }
-  if (p.unit_variant && threadIdx.x == 0) p.unit_variant[u] = (uint8_t)s_vid;
+  return sw;
+}
+
+template <int VID>
+__global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
+    spmv_claim_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const uint32_t FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const uint32_t n_slots = (p.n_units - p.p_end) * kSlots;
+  const uint32_t n_warps = gridDim.x * (kUnitRows / 32);
+  const uint32_t gid = blockIdx.x * (kUnitRows / 32) + (threadIdx.x >> 5);
+  // Claims.  A warp's first slot of a pure run or of the remainder is static
+  // (slot base + warp id: no atomic), later ones come from one global counter
+  // per phase, k slots per atomic: k = min(p.k_claim, remaining / (2 x warps))
+  // >= 1 (p.k_claim ~ 1024 nnz of work per claim: the counter serialises
+  // claims, ~1 per ns, which capped 1-nnz rows).  Claims are made on demand:
+  // issuing the next claim before running the current slots (to hide its
+  // latency) measured 7% slower on D4 (a warp stuck on a long slot holds its
+  // prefetched one back), and 40% slower on CSR-S.
+  auto batch = [&](uint32_t rest) -> uint32_t {
+    const uint32_t k = rest / (2u * n_warps);
+    return k < 1u ? 1u : (k > p.k_claim ? p.k_claim : k);
+  };
+  // phase 0: pure run; 1: eager (default, ASYNC) from c1; 2: after the selection
+  int phase = p.pure ? 0 : ((pv == p.def && p.async) ? 1 : 2);
+  uint32_t S = 0, eager = 0, done = 0;
+  uint32_t t = 0, e = 0;               // current claim [t, e)
+  bool dyn = false;                    // dynamic claims in this phase
+  auto claim = [&](uint32_t k) -> uint64_t {   // lane 0 claims k slots of this phase's counter
+    uint64_t raw = 0;
+    if (lane == 0)
+      raw = phase == 0 ? atomicAdd((unsigned long long *)&st->pure_ctr, (unsigned long long)k)
+          : phase == 1 ? atomicAdd((unsigned long long *)&st->c1, (unsigned long long)k)
+                       : (uint64_t)atomicAdd(&st->c2, k);
+    return __shfl_sync(FULL, raw, 0);
+  };
+  // a warp's first slot of a pure run / of the remainder is static: measured
+  // on D3, claiming it instead cost 30-45% (ELL 15.9 vs 11.0 us)
+  const bool stat = true;
+  // entering the remainder: false if another variant won
+  auto enter_remainder = [&]() -> bool {
+    uint64_t sw = 0;
+    if (lane == 0) sw = wait_published(&st->sw);
+    sw = __shfl_sync(FULL, sw, 0);
+    if ((sw & 0xff) != pv) return false;
+    phase = 2;
+    S = min((uint32_t)(sw >> 8), n_slots);
+    dyn = n_slots - S > n_warps;
+    t = S + gid;
+    e = t < n_slots ? t + 1 : t;
+    if (!stat) { dyn = true; t = e = 0; }
+    return true;
+  };
+  if (phase == 0) {
+    dyn = n_slots > n_warps;
+    t = gid;
+    e = gid < n_slots ? gid + 1 : gid;
+    if (!stat) { dyn = true; t = e = 0; }
+  } else if (phase == 2) {
+    if (!enter_remainder()) return;
+  } else {
+    dyn = true;
+  }
+  for (;;) {
+    if (t >= e) {   // need a claim
+      if (!dyn) break;
+      const uint32_t k = batch(n_slots - min(e, n_slots));
+      const uint64_t r = claim(k);
+      if (phase == 0) {
+        const uint64_t c = (stat ? n_warps : 0u) + r;
+        if (c >= n_slots) {   // each warp ends on one failed claim; the last one resets the counters
+          if (lane == 0 && atomicAdd(&st->pure_done, 1u) == n_warps - 1) {
+            st->pure_ctr = 0;
+            st->pure_done = 0;
+          }
+          break;
+        }
+        t = (uint32_t)c;
+        e = min(t + k, n_slots);
+      } else if (phase == 1) {
+        t = (uint32_t)r;
+        uint32_t lim = n_slots;
+        if (r >> 32) {   // claimed after the selection was published: only below the switch point
+          uint64_t sw = 0;
+          if (lane == 0) sw = wait_published(&st->sw);
+          lim = (uint32_t)(__shfl_sync(FULL, sw, 0) >> 8);
+        }
+        if (t >= lim) {   // eager range closed: hand over to the selection
+          if (!enter_remainder()) break;
+          continue;
+        }
+        e = min(t + k, lim);
+        if (p.tl && lane == 0 && eager == 0)
+          atomicMin((unsigned long long *)&p.tl[3], (unsigned long long)dysel_globaltimer());
+        eager += e - t;
+      } else {
+        t = S + (stat ? n_warps : 0u) + (uint32_t)r;
+        if (t >= n_slots) break;
+        e = min(t + k, n_slots);
+      }
+    }
+    if (phase == 2) {
+      if (p.tl && lane == 0 && done == 0)
+        atomicMin((unsigned long long *)&p.tl[5], (unsigned long long)dysel_globaltimer());
+      done += e - t;
+    }
+    for (uint32_t q = t; q < e; ++q) {
+      const uint32_t u = p.p_end + q / kSlots;
+      run_slot<VID>(A, u, (int)(q % kSlots), y + (size_t)u * kUnitRows);
+      if (lane == 0 && p.unit_variant && q % kSlots == 0) p.unit_variant[u] = (uint8_t)VID;
+    }
+    t = e;
+  }
+  if (p.tl && lane == 0) {
+    if (eager) atomicMax((unsigned long long *)&p.tl[4], (unsigned long long)dysel_globaltimer());
+    if (done) atomicMax((unsigned long long *)&p.tl[6], (unsigned long long)dysel_globaltimer());
+  }
+}
+
+// debug: selection preset to pool index pv with no eager range (claim kernel alone)
+// eager_all: the eager range stays open (c1 unpublished) and S = n_slots, so
+// the default's eager phase runs the whole grid
+__global__ void spmv_state_preset_kernel(SpmvState *s, uint32_t pv, int eager_all, uint64_t n_slots) {
+  s->sel = pv;
+  s->c1 = eager_all ? 0ull : 1ull << 32;
+  s->sw = ((eager_all ? n_slots : 0ull) << 8) | pv;
 }
 
 // Eager copy of the default variant (ASYNC): persistent CTAs claim remainder
 // units by ticket until the selection grabs the rest.
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
-    spmv_eager_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, uint32_t p_end, uint32_t n_units, uint8_t *uv) {
+    spmv_eager_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, uint32_t p_end, uint32_t n_units, uint8_t *uv,
+                      uint64_t *tl) {
   __shared__ uint32_t s_t;
+  if (tl && threadIdx.x == 0) atomicMin((unsigned long long *)&tl[3], (unsigned long long)dysel_globaltimer());
   if (threadIdx.x == 0) s_t = atomicAdd(&st->ticket, 1u);
   __syncthreads();
   uint32_t t = s_t, mine = 0;
@@ -426,6 +704,7 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     t = s_t;
   }
   if (threadIdx.x == 0 && mine) atomicAdd((unsigned long long *)&st->eager_units, (unsigned long long)mine);
+  if (tl && threadIdx.x == 0) atomicMax((unsigned long long *)&tl[4], (unsigned long long)dysel_globaltimer());
 }
 
 // ----------------------------------------------------------------- host side
@@ -435,8 +714,12 @@ static dysel_status spmv_variant_fn(const dysel_slice *s, void *const *args, voi
   if (s->granule_count == 0) return DYSEL_OK;
   SpmvDev A = pl->dev;
   A.x = (const float *)args[1];
-  spmv_slice_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(A, (float *)args[0], *s,
-                                                                                            nullptr);
+  if (s->timer)
+    spmv_slice_timed_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(
+        A, (float *)args[0], *s);
+  else
+    spmv_slice_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(A, (float *)args[0], *s,
+                                                                                              nullptr, nullptr);
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
 
@@ -449,21 +732,33 @@ struct SpmvCtxState {
   SpmvState *h_state = nullptr;   // pinned
   int occ_slice[DYSEL_SPMV_NVARIANTS] = {};
   int occ_eager[DYSEL_SPMV_NVARIANTS] = {};
+  int occ_claim[DYSEL_SPMV_NVARIANTS] = {};
 };
 
 dysel_status spmv_ctx_init(dysel_ctx *ctx) {
   SpmvCtxState *s = new SpmvCtxState();
   ctx->d_spmv_state = s;
   if (cudaMalloc(&s->d_state, sizeof(SpmvState)) != cudaSuccess) return DYSEL_ERR_NOMEM;
+  if (cudaMemset(s->d_state, 0, sizeof(SpmvState)) != cudaSuccess) return DYSEL_ERR_CUDA;
   if (cudaMallocHost(&s->h_state, sizeof(SpmvState)) != cudaSuccess) return DYSEL_ERR_NOMEM;
   const void *slice[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_slice_kernel<0>, (const void *)spmv_slice_kernel<1>,
                                             (const void *)spmv_slice_kernel<2>, (const void *)spmv_slice_kernel<3>,
                                             (const void *)spmv_slice_kernel<4>};
+  const void *claim[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_claim_kernel<0>, (const void *)spmv_claim_kernel<1>,
+                                            (const void *)spmv_claim_kernel<2>, (const void *)spmv_claim_kernel<3>,
+                                            (const void *)spmv_claim_kernel<4>};
   const void *eager[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_eager_kernel<0>, (const void *)spmv_eager_kernel<1>,
                                             (const void *)spmv_eager_kernel<2>, (const void *)spmv_eager_kernel<3>,
                                             (const void *)spmv_eager_kernel<4>};
   for (int v = 0; v < DYSEL_SPMV_NVARIANTS; ++v) {
+    // largest L1 for host launches (tuning knob DYSEL_SPMV_CARVEOUT = percent)
+    const char *cv = getenv("DYSEL_SPMV_CARVEOUT");
+    const int carve = cv ? atoi(cv) : (int)cudaSharedmemCarveoutMaxL1;
+    cudaFuncSetAttribute(slice[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+    cudaFuncSetAttribute(eager[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_slice[v], slice[v], kUnitRows, 0);
+    cudaFuncSetAttribute(claim[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_claim[v], claim[v], kUnitRows, 0);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_eager[v], eager[v], kUnitRows, 0);
   }
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
@@ -504,13 +799,51 @@ static dysel_slice unit_slice(uint64_t u0, uint64_t count, uint64_t n_units, int
   return s;
 }
 
+template <int VID>
+static dysel_status launch_claim(const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p, uint32_t pv,
+                                 unsigned grid, cudaStream_t s, bool pdl) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kUnitRows);
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, spmv_claim_kernel<VID>, A, y, st, p, pv) == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
+}
+typedef dysel_status (*ClaimLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, uint32_t, unsigned,
+                                      cudaStream_t, bool);
+static const ClaimLauncher kClaim[DYSEL_SPMV_NVARIANTS] = {launch_claim<0>, launch_claim<1>, launch_claim<2>,
+                                                           launch_claim<3>, launch_claim<4>};
+
+// Slots per claim: about kClaimNnz nonzeros of work (at least 1, at most a unit).
+constexpr int64_t kClaimNnz = 1024;
+static uint32_t claim_batch(const dysel_spmv_plan *pl) {
+  const int64_t slots = (int64_t)pl->n_units * kSlots;
+  const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
+  return (uint32_t)std::min<int64_t>(kSlots, std::max<int64_t>(1, kClaimNnz / per_slot));
+}
+
+// Pure version of one variant over the whole grid: the variant's claim kernel
+// with every slot its own (the same code and occupancy that runs the DySel
+// remainder, so T* and the remainder are measured on the same kernel).
 static dysel_status launch_variant_full(dysel_ctx *ctx, dysel_spmv_plan *pl, int vid, const float *x, float *y,
                                         cudaStream_t st) {
   if (pl->n_units == 0) return DYSEL_OK;
-  dysel_slice s = unit_slice(0, pl->n_units, pl->n_units, vid);
-  void *args[2] = {y, (void *)x};
-  DYSEL_TRY(kVariantFns[vid](&s, args, st, pl));
-  return check_launch(ctx, "spmv full-grid variant");
+  SpmvCtxState *cs = (SpmvCtxState *)ctx->d_spmv_state;
+  ProfParams p;
+  memset(&p, 0, sizeof(p));
+  p.K = (uint32_t)pl->K;
+  p.n_units = pl->n_units;
+  p.pure = 1;
+  p.k_claim = claim_batch(pl);
+  const uint64_t grid = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[vid]) * ctx->n_sm, pl->n_units);
+  SpmvDev A = pl->dev;
+  A.x = x;
+  DYSEL_TRY(kClaim[vid](A, y, cs->d_state, p, 0, (unsigned)grid, st, false));
+  return check_launch(ctx, "spmv pure claim kernel");
 }
 
 template <int VID>
@@ -537,6 +870,61 @@ dysel_status dysel_spmv_variant(dysel_ctx *ctx, dysel_spmv_plan *pl, int variant
   return launch_variant_full(ctx, pl, variant_id, d_x, d_y, (cudaStream_t)stream);
 }
 
+dysel_status dysel_debug_spmv_device_launch(dysel_ctx *ctx, dysel_spmv_plan *pl, int variant_id, const float *d_x,
+                                            float *d_y, int how, void *stream, uint32_t *h_resident_max, int n_sm) {
+  if (!ctx || !pl || spmv_pool_index(pl, variant_id) < 0 || how < 0 || how > 4 || n_sm > 1024)
+    return DYSEL_ERR_INVALID;
+  cudaStream_t st = (cudaStream_t)stream;
+  SpmvDev A = pl->dev;
+  A.x = d_x;
+  uint64_t *tl = nullptr;
+  if (h_resident_max) {
+    void *g = nullptr;
+    DYSEL_CUDA_TRY(ctx, cudaGetSymbolAddress(&g, g_resident));
+    DYSEL_CUDA_TRY(ctx, cudaMemsetAsync(g, 0, sizeof(g_resident), st));
+    tl = ((SpmvCtxState *)ctx->d_spmv_state)->d_state->tl;
+  }
+  if (how == 3 || how == 4) {   // the claim kernel alone, selection preset (4: all eager)
+    SpmvCtxState *cs = (SpmvCtxState *)ctx->d_spmv_state;
+    const int pv = spmv_pool_index(pl, variant_id);
+    spmv_state_init_kernel<<<1, 32, 0, st>>>(cs->d_state, pl->K, pv);
+    spmv_state_preset_kernel<<<1, 1, 0, st>>>(cs->d_state, (uint32_t)pv, how == 4, (uint64_t)pl->n_units * kSlots);
+    ProfParams p;
+    memset(&p, 0, sizeof(p));
+    p.K = pl->K;
+    p.n_units = pl->n_units;
+    p.def = pv;
+    p.async = how == 4;
+    p.k_claim = claim_batch(pl);
+    for (int i = 0; i < pl->K; ++i) p.vids[i] = pl->vids[i];
+    const uint64_t g = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[variant_id]) * ctx->n_sm, pl->n_units);
+    DYSEL_TRY(kClaim[variant_id](A, d_y, cs->d_state, p, pv, (unsigned)g, st, false));
+    DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+    return check_launch(ctx, "claim");
+  }
+  if (how == 0) {
+    dysel_slice s = unit_slice(0, pl->n_units, pl->n_units, variant_id);
+    switch (variant_id) {
+      case 0: spmv_slice_kernel<0><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
+      case 1: spmv_slice_kernel<1><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
+      case 2: spmv_slice_kernel<2><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
+      case 3: spmv_slice_kernel<3><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
+      default: spmv_slice_kernel<4><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
+    }
+  } else {
+    spmv_device_launch_kernel<<<1, 1, 0, st>>>(A, d_y, variant_id, pl->n_units, how, tl);
+  }
+  DYSEL_TRY(check_launch(ctx, "spmv_device_launch_kernel"));
+  if (h_resident_max) {
+    void *g = nullptr;
+    DYSEL_CUDA_TRY(ctx, cudaGetSymbolAddress(&g, g_resident));
+    DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(h_resident_max, (uint32_t *)g + 1024, n_sm * sizeof(uint32_t),
+                                        cudaMemcpyDeviceToHost, st));
+    DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+  }
+  return DYSEL_OK;
+}
+
 dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, float *d_y, float f, uint32_t mode,
                         void *stream, dysel_report *rep) {
   const uint64_t t_host0 = now_ns();
@@ -549,6 +937,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   if (rep) {
     rep->n_slices = 0;
     rep->eager_units = rep->tail_units = 0;
+    for (int i = 0; i < 8; ++i) rep->timeline_ns[i] = ~0ull;
     for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v)
       rep->score[v] = rep->makespan_ns[v] = rep->units[v] = rep->cycles[v] = rep->busy_ns[v] = rep->aborted[v] = 0;
   }
@@ -643,21 +1032,25 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.score_mode = (mode & DYSEL_SCORE_CYCLES) ? 1u : ((mode & DYSEL_SCORE_MAKESPAN) || sequential ? 2u : 0u);
   if (sequential) p.async = 0;   // a variant profiled alone: no eager work beside it
   p.def = (uint32_t)pl->def;
-  p.tail = (mode & DYSEL_NO_TAIL) ? 0u : 1u;
+  p.k_claim = claim_batch(pl);
+  const bool cdp = (mode & DYSEL_DEVICE_LAUNCH) != 0;   // round-1 scheme: eager + remainder launched on the device
+  p.tail = (cdp && !(mode & DYSEL_NO_TAIL)) ? 1u : 0u;
   p.abort = ((mode & DYSEL_NO_ABORT) || p.score_mode == 1) ? 0u : 1u;   // dominance needs busy or makespan
   for (int i = 0; i < pl->K; ++i) {
     p.vids[i] = pl->vids[i];
-    p.occ[i] = (uint32_t)std::max(1, cs->occ_slice[pl->vids[i]]);
+    // occupancy of the kernel that will run the remainder with this variant
+    p.occ[i] = (uint32_t)std::max(1, cdp ? cs->occ_slice[pl->vids[i]] : cs->occ_claim[pl->vids[i]]);
   }
   if (p.hybrid) {
-    DYSEL_TRY(scratch(ctx, ctx->sandbox[0], (size_t)(pl->K - 1) * P.c * kUnitRows * sizeof(float)));
+    DYSEL_TRY(scratch(ctx, ctx->sandbox[0], (size_t)pl->K * P.c * kUnitRows * sizeof(float)));
     p.sandbox = (float *)ctx->sandbox[0].ptr;
   }
   p.unit_variant = d_uv;
+  if (rep) p.tl = cs->d_state->tl;
   SpmvDev A = pl->dev;
   A.x = d_x;
   SpmvState *dst = cs->d_state;
-  if (p.async && p.p_end < p.n_units) {
+  if (cdp && p.async && p.p_end < p.n_units) {
     const int dv = pl->vids[pl->def];
     p.eager_grid =
         (uint32_t)std::min<uint64_t>((uint64_t)std::max(1, cs->occ_eager[dv]) * ctx->n_sm, p.n_units - p.p_end);
@@ -673,12 +1066,37 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       DYSEL_TRY(check_launch(ctx, "spmv_prof_kernel"));
     }
   } else {   // all K profiling slices in one launch on the stream
-    spmv_prof_all_kernel<<<p.K * p.c, kUnitRows, 0, st>>>(A, d_y, dst, p);
+    if (cdp)
+      spmv_prof_all_kernel<true><<<p.K * p.c, kUnitRows, 0, st>>>(A, d_y, dst, p);
+    else
+      spmv_prof_all_kernel<false><<<p.K * p.c, kUnitRows, 0, st>>>(A, d_y, dst, p);
     DYSEL_TRY(check_launch(ctx, "spmv_prof_all_kernel"));
   }
-  if (!p.tail && !p.async && p.p_end < p.n_units) {   // NO_TAIL: host-launched switch remainder
-    spmv_remainder_switch_kernel<<<p.n_units - p.p_end, kUnitRows, 0, st>>>(A, d_y, dst, p);
-    DYSEL_TRY(check_launch(ctx, "spmv_remainder_switch_kernel"));
+  if (!cdp && p.p_end < p.n_units) {
+    // host-launched claim kernels, default first; programmatic dependent
+    // launch lets them start while profiling runs (not after NO_TAIL or a
+    // sequential profile: then they follow in stream order)
+    const bool pdl = !(mode & DYSEL_NO_TAIL) && !sequential;
+#ifdef DYSEL_EXP_DEF_ONLY
+    for (int k = 0; k < 1; ++k) {
+#else
+    for (int k = 0; k < pl->K; ++k) {
+#endif
+      const uint32_t i = (uint32_t)(k == 0 ? pl->def : (k <= pl->def ? k - 1 : k));
+      const int v = pl->vids[i];
+      const uint64_t g = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[v]) * ctx->n_sm,
+                                            p.n_units - p.p_end);
+      DYSEL_TRY(kClaim[v](A, d_y, dst, p, i, (unsigned)g, st, pdl));
+      DYSEL_TRY(check_launch(ctx, "spmv_claim_kernel"));
+    }
+  } else if (cdp && !p.tail && !p.async && p.p_end < p.n_units) {   // CDP scheme, NO_TAIL: winner via claim kernels
+    for (int i = 0; i < pl->K; ++i) {
+      const int v = pl->vids[i];
+      const uint64_t g = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[v]) * ctx->n_sm,
+                                            p.n_units - p.p_end);
+      DYSEL_TRY(kClaim[v](A, d_y, dst, p, (uint32_t)i, (unsigned)g, st, false));
+      DYSEL_TRY(check_launch(ctx, "spmv_claim_kernel"));
+    }
   }
   DYSEL_TRY(commit_pending_sel(ctx, pend, pl->sig, st));
   if (rep) {
@@ -691,7 +1109,10 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
     const int sel_pool = (int)(h->sel & 0xff);
     rep->selected = sel_pool < pl->K ? pl->vids[sel_pool] : -1;
     rep->eager_units = h->eager_units;
-    rep->tail_units = h->tail_begin != ~0ull ? pl->n_units - h->tail_begin : 0;
+    const bool claimed = !cdp || !p.tail;   // remainder run by the claim kernels
+    if (claimed) rep->eager_units = h->sw != ~0ull ? (h->sw >> 8) / kSlots : 0;
+    rep->tail_units = !claimed ? (h->tail_begin != ~0ull ? pl->n_units - h->tail_begin : 0)
+                          : (p.n_units - p.p_end - std::min<uint64_t>(rep->eager_units, p.n_units - p.p_end));
     const uint64_t cap = (1ull << 56) - 1;
     for (int v = 0; v < pl->K; ++v) {
       const int id = pl->vids[v];
@@ -709,6 +1130,9 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
                                                                 h->max_busy[v]);
     }
     if (sel_pool < pl->K) ctx->sel_cache[pl->sig] = sel_pool;
+    for (int i = 0; i < 7; ++i)
+      rep->timeline_ns[i] = (h->tl[i] == ~0ull || h->tl[i] == 0 || h->tl[0] == ~0ull) ? ~0ull : h->tl[i] - h->tl[0];
+    rep->timeline_ns[7] = h->tl[7];
     rep->host_ns = now_ns() - t_host0;
   }
   return DYSEL_OK;

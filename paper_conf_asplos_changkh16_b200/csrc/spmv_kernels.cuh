@@ -33,6 +33,7 @@ namespace dysel {
 constexpr int kUnitRows = 256;
 constexpr int kVecMin = 128;   // CSR-V: rows at least this long use 128-bit loads
 constexpr int kRowBatch = 4;   // CSR-V: rows in flight per warp
+constexpr int kChunk = 8;      // CSR-S / ELL / JDS: entries per thread in flight
 constexpr int kStreamUnroll = 4;   // CSR-W: 32-entry chunks in flight per warp
 constexpr int kStreamLong = 512;   // CSR-W: open-row stretch that switches to 128-bit loads
 
@@ -110,19 +111,34 @@ __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
 }
 
 // ------------------------------------------------------------------ CSR-S
+// The row is walked in chunks of kChunk entries: the chunk's col/val loads,
+// then its x gathers, are all issued before the first fma, so a thread has
+// kChunk independent loads in flight instead of one dependent chain per entry.
+// The fmas still run one by one in CSR order (same bits as the plain loop).
 template <class Poll>
-__device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, float *__restrict__ out,
+__device__ __forceinline__ void unit_csr_scalar(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
                                                 const Poll &poll) {
-  const int i = threadIdx.x;
+  const int i = w * 32 + (threadIdx.x & 31);
   const int64_t r = (int64_t)j * kUnitRows + i;
   if (r >= A.n_rows) return;
   const uint64_t px = policy_evict_last();
   const int b = __ldg(A.row_ptr + r), e = __ldg(A.row_ptr + r + 1);
   float s = 0.0f;
-#pragma unroll 4
-  for (int k = b; k < e; ++k) {
-    s = __fmaf_rn(__ldg(A.val + k), ld_x(A.x + __ldg(A.col + k), px), s);
-    if (Poll::active && ((k - b) & 63) == 63 && poll()) break;
+  for (int k = b; k < e; k += kChunk) {
+    int c[kChunk];
+    float v[kChunk], xv[kChunk];
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) {
+      const bool ok = k + u < e;
+      c[u] = ok ? __ldg(A.col + k + u) : 0;
+      v[u] = ok ? __ldg(A.val + k + u) : 0.0f;
+    }
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) xv[u] = k + u < e ? ld_x(A.x + c[u], px) : 0.0f;
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u)
+      if (k + u < e) s = __fmaf_rn(v[u], xv[u], s);
+    if (Poll::active && ((k - b) & 63) >= 64 - kChunk && poll()) break;
   }
   out[i] = s;
 }
@@ -178,9 +194,9 @@ __device__ __forceinline__ float csrv_long_row(const SpmvDev &A, int b, int e, i
 }
 
 template <class Poll>
-__device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, float *__restrict__ out,
+__device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
                                                 const Poll &poll) {
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
   const int64_t base = (int64_t)j * kUnitRows + w * 32;
   const int nr = (int)min((int64_t)32, (int64_t)A.n_rows - base);
   if (nr <= 0) return;
@@ -232,48 +248,46 @@ __device__ __forceinline__ void unit_csr_vector(const SpmvDev &A, uint32_t j, fl
 }
 
 // -------------------------------------------------------------------- ELL
+// Chunks of kChunk slots: loads first, then the gathers of the live slots,
+// then the fmas in slot order.  Pads only follow a row's entries, so a chunk
+// ending in a pad ends the row.
 template <class Poll>
-__device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, float *__restrict__ out, const Poll &poll) {
-  const int i = threadIdx.x;
+__device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out, const Poll &poll) {
+  const int i = w * 32 + (threadIdx.x & 31);
   const int64_t r = (int64_t)j * kUnitRows + i;
   if (r >= A.n_rows) return;
   const uint64_t ps = policy_evict_first(), px = policy_evict_last();
   const int32_t *cp = A.ell_col + r;
   const float *vp = A.ell_val + r;
+  const int W = A.ell_W;
   float s = 0.0f;
-  int k = 0;
-  bool live = true;   // pads (col = -1) only follow a row's entries
-  for (; k + 2 <= A.ell_W; k += 2) {
-    const int c0 = ld_stream(cp + (int64_t)k * A.n_pad, ps);
-    const int c1 = ld_stream(cp + (int64_t)(k + 1) * A.n_pad, ps);
-    const float v0 = ld_stream(vp + (int64_t)k * A.n_pad, ps);
-    const float v1 = ld_stream(vp + (int64_t)(k + 1) * A.n_pad, ps);
-    if (c0 < 0) {
-      live = false;
-      break;
+  for (int k = 0; k < W; k += kChunk) {
+    int c[kChunk];
+    float v[kChunk], xv[kChunk];
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) {
+      const bool ok = k + u < W;
+      c[u] = ok ? ld_stream(cp + (int64_t)(k + u) * A.n_pad, ps) : -1;
+      v[u] = ok ? ld_stream(vp + (int64_t)(k + u) * A.n_pad, ps) : 0.0f;
     }
-    s = __fmaf_rn(v0, ld_x(A.x + c0, px), s);
-    if (c1 < 0) {
-      live = false;
-      break;
-    }
-    s = __fmaf_rn(v1, ld_x(A.x + c1, px), s);
-    if (Poll::active && (k & 63) == 62 && poll()) {
-      live = false;
-      break;
-    }
-  }
-  if (live && k < A.ell_W) {
-    const int c0 = ld_stream(cp + (int64_t)k * A.n_pad, ps);
-    if (c0 >= 0) s = __fmaf_rn(ld_stream(vp + (int64_t)k * A.n_pad, ps), ld_x(A.x + c0, px), s);
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) xv[u] = c[u] >= 0 ? ld_x(A.x + c[u], px) : 0.0f;
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u)
+      if (c[u] >= 0) s = __fmaf_rn(v[u], xv[u], s);
+    if (c[kChunk - 1] < 0) break;
+    if (Poll::active && (k & 63) >= 64 - kChunk && poll()) break;
   }
   out[i] = s;
 }
 
 // -------------------------------------------------------------------- JDS
+// Chunks of kChunk diagonals; the jd_ptr offsets of the next chunk (the same
+// for every thread of the block: broadcast loads) are fetched while the
+// current chunk's col/val loads and gathers are in flight.
 template <class Poll>
-__device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, float *__restrict__ out, const Poll &poll) {
-  const int p = threadIdx.x;
+__device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out, const Poll &poll) {
+  const int p = w * 32 + (threadIdx.x & 31);
   const int64_t q = (int64_t)j * kUnitRows + p;
   if (q >= A.n_rows) return;
   const uint64_t ps = policy_evict_first(), px = policy_evict_last();
@@ -281,11 +295,26 @@ __device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, float *__
   const int32_t *jp = A.jd_ptr + __ldg(A.jd_off + j);
   const int64_t base = __ldg(A.blk_off + j) + p;
   float s = 0.0f;
-#pragma unroll 4
-  for (int k = 0; k < len; ++k) {
-    const int64_t idx = base + __ldg(jp + k);
-    s = __fmaf_rn(ld_stream(A.jds_val + idx, ps), ld_x(A.x + ld_stream(A.jds_col + idx, ps), px), s);
-    if (Poll::active && (k & 63) == 63 && poll()) break;
+  int off[kChunk];
+#pragma unroll
+  for (int u = 0; u < kChunk; ++u) off[u] = u < len ? __ldg(jp + u) : 0;
+  for (int k = 0; k < len; k += kChunk) {
+    int c[kChunk];
+    float v[kChunk], xv[kChunk];
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) {
+      const bool ok = k + u < len;
+      c[u] = ok ? ld_stream(A.jds_col + base + off[u], ps) : 0;
+      v[u] = ok ? ld_stream(A.jds_val + base + off[u], ps) : 0.0f;
+    }
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) off[u] = k + kChunk + u < len ? __ldg(jp + k + kChunk + u) : 0;
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u) xv[u] = k + u < len ? ld_x(A.x + c[u], px) : 0.0f;
+#pragma unroll
+    for (int u = 0; u < kChunk; ++u)
+      if (k + u < len) s = __fmaf_rn(v[u], xv[u], s);
+    if (Poll::active && (k & 63) >= 64 - kChunk && poll()) break;
   }
   out[__ldg(A.perm + q) - (int64_t)j * kUnitRows] = s;
 }
@@ -300,10 +329,10 @@ __device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, float *__
 // takes the scan value at the last lane of its segment.  The per-row order
 // depends only on the row's offset inside its group: deterministic (c-6).
 template <class Poll>
-__device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, float *__restrict__ out,
+__device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
                                                 const Poll &poll) {
   const uint32_t FULL = 0xffffffffu;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
   const int64_t base = (int64_t)j * kUnitRows + w * 32;
   const int nr = (int)min((int64_t)32, (int64_t)A.n_rows - base);
   if (nr <= 0) return;
@@ -407,23 +436,34 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, fl
   if (lane < nr) out[w * 32 + lane] = acc;
 }
 
+// One 32-row warp slot w (0..7) of unit j: rows 256 j + 32 w + lane (JDS:
+// permuted positions 32 w + lane of block j, whose rows lie anywhere in the
+// unit).  The 8 slots of a unit, run by the same variant in any order and by
+// any warps, compute the whole unit; the per-row arithmetic does not depend on
+// which warp runs it.
+template <int VID, class Poll = NoPoll>
+__device__ __forceinline__ void run_slot(const SpmvDev &A, uint32_t j, int w, float *out, const Poll &poll = Poll()) {
+  if constexpr (VID == 0) unit_csr_scalar(A, j, w, out, poll);
+  else if constexpr (VID == 1) unit_csr_vector(A, j, w, out, poll);
+  else if constexpr (VID == 2) unit_ell(A, j, w, out, poll);
+  else if constexpr (VID == 3) unit_jds(A, j, w, out, poll);
+  else unit_csr_stream(A, j, w, out, poll);
+}
+
+// Whole unit by a 256-thread CTA: warp w runs slot w.
 template <int VID, class Poll = NoPoll>
 __device__ __forceinline__ void run_unit(const SpmvDev &A, uint32_t j, float *out, const Poll &poll = Poll()) {
-  if constexpr (VID == 0) unit_csr_scalar(A, j, out, poll);
-  else if constexpr (VID == 1) unit_csr_vector(A, j, out, poll);
-  else if constexpr (VID == 2) unit_ell(A, j, out, poll);
-  else if constexpr (VID == 3) unit_jds(A, j, out, poll);
-  else unit_csr_stream(A, j, out, poll);
+  run_slot<VID, Poll>(A, j, (int)(threadIdx.x >> 5), out, poll);
 }
 
 template <class Poll>
 __device__ __forceinline__ void run_unit_dyn(int vid, const SpmvDev &A, uint32_t j, float *out, const Poll &poll) {
   switch (vid) {
-    case 0: unit_csr_scalar(A, j, out, poll); break;
-    case 1: unit_csr_vector(A, j, out, poll); break;
-    case 2: unit_ell(A, j, out, poll); break;
-    case 3: unit_jds(A, j, out, poll); break;
-    default: unit_csr_stream(A, j, out, poll); break;
+    case 0: run_unit<0>(A, j, out, poll); break;
+    case 1: run_unit<1>(A, j, out, poll); break;
+    case 2: run_unit<2>(A, j, out, poll); break;
+    case 3: run_unit<3>(A, j, out, poll); break;
+    default: run_unit<4>(A, j, out, poll); break;
   }
 }
 

@@ -124,7 +124,7 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
                                 void *stream, dysel_spmv_plan **out) {
   if (!ctx || !out || n_rows < 0 || n_cols < 0 || nnz < 0 || nnz >= (1ll << 31) || n_rows >= (1ll << 31) ||
       n_cols >= (1ll << 31) || (n_rows > 0 && !d_row_ptr) || (nnz > 0 && (!d_col || !d_val)) ||
-      default_variant < 0 || default_variant >= DYSEL_SPMV_NVARIANTS) {
+      default_variant < DYSEL_SPMV_DEFAULT_AUTO || default_variant >= DYSEL_SPMV_NVARIANTS) {
     set_error(ctx, "dysel_spmv_prepare: invalid arguments");
     return DYSEL_ERR_INVALID;
   }
@@ -231,6 +231,12 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
   }
   if (formats_mask & DYSEL_FMT_STREAM) pl->vids[pl->K++] = DYSEL_SPMV_CSR_STREAM;
   if (cudaStreamSynchronize(st) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (default_variant == DYSEL_SPMV_DEFAULT_AUTO) {   // reading A-30: initial version from row statistics
+    if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
+    else if (spmv_pool_index(pl, DYSEL_SPMV_CSR_STREAM) >= 0) default_variant = DYSEL_SPMV_CSR_STREAM;
+    else default_variant = DYSEL_SPMV_CSR_VECTOR;
+  }
+  I.default_variant = default_variant;
   pl->def = spmv_pool_index(pl, default_variant);
   if (pl->def < 0) {
     set_error(ctx, "dysel_spmv_prepare: default variant not in the pool (ELL inapplicable? A-15)");

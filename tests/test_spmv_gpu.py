@@ -119,7 +119,8 @@ def test_identity_and_diagonal_exact(ctx):
 
 
 MODES = ["fully_sync", "fully_async", "hybrid_sync", "hybrid_async", "fully_sync_host", "fully_async_host",
-         "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles"]
+         "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles", "hybrid_async_cdp", "fully_sync_cdp",
+         "hybrid_async_notail", "fully_sync_seq"]
 
 
 def mode_bits(D, m):
@@ -129,6 +130,9 @@ def mode_bits(D, m):
     b |= D.HOST_ORCH if m.endswith("host") else 0
     b |= D.CONTIGUOUS if "contig" in m else 0
     b |= D.SCORE_CYCLES if "cycles" in m else 0
+    b |= D.DEVICE_LAUNCH if "cdp" in m else 0
+    b |= D.NO_TAIL if "notail" in m else 0
+    b |= D.SEQUENTIAL if "seq" in m else 0
     return b
 
 
@@ -166,12 +170,16 @@ def test_dysel_composition(ctx, D, name, m):
         v = uv[u]
         assert v in full, (u, v)
         assert np.array_equal(yy[r0:r1], full[v][r0:r1]), (u, v)
-    # profiling granules carry the ticket's variant, remainder the selection (sync)
+    # profiling granules carry the ticket's variant, remainder the selection (sync).
+    # Device-path hybrid (reading A-4'): the shared profiled units are the
+    # winner's (its sandbox is copied in); the host path keeps the paper's
+    # productive default (A-4).
     pool = plan.variant_ids
     owner = slice_plan.productive_cover(p, pool.index(sel))
+    dev_hybrid = p.mode == slice_plan.HYBRID and not m.endswith("host")
     for j in range(p.Gn):
         if j < len(owner) and (j < p.c * (K if p.mode == slice_plan.FULLY else 1)):
-            assert uv[j] == pool[owner[j]], j
+            assert uv[j] == (sel if dev_hybrid else pool[owner[j]]), j
         elif "async" not in m:
             assert uv[j] == sel, j
     plan.destroy()
@@ -238,23 +246,33 @@ def test_edge_cases(ctx, D):
 
 
 @pytest.mark.parametrize("asy", [False, True])
-def test_tail_launch_hands_off_remainder(ctx, D, asy):
-    """The winner's plain kernel runs the unclaimed remainder (CDP2 tail
-    launch); NO_TAIL keeps it inside the dispatcher.  Same output either way."""
+def test_remainder_hand_off(ctx, D, asy):
+    """The remainder goes to the winner in every launch scheme: host-launched
+    claim kernels started beside profiling (PDL, default), the same after
+    profiling completes (NO_TAIL), and the round-1 device-launched scheme
+    (DEVICE_LAUNCH: CDP2 eager + remainder, with and without NO_TAIL).
+    Sync: every remainder unit is the winner's (eager = 0); async: the
+    eager units are whole units of the default, the rest the winner's."""
     import torch
     A = MATS["powerlaw"]()
     x = uniform_f32(11, A.n_cols)
-    plan = prepared(ctx, A)
-    mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0)
-    y1 = torch.empty(A.n_rows, device="cuda")
-    r1 = ctx.spmv(plan, vec(x), y1, f=0.05, mode=mode, report=True, unit_map=True)
-    if not asy:
-        assert r1["tail_units"] == plan.n_units - len(plan.variant_ids) * r1["c"]
-    assert spmv_err(A, x, y1) <= SPMV_TOL
-    y2 = torch.empty(A.n_rows, device="cuda")
-    r2 = ctx.spmv(plan, vec(x), y2, f=0.05, mode=mode | D.NO_TAIL, report=True)
-    assert r2["tail_units"] == 0
-    assert spmv_err(A, x, y2) <= SPMV_TOL
+    plan = prepared(ctx, A, default=1)
+    K = len(plan.variant_ids)
+    for extra in (0, D.NO_TAIL, D.DEVICE_LAUNCH, D.DEVICE_LAUNCH | D.NO_TAIL):
+        mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0) | extra
+        y = torch.full((A.n_rows,), float("nan"), device="cuda")
+        r = ctx.spmv(plan, vec(x), y, f=0.05, mode=mode, report=True, unit_map=True)
+        assert spmv_err(A, x, y) <= SPMV_TOL, extra
+        rem = plan.n_units - K * r["c"]
+        uv = r["unit_variant"]
+        if not asy:
+            assert r["eager_units"] == 0 and r["tail_units"] == rem, (extra, r)
+            assert all(uv[u] == r["selected"] for u in range(K * r["c"], plan.n_units)), extra
+        elif not (extra & D.DEVICE_LAUNCH):
+            e = r["eager_units"]
+            assert e + r["tail_units"] == rem, (extra, r)
+            assert all(uv[u] == 1 for u in range(K * r["c"], K * r["c"] + e)), extra
+            assert all(uv[u] == r["selected"] for u in range(K * r["c"] + e, plan.n_units)), extra
     plan.destroy()
 
 
@@ -270,7 +288,8 @@ def test_tail_launch_is_stream_ordered(ctx, D):
     ref = torch.empty(A.n_rows, device="cuda")
     ctx.spmv_variant(plan, 1, xd, ref)
     torch.cuda.synchronize()
-    for mode in (D.HYBRID | D.SYNC, D.HYBRID | D.ASYNC, D.FULLY | D.SYNC):
+    for mode in (D.HYBRID | D.SYNC, D.HYBRID | D.ASYNC, D.FULLY | D.SYNC, D.HYBRID | D.ASYNC | D.DEVICE_LAUNCH,
+                 D.FULLY | D.SYNC | D.DEVICE_LAUNCH):
         for _ in range(3):
             y = torch.full((A.n_rows,), float("nan"), device="cuda")
             ctx.spmv(plan, xd, y, f=0.01, mode=mode | D.FORCE_PROFILE)
