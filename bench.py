@@ -153,7 +153,7 @@ METRIC = "DySel SpMV GB/s (power-law 1e7 rows, profiling on every call) + overhe
 def config(A, world):
     return {"workload": "D4 power-law SpMV: 10^7 rows, p(L)~L^-1.761 on [1,16384], uniform cols, fp32 CSR",
             "n_rows": int(A.n_rows), "nnz": int(A.nnz), "parallelism": f"row-shard{world}",
-            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": "AUTO|ASYNC (hybrid), f=0.005",
+            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": "AUTO|ASYNC (hybrid), f=0.002",
             "default_variant": "DYSEL_SPMV_DEFAULT_AUTO (A-30)"}
 
 
@@ -261,7 +261,7 @@ def dysel_arm(args, world, rank, local_rank):
         ablation["sync_overhead_pct"] = round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=D.AUTO), 10, stream)
                                                / T_star - 1) * 100, 2)
         ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10, stream)
-                                                      / T_star - 1) * 100, 2) for ff in (0.001, 0.002, 0.01, 0.02)}
+                                                      / T_star - 1) * 100, 2) for ff in (0.001, 0.005, 0.01, 0.02)}
         for dname, dv in (("csr_vector", D.SPMV_CSR_VECTOR), ("jds", D.SPMV_JDS)):
             pd = ctx.spmv_prepare(rp, col, val, A.n_cols, default=dv)
             td = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode), 10, stream)
@@ -482,7 +482,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="dysel", choices=["dysel", "reference"])
     ap.add_argument("--rows", type=int, default=10_000_000)
-    ap.add_argument("--f", type=float, default=0.005)
+    ap.add_argument("--f", type=float, default=0.002)
     ap.add_argument("--oracle-reps", type=int, default=15)
     ap.add_argument("--amortize", type=int, default=20)
     ap.add_argument("--cpu-reps", type=int, default=5)

@@ -106,7 +106,13 @@ __device__ __forceinline__ float4 ld_stream4(const float *p, uint64_t pol) {
 // kept in L2.
 __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
   float v;
+#if defined(DYSEL_EXP_LDX) && DYSEL_EXP_LDX == 1
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+#elif defined(DYSEL_EXP_LDX) && DYSEL_EXP_LDX == 2
+  asm volatile("ld.global.cg.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+#else
   asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+#endif
   return v;
 }
 
