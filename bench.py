@@ -351,7 +351,7 @@ def secondary_workloads(ctx, D, args, stream):
     A = d3_fem()
     x = torch.from_numpy(uniform_f32(384, A.n_cols)).cuda()
     rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
-    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO)
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ALL)
     y = torch.empty(A.n_rows, device="cuda")
     nb = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -391,7 +391,7 @@ def secondary_workloads(ctx, D, args, stream):
     for name, A6 in (("d6_random_16k_1pct", d6_random()), ("d6_diagonal_2M", d6_diag())):
         x6 = torch.from_numpy(uniform_f32(6, A6.n_cols)).cuda()
         rp6, col6, val6 = (torch.from_numpy(a).cuda() for a in (A6.row_ptr, A6.col, A6.val))
-        plan6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_DEFAULT_AUTO)
+        plan6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ALL)
         y6 = torch.empty(A6.n_rows, device="cuda")
         r6 = {D.SPMV_NAMES[v]: time_b2b(lambda: ctx.spmv_variant(plan6, v, x6, y6), 20, stream)
               for v in plan6.variant_ids}

@@ -256,15 +256,18 @@ dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key); /* NULL key
  * P:L1128-1131).  Unit = 256 consecutive original rows.
  * Built-in variants (ids): 0 CSR-scalar (thread per row), 1 CSR-vector (warp
  * per row), 2 ELL (column-major, padded), 3 block-local JDS (A-14), 4 CSR-W
- * (warp-streaming CSR with a warp-level segmented reduction; B200 addition). */
+ * (warp-streaming CSR with a warp-level segmented reduction; B200 addition),
+ * 5 CSR-T (CSR-S with each warp's nonzeros staged in shared memory by the
+ * bulk-copy / TMA engine; data-placement variant). */
 enum { DYSEL_SPMV_CSR_SCALAR = 0, DYSEL_SPMV_CSR_VECTOR = 1, DYSEL_SPMV_ELL = 2, DYSEL_SPMV_JDS = 3,
-       DYSEL_SPMV_CSR_STREAM = 4, DYSEL_SPMV_NVARIANTS = 5 };
+       DYSEL_SPMV_CSR_STREAM = 4, DYSEL_SPMV_CSR_TMA = 5, DYSEL_SPMV_NVARIANTS = 6 };
 /* default_variant = DYSEL_SPMV_DEFAULT_AUTO: the library picks the initial
  * version from the prepare-time row statistics (reading A-30): uniform rows
  * (A-13) -> ELL when in the pool; otherwise CSR-W when in the pool, else
  * CSR-V.  The choice is visible in dysel_spmv_plan_info.default_variant. */
 #define DYSEL_SPMV_DEFAULT_AUTO (-1)
 #define DYSEL_FMT_STREAM 4u   /* include CSR-W in the pool (reads the CSR arrays directly) */
+#define DYSEL_FMT_TMA 8u      /* include CSR-T in the pool (reads the CSR arrays directly) */
 #define DYSEL_FMT_ELL 1u
 #define DYSEL_FMT_JDS 2u
 

@@ -203,10 +203,17 @@ struct SandboxPoll {
 
 // resident CTAs per SM each plain variant kernel is compiled for (register cap)
 // (CSR-V at 6/SM spills and measured slower on D4: 1.44 vs 1.35 ms)
-constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 5};
+constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 5, 3};
 constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
+// dynamic shared memory of each variant's kernels (CSR-T's staging buffers)
+__host__ __device__ constexpr size_t dyn_smem(int vid) { return vid == DYSEL_SPMV_CSR_TMA ? sizeof(TmaStageBufs) : 0; }
+inline size_t pool_dyn_smem(const ProfParams &p) {
+  size_t b = 0;
+  for (uint32_t i = 0; i < p.K; ++i) b = std::max(b, dyn_smem(p.vids[i]));
+  return b;
+}
 // claim kernels: CTAs per SM (CSR-S / ELL at 8 spilled ~200 B in the claim loop)
-constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {6, 4, 6, 6, 5};
+constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {6, 4, 6, 6, 5, 3};
 
 // Plain kernel of one variant over a slice: the exhaustive oracle's pure
 // version, the activation-flag-off path, the tail-launched remainder, the
@@ -231,6 +238,7 @@ __device__ __forceinline__ uint32_t smid() {
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     spmv_slice_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s, uint8_t *uv, uint64_t *tl) {
+  if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
   if (!dysel_gate_open(s)) return;
   if (tl && threadIdx.x == 0) {
     atomicMin((unsigned long long *)&tl[5], (unsigned long long)dysel_globaltimer());
@@ -253,6 +261,7 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     spmv_slice_timed_kernel(SpmvDev A, float *__restrict__ y, dysel_slice s) {
+  if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
   __shared__ dysel_prof_smem psm;
   if (!dysel_gate_open(s)) return;
   dysel_prof_begin(s, psm);
@@ -283,11 +292,12 @@ __device__ void tail_launch(int vid, const SpmvDev &A, float *y, uint64_t u0, ui
   // kept: a grid completes only with all its device-launched children.
   const cudaStream_t ff = cudaStreamFireAndForget;
   switch (vid) {
-    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
-    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
-    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
-    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
-    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, ff>>>(A, y, s, uv, tl); break;
+    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, dyn_smem(0), ff>>>(A, y, s, uv, tl); break;
+    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, dyn_smem(1), ff>>>(A, y, s, uv, tl); break;
+    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, dyn_smem(2), ff>>>(A, y, s, uv, tl); break;
+    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, dyn_smem(3), ff>>>(A, y, s, uv, tl); break;
+    case 4: spmv_slice_kernel<4><<<grid, kUnitRows, dyn_smem(4), ff>>>(A, y, s, uv, tl); break;
+    default: spmv_slice_kernel<5><<<grid, kUnitRows, dyn_smem(5), ff>>>(A, y, s, uv, tl); break;
   }
 }
 
@@ -317,11 +327,12 @@ __global__ void spmv_device_launch_kernel(SpmvDev A, float *y, int vid, uint64_t
   const unsigned grid = (unsigned)n_units;
   const cudaStream_t ts = cudaStreamTailLaunch;
   switch (vid) {
-    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
-    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
-    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
-    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
-    default: spmv_slice_kernel<4><<<grid, kUnitRows, 0, ts>>>(A, y, s, nullptr, tl); break;
+    case 0: spmv_slice_kernel<0><<<grid, kUnitRows, dyn_smem(0), ts>>>(A, y, s, nullptr, tl); break;
+    case 1: spmv_slice_kernel<1><<<grid, kUnitRows, dyn_smem(1), ts>>>(A, y, s, nullptr, tl); break;
+    case 2: spmv_slice_kernel<2><<<grid, kUnitRows, dyn_smem(2), ts>>>(A, y, s, nullptr, tl); break;
+    case 3: spmv_slice_kernel<3><<<grid, kUnitRows, dyn_smem(3), ts>>>(A, y, s, nullptr, tl); break;
+    case 4: spmv_slice_kernel<4><<<grid, kUnitRows, dyn_smem(4), ts>>>(A, y, s, nullptr, tl); break;
+    default: spmv_slice_kernel<5><<<grid, kUnitRows, dyn_smem(5), ts>>>(A, y, s, nullptr, tl); break;
   }
 }
 
@@ -333,11 +344,12 @@ __global__ void spmv_device_launch_kernel(SpmvDev A, float *y, int vid, uint64_t
 __device__ void eager_launch(int vid, const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p) {
   const unsigned g = p.eager_grid;
   switch (vid) {
-    case 0: spmv_eager_kernel<0><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
-    case 1: spmv_eager_kernel<1><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
-    case 2: spmv_eager_kernel<2><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
-    case 3: spmv_eager_kernel<3><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
-    default: spmv_eager_kernel<4><<<g, kUnitRows, 0, cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 0: spmv_eager_kernel<0><<<g, kUnitRows, dyn_smem(0), cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 1: spmv_eager_kernel<1><<<g, kUnitRows, dyn_smem(1), cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 2: spmv_eager_kernel<2><<<g, kUnitRows, dyn_smem(2), cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 3: spmv_eager_kernel<3><<<g, kUnitRows, dyn_smem(3), cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    case 4: spmv_eager_kernel<4><<<g, kUnitRows, dyn_smem(4), cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
+    default: spmv_eager_kernel<5><<<g, kUnitRows, dyn_smem(5), cudaStreamFireAndForget>>>(A, y, st, p.p_end, p.n_units, p.unit_variant, p.tl); break;
   }
 }
 
@@ -385,7 +397,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     // row makes their units take milliseconds); the warp-cooperative ones
     // (CSR-V, CSR-W) finish any unit in tens of us, and polling inside their
     // loops measured +60% per-unit time on D4 (CSR-W 15 -> 24.6 us).
-    constexpr bool kPolled = VID == 0 || VID == 2 || VID == 3;
+    constexpr bool kPolled = VID == 0 || VID == 2 || VID == 3 || VID == 5;
     if (kPolled && sandbox && p.abort)
       run_unit<VID>(A, j, out,
                     SandboxPoll{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
@@ -496,6 +508,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     spmv_prof_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
+  if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
   prof_unit<VID, false>(A, y, st, p, pv, blockIdx.x);
 }
 
@@ -511,6 +524,7 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
 template <bool CDP>
 __global__ void __launch_bounds__(kUnitRows, DYSEL_PROF_MINB)
     spmv_prof_all_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p) {
+  tma_stage_prologue();
   // programmatic dependent launch: the claim kernels queued behind this one
   // may start as soon as every profiling CTA is resident
   if constexpr (!CDP) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -520,7 +534,8 @@ __global__ void __launch_bounds__(kUnitRows, DYSEL_PROF_MINB)
     case 1: prof_unit<1, CDP>(A, y, st, p, pv, b); break;
     case 2: prof_unit<2, CDP>(A, y, st, p, pv, b); break;
     case 3: prof_unit<3, CDP>(A, y, st, p, pv, b); break;
-    default: prof_unit<4, CDP>(A, y, st, p, pv, b); break;
+    case 4: prof_unit<4, CDP>(A, y, st, p, pv, b); break;
+    default: prof_unit<5, CDP>(A, y, st, p, pv, b); break;
   }
 }
 
@@ -557,6 +572,7 @@ __device__ __forceinline__ uint64_t wait_published(const uint64_t *sw_p) {
 template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     spmv_claim_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
+  if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const uint32_t FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
@@ -686,6 +702,7 @@ template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     spmv_eager_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, uint32_t p_end, uint32_t n_units, uint8_t *uv,
                       uint64_t *tl) {
+  if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
   __shared__ uint32_t s_t;
   if (tl && threadIdx.x == 0) atomicMin((unsigned long long *)&tl[3], (unsigned long long)dysel_globaltimer());
   if (threadIdx.x == 0) s_t = atomicAdd(&st->ticket, 1u);
@@ -715,17 +732,18 @@ static dysel_status spmv_variant_fn(const dysel_slice *s, void *const *args, voi
   SpmvDev A = pl->dev;
   A.x = (const float *)args[1];
   if (s->timer)
-    spmv_slice_timed_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(
+    spmv_slice_timed_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, dyn_smem(VID), (cudaStream_t)stream>>>(
         A, (float *)args[0], *s);
   else
-    spmv_slice_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, 0, (cudaStream_t)stream>>>(A, (float *)args[0], *s,
+    spmv_slice_kernel<VID><<<(unsigned)s->granule_count, kUnitRows, dyn_smem(VID), (cudaStream_t)stream>>>(A, (float *)args[0], *s,
                                                                                               nullptr, nullptr);
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
 
 static dysel_variant_fn kVariantFns[DYSEL_SPMV_NVARIANTS] = {spmv_variant_fn<0>, spmv_variant_fn<1>, spmv_variant_fn<2>,
-                                                             spmv_variant_fn<3>, spmv_variant_fn<4>};
-static const char *kVariantNames[DYSEL_SPMV_NVARIANTS] = {"csr_scalar", "csr_vector", "ell", "jds", "csr_stream"};
+                                                             spmv_variant_fn<3>, spmv_variant_fn<4>,
+                                                             spmv_variant_fn<5>};
+static const char *kVariantNames[DYSEL_SPMV_NVARIANTS] = {"csr_scalar", "csr_vector", "ell", "jds", "csr_stream", "csr_tma"};
 
 struct SpmvCtxState {
   SpmvState *d_state = nullptr;
@@ -743,23 +761,39 @@ dysel_status spmv_ctx_init(dysel_ctx *ctx) {
   if (cudaMallocHost(&s->h_state, sizeof(SpmvState)) != cudaSuccess) return DYSEL_ERR_NOMEM;
   const void *slice[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_slice_kernel<0>, (const void *)spmv_slice_kernel<1>,
                                             (const void *)spmv_slice_kernel<2>, (const void *)spmv_slice_kernel<3>,
-                                            (const void *)spmv_slice_kernel<4>};
+                                            (const void *)spmv_slice_kernel<4>,
+                                            (const void *)spmv_slice_kernel<5>};
   const void *claim[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_claim_kernel<0>, (const void *)spmv_claim_kernel<1>,
                                             (const void *)spmv_claim_kernel<2>, (const void *)spmv_claim_kernel<3>,
-                                            (const void *)spmv_claim_kernel<4>};
+                                            (const void *)spmv_claim_kernel<4>,
+                                            (const void *)spmv_claim_kernel<5>};
   const void *eager[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_eager_kernel<0>, (const void *)spmv_eager_kernel<1>,
                                             (const void *)spmv_eager_kernel<2>, (const void *)spmv_eager_kernel<3>,
-                                            (const void *)spmv_eager_kernel<4>};
+                                            (const void *)spmv_eager_kernel<4>,
+                                            (const void *)spmv_eager_kernel<5>};
+  {   // CSR-T's staging buffers exceed the 48 KB default dynamic limit
+    const int m = (int)dyn_smem(DYSEL_SPMV_CSR_TMA);
+    const void *k5[] = {(const void *)spmv_slice_kernel<5>, (const void *)spmv_slice_timed_kernel<5>,
+                        (const void *)spmv_claim_kernel<5>, (const void *)spmv_eager_kernel<5>,
+                        (const void *)spmv_prof_kernel<5>, (const void *)spmv_prof_all_kernel<true>,
+                        (const void *)spmv_prof_all_kernel<false>};
+    for (const void *k : k5)
+      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, m) != cudaSuccess) return DYSEL_ERR_CUDA;
+  }
   for (int v = 0; v < DYSEL_SPMV_NVARIANTS; ++v) {
     // largest L1 for host launches (tuning knob DYSEL_SPMV_CARVEOUT = percent)
     const char *cv = getenv("DYSEL_SPMV_CARVEOUT");
-    const int carve = cv ? atoi(cv) : (int)cudaSharedmemCarveoutMaxL1;
+    int carve = cv ? atoi(cv) : (int)cudaSharedmemCarveoutMaxL1;
+    // CSR-T holds its staging buffers in static shared memory: the smallest
+    // carveout that keeps the claim kernel's compiled CTAs/SM resident
+    if (v == DYSEL_SPMV_CSR_TMA && !cv)
+      carve = std::min(100, (int)((kClaimMinBlocks[v] * (sizeof(TmaStageBufs) + 2048) * 100 + 232447) / 232448));
     cudaFuncSetAttribute(slice[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
     cudaFuncSetAttribute(eager[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_slice[v], slice[v], kUnitRows, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_slice[v], slice[v], kUnitRows, dyn_smem(v));
     cudaFuncSetAttribute(claim[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_claim[v], claim[v], kUnitRows, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_eager[v], eager[v], kUnitRows, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_claim[v], claim[v], kUnitRows, dyn_smem(v));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_eager[v], eager[v], kUnitRows, dyn_smem(v));
   }
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
@@ -805,6 +839,7 @@ static dysel_status launch_claim(const SpmvDev &A, float *y, SpmvState *st, cons
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kUnitRows);
+  cfg.dynamicSmemBytes = dyn_smem(VID);
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -816,7 +851,7 @@ static dysel_status launch_claim(const SpmvDev &A, float *y, SpmvState *st, cons
 typedef dysel_status (*ClaimLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, uint32_t, unsigned,
                                       cudaStream_t, bool);
 static const ClaimLauncher kClaim[DYSEL_SPMV_NVARIANTS] = {launch_claim<0>, launch_claim<1>, launch_claim<2>,
-                                                           launch_claim<3>, launch_claim<4>};
+                                                           launch_claim<3>, launch_claim<4>, launch_claim<5>};
 
 // Slots per claim: about kClaimNnz nonzeros of work (at least 1, at most a unit).
 constexpr int64_t kClaimNnz = 1024;
@@ -848,11 +883,11 @@ static dysel_status launch_variant_full(dysel_ctx *ctx, dysel_spmv_plan *pl, int
 
 template <int VID>
 static void launch_prof(const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p, uint32_t pv, cudaStream_t s) {
-  spmv_prof_kernel<VID><<<p.c, kUnitRows, 0, s>>>(A, y, st, p, pv);
+  spmv_prof_kernel<VID><<<p.c, kUnitRows, dyn_smem(VID), s>>>(A, y, st, p, pv);
 }
 typedef void (*ProfLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, uint32_t, cudaStream_t);
 static const ProfLauncher kProf[DYSEL_SPMV_NVARIANTS] = {launch_prof<0>, launch_prof<1>, launch_prof<2>, launch_prof<3>,
-                                                         launch_prof<4>};
+                                                         launch_prof<4>, launch_prof<5>};
 
 }  // namespace dysel
 
@@ -905,11 +940,12 @@ dysel_status dysel_debug_spmv_device_launch(dysel_ctx *ctx, dysel_spmv_plan *pl,
   if (how == 0) {
     dysel_slice s = unit_slice(0, pl->n_units, pl->n_units, variant_id);
     switch (variant_id) {
-      case 0: spmv_slice_kernel<0><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
-      case 1: spmv_slice_kernel<1><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
-      case 2: spmv_slice_kernel<2><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
-      case 3: spmv_slice_kernel<3><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
-      default: spmv_slice_kernel<4><<<(unsigned)pl->n_units, kUnitRows, 0, st>>>(A, d_y, s, nullptr, tl); break;
+      case 0: spmv_slice_kernel<0><<<(unsigned)pl->n_units, kUnitRows, dyn_smem(0), st>>>(A, d_y, s, nullptr, tl); break;
+      case 1: spmv_slice_kernel<1><<<(unsigned)pl->n_units, kUnitRows, dyn_smem(1), st>>>(A, d_y, s, nullptr, tl); break;
+      case 2: spmv_slice_kernel<2><<<(unsigned)pl->n_units, kUnitRows, dyn_smem(2), st>>>(A, d_y, s, nullptr, tl); break;
+      case 3: spmv_slice_kernel<3><<<(unsigned)pl->n_units, kUnitRows, dyn_smem(3), st>>>(A, d_y, s, nullptr, tl); break;
+      case 4: spmv_slice_kernel<4><<<(unsigned)pl->n_units, kUnitRows, dyn_smem(4), st>>>(A, d_y, s, nullptr, tl); break;
+    default: spmv_slice_kernel<5><<<(unsigned)pl->n_units, kUnitRows, dyn_smem(5), st>>>(A, d_y, s, nullptr, tl); break;
     }
   } else {
     spmv_device_launch_kernel<<<1, 1, 0, st>>>(A, d_y, variant_id, pl->n_units, how, tl);
@@ -1067,9 +1103,9 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
     }
   } else {   // all K profiling slices in one launch on the stream
     if (cdp)
-      spmv_prof_all_kernel<true><<<p.K * p.c, kUnitRows, 0, st>>>(A, d_y, dst, p);
+      spmv_prof_all_kernel<true><<<p.K * p.c, kUnitRows, pool_dyn_smem(p), st>>>(A, d_y, dst, p);
     else
-      spmv_prof_all_kernel<false><<<p.K * p.c, kUnitRows, 0, st>>>(A, d_y, dst, p);
+      spmv_prof_all_kernel<false><<<p.K * p.c, kUnitRows, pool_dyn_smem(p), st>>>(A, d_y, dst, p);
     DYSEL_TRY(check_launch(ctx, "spmv_prof_all_kernel"));
   }
   if (!cdp && p.p_end < p.n_units) {

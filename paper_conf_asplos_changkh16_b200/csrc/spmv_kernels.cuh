@@ -442,6 +442,129 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, in
   if (lane < nr) out[w * 32 + lane] = acc;
 }
 
+// ------------------------------------------------------------------ CSR-T
+// Bulk-staged CSR (B200 data-placement variant; north_star
+// "TMA or shared-memory staging"): the nonzeros of the warp's 32-row group
+// are moved into shared memory by the bulk-copy (TMA) engine in ONE request
+// per array (cp.async.bulk + mbarrier complete_tx), instead of one dependent
+// col/val load chain per thread; each lane then walks its row from shared
+// memory with kTmaGather x gathers in flight.  Compute is CSR-S's: lane i owns
+// row i and fmas its entries in CSR order from +0, so CSR-T is bit-identical
+// to CSR-S / ELL / JDS.  A group of more than kTmaCap nonzeros (heavy rows),
+// or unaligned col / val (vec_ok = 0), runs the CSR-S code.
+constexpr int kTmaCap = 1024;     // entries staged per warp (4 KB col + 4 KB val)
+constexpr int kTmaGather = 16;    // x gathers in flight per lane
+constexpr int kTmaWarps = kUnitRows / 32;
+struct TmaStageBufs {
+  int32_t col[kTmaWarps][kTmaCap];
+  float val[kTmaWarps][kTmaCap];
+  unsigned long long bar[kTmaWarps];   // one mbarrier per warp, initialised once per CTA
+  uint32_t phase[kTmaWarps];           // its current phase parity
+};
+
+// dynamic shared memory (kernels that can run CSR-T are launched with
+// sizeof(TmaStageBufs) bytes of it, spmv.cu kDynSmem)
+__device__ __forceinline__ TmaStageBufs &tma_stage_bufs() {
+  extern __shared__ __align__(128) unsigned char spmv_dyn_smem[];
+  return *reinterpret_cast<TmaStageBufs *>(spmv_dyn_smem);
+}
+
+__device__ __forceinline__ uint32_t spmv_smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// CTA prologue of every kernel that may run CSR-T: initialise the per-warp
+// mbarriers once (re-initialising a live mbarrier is undefined).  A no-op in a
+// launch without the staging buffers (%dynamic_smem_size too small).
+__device__ __forceinline__ void tma_stage_prologue() {
+  uint32_t dyn;
+  asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(dyn));
+  if (dyn < sizeof(TmaStageBufs)) return;
+  TmaStageBufs &t = tma_stage_bufs();
+  if (threadIdx.x < kTmaWarps) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(spmv_smem_u32(&t.bar[threadIdx.x])) : "memory");
+    t.phase[threadIdx.x] = 0;
+  }
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncthreads();
+}
+
+template <class Poll>
+__device__ __forceinline__ void unit_csr_tma(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
+                                             const Poll &poll) {
+  const uint32_t FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int64_t base = (int64_t)j * kUnitRows + w * 32;
+  const int nr = (int)min((int64_t)32, (int64_t)A.n_rows - base);
+  if (nr <= 0) return;
+  const int rb = lane < nr ? __ldg(A.row_ptr + base + lane) : 0;
+  const int re = lane < nr ? __ldg(A.row_ptr + base + lane + 1) : 0;
+  const int s = __shfl_sync(FULL, rb, 0);
+  const int e = __shfl_sync(FULL, re, nr - 1);
+  const int a = s & ~3;   // 16-byte aligned start (entries [a, s) are loaded, never used)
+  if (!A.vec_ok || e - a > kTmaCap) {
+    unit_csr_scalar(A, j, w, out, poll);
+    return;
+  }
+  TmaStageBufs &tsm = tma_stage_bufs();
+  const int wl = (threadIdx.x >> 5) & (kTmaWarps - 1);   // this warp's buffers (any slot w may run here)
+  const uint64_t px = policy_evict_last();
+  const int nb = (e - a) & ~3;   // bulk part; the < 4 tail entries by lanes 0..2
+  const uint32_t bar = spmv_smem_u32(&tsm.bar[wl]);
+  __syncwarp();   // the previous slot's reads of the buffers and its phase flip are done
+  const uint32_t par = tsm.phase[wl];
+  __syncwarp();
+  if (lane == 0) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(nb * 8) : "memory");
+    if (nb > 0) {
+      const uint64_t pst = policy_evict_first();
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+              spmv_smem_u32(&tsm.col[wl][0])),
+          "l"(A.col + a), "r"(nb * 4), "r"(bar), "l"(pst)
+          : "memory");
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+              spmv_smem_u32(&tsm.val[wl][0])),
+          "l"(A.val + a), "r"(nb * 4), "r"(bar), "l"(pst)
+          : "memory");
+    }
+  }
+  if (lane < (e - a) - nb) {
+    tsm.col[wl][nb + lane] = __ldg(A.col + a + nb + lane);
+    tsm.val[wl][nb + lane] = __ldg(A.val + a + nb + lane);
+  }
+  {
+    uint32_t ok = 0;
+    while (!ok)
+      asm volatile(
+          "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+          : "=r"(ok)
+          : "r"(bar), "r"(par)
+          : "memory");
+  }
+  __syncwarp();   // tail entries stored by lanes; every lane has seen the phase complete
+  if (lane == 0) tsm.phase[wl] = par ^ 1u;
+  const int32_t *cs = tsm.col[wl] - a;
+  const float *vs = tsm.val[wl] - a;
+  float acc = 0.0f;
+  for (int k = rb; k < re; k += kTmaGather) {
+    float v[kTmaGather], xv[kTmaGather];
+#pragma unroll
+    for (int u = 0; u < kTmaGather; ++u) {
+      const bool ok = k + u < re;
+      v[u] = ok ? vs[k + u] : 0.0f;
+      xv[u] = ok ? ld_x(A.x + cs[k + u], px) : 0.0f;
+    }
+#pragma unroll
+    for (int u = 0; u < kTmaGather; ++u)
+      if (k + u < re) acc = __fmaf_rn(v[u], xv[u], acc);
+    if (Poll::active && ((k - rb) & 127) >= 128 - kTmaGather && poll()) break;
+  }
+  if (lane < nr) out[w * 32 + lane] = acc;
+}
+
 // One 32-row warp slot w (0..7) of unit j: rows 256 j + 32 w + lane (JDS:
 // permuted positions 32 w + lane of block j, whose rows lie anywhere in the
 // unit).  The 8 slots of a unit, run by the same variant in any order and by
@@ -453,7 +576,8 @@ __device__ __forceinline__ void run_slot(const SpmvDev &A, uint32_t j, int w, fl
   else if constexpr (VID == 1) unit_csr_vector(A, j, w, out, poll);
   else if constexpr (VID == 2) unit_ell(A, j, w, out, poll);
   else if constexpr (VID == 3) unit_jds(A, j, w, out, poll);
-  else unit_csr_stream(A, j, w, out, poll);
+  else if constexpr (VID == 4) unit_csr_stream(A, j, w, out, poll);
+  else unit_csr_tma(A, j, w, out, poll);
 }
 
 // Whole unit by a 256-thread CTA: warp w runs slot w.
@@ -469,7 +593,8 @@ __device__ __forceinline__ void run_unit_dyn(int vid, const SpmvDev &A, uint32_t
     case 1: run_unit<1>(A, j, out, poll); break;
     case 2: run_unit<2>(A, j, out, poll); break;
     case 3: run_unit<3>(A, j, out, poll); break;
-    default: run_unit<4>(A, j, out, poll); break;
+    case 4: run_unit<4>(A, j, out, poll); break;
+    default: run_unit<5>(A, j, out, poll); break;
   }
 }
 

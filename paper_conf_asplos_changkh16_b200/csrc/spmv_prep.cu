@@ -230,6 +230,7 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
     pl->vids[pl->K++] = DYSEL_SPMV_JDS;
   }
   if (formats_mask & DYSEL_FMT_STREAM) pl->vids[pl->K++] = DYSEL_SPMV_CSR_STREAM;
+  if (formats_mask & DYSEL_FMT_TMA) pl->vids[pl->K++] = DYSEL_SPMV_CSR_TMA;
   if (cudaStreamSynchronize(st) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (default_variant == DYSEL_SPMV_DEFAULT_AUTO) {   // reading A-30: initial version from row statistics
     if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;

@@ -31,11 +31,13 @@ DEFAULT_MODE = FULLY | ASYNC
 V_ATOMICS, V_NONUNIFORM = 1, 2
 ROLE_PRODUCTIVE, ROLE_SANDBOX, ROLE_BATCH, ROLE_PRIVATE, ROLE_EAGER = range(5)
 MAX_VARIANTS = 16
-SPMV_CSR_SCALAR, SPMV_CSR_VECTOR, SPMV_ELL, SPMV_JDS, SPMV_CSR_STREAM = range(5)
-SPMV_NVARIANTS = 5
-SPMV_NAMES = ["csr_scalar", "csr_vector", "ell", "jds", "csr_stream"]
-FMT_ELL, FMT_JDS, FMT_STREAM = 1, 2, 4
-FMT_ALL = FMT_ELL | FMT_JDS | FMT_STREAM
+SPMV_CSR_SCALAR, SPMV_CSR_VECTOR, SPMV_ELL, SPMV_JDS, SPMV_CSR_STREAM, SPMV_CSR_TMA = range(6)
+SPMV_NVARIANTS = 6
+SPMV_NAMES = ["csr_scalar", "csr_vector", "ell", "jds", "csr_stream", "csr_tma"]
+FMT_ELL, FMT_JDS, FMT_STREAM, FMT_TMA = 1, 2, 4, 8
+FMT_ALL = FMT_ELL | FMT_JDS | FMT_STREAM | FMT_TMA
+# default pool: CSR-T (bulk-staged data-placement variant) is opt-in
+FMT_DEFAULT = FMT_ELL | FMT_JDS | FMT_STREAM
 SPMV_DEFAULT_AUTO = -1
 SGEMM_S64, SGEMM_S128, SGEMM_T128x64, SGEMM_T128x128 = range(4)
 SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"]
@@ -250,7 +252,7 @@ class Context:
         return int(dysel_kernel_launches(self.h))
 
     # ------------------------------------------------------------- SpMV
-    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_ALL, default=SPMV_CSR_VECTOR,
+    def spmv_prepare(self, row_ptr, col, val, n_cols, formats=FMT_DEFAULT, default=SPMV_CSR_VECTOR,
                      stream=None) -> SpmvPlan:
         n = row_ptr.numel() - 1
         nnz = col.numel()
