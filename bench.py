@@ -442,6 +442,10 @@ def secondary_workloads(ctx, D, args, stream):
     t4 = {D.SGEMM_NAMES[v]: time_b2b(lambda: ctx.sgemm_variant(v, Ad, Bd, C), 5, stream) for v in (1, 2, 3)}
     td4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY), 5, stream)
     rep4 = ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY, report=True)
+    # hybrid + eager wave: dominated SIMT sandboxes stop (A-32), the default fills free slots (A-33)
+    th4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.01, mode=D.HYBRID | D.ASYNC), 5, stream)
+    reph4 = ctx.sgemm(Ad, Bd, C, f=0.01, mode=D.HYBRID | D.ASYNC, report=True)
+    tn4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY | D.NO_ABORT), 5, stream)
     ta4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY | D.ASYNC | D.HOST_ORCH), 5, stream)
     I4 = 20
     def amort4():
@@ -455,6 +459,9 @@ def secondary_workloads(ctx, D, args, stream):
                          "all_tflops": {k: round(fl4 / v / 1e12, 1) for k, v in t4.items()},
                          "dysel_tflops": round(fl4 / td4 / 1e12, 1), "selected": rep4["selected_name"],
                          "overhead_pct": round((td4 / t4[b4] - 1) * 100, 2),
+                         "no_dominance_overhead_pct": round((tn4 / t4[b4] - 1) * 100, 2),
+                         "hybrid_async_overhead_pct": round((th4 / t4[b4] - 1) * 100, 2),
+                         "hybrid_async_selected": reph4["selected_name"], "hybrid_async_eager_granules": reph4["eager_units"],
                          "host_async_overhead_pct": round((ta4 / t4[b4] - 1) * 100, 2),
                          "amortized_overhead_pct": round((tam4 / t4[b4] - 1) * 100, 2),
                          "tensor_roofline_note": "3xTF32 = 3 tf32 MMAs per fp32 product; ceiling ~ tf32 peak / 3"}

@@ -85,7 +85,8 @@ const char *dysel_status_str(dysel_status s);
 #define DYSEL_SCORE_MAKESPAN 256u /* score = latest CTA end - earliest CTA start (%globaltimer), Fig. 7b */
 #define DYSEL_NO_TAIL 512u      /* SpMV device path: the remainder kernel waits for the profiling kernel to
                                    complete (stream order) instead of starting beside it (PDL) / no CDP2 tail */
-#define DYSEL_NO_ABORT 1024u    /* SpMV device path: never stop dominated sandbox units early */
+#define DYSEL_NO_ABORT 1024u    /* no dominance: never stop dominated sandbox units early (SpMV, A-26) nor decide
+                                   a variant before its profiling CTAs finish (generic launcher, A-32) */
 #define DYSEL_SEQUENTIAL 2048u  /* SpMV device path: profile the variants one after another, each alone on the
                                    GPU (default variant first), scored by makespan (reading A-23) */
 #define DYSEL_DEVICE_LAUNCH 4096u /* SpMV device path, round-1 scheme (ablation): eager kernel and remainder
@@ -166,6 +167,16 @@ typedef struct {
   uint64_t *sel;             /* final packed selection (~0 until profiling completes) */
   /* gated batch: when non-NULL the copy runs only if (*gate & 0xff) == variant */
   const uint64_t *gate;
+  /* dominance (reading A-32; NULL = off): a running variant whose lower-bound
+   * score already exceeds the best completed score cannot win, so it is
+   * decided (maximal score) without waiting for its CTAs; its sandbox CTAs
+   * may stop (dysel_prof_poll).  lb = running sum of the variant's CTA
+   * clock64 cycles (each CTA adds its elapsed cycles when it polls);
+   * decided = 0 running, 1 completed, 2 dominated (set once, by CAS);
+   * units_total = units of the variant's profiling slice. */
+  uint64_t *lb;
+  uint32_t *decided;
+  uint64_t units_total;
 } dysel_slice;
 
 /* A variant = a host function that launches its kernel(s) over a slice on

@@ -79,17 +79,70 @@ __device__ __forceinline__ bool dysel_gate_open(const dysel_slice &s) {
 
 struct dysel_prof_smem {
   unsigned long long t0[32], t1[32], c0[32], c1[32];
+  unsigned long long c_last;   /* thread 0: clock64 of the CTA's last dominance report */
+  int dominated;               /* broadcast of the last dysel_prof_poll result */
 };
+
+/* Packed selection bookkeeping shared by completion and dominance: called
+ * once per variant (by whoever decided it); the last variant publishes. */
+__device__ __forceinline__ void dysel_variant_decided(const dysel_slice &s) {
+  __threadfence();
+  const uint32_t vd = atomicAdd(s.variants_done, 1u) + 1u;
+  if (vd == s.n_variants) {           /* last variant: publish the selection */
+    __threadfence();
+    const unsigned long long fin = atomicAdd((unsigned long long *)s.best, 0ull);
+    atomicExch((unsigned long long *)s.sel, fin);
+  }
+}
 
 /* Call with all threads of the CTA at kernel entry (after any early exit
  * that is uniform for the CTA).  No-op when s.timer == NULL. */
 __device__ __forceinline__ void dysel_prof_begin(const dysel_slice &s, dysel_prof_smem &sm) {
   if (s.timer == nullptr) return;
-  if ((threadIdx.x & 31) == 0) {
-    const uint32_t w = (threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z)) >> 5;
-    sm.c0[w] = dysel_clock64();
-    sm.t0[w] = dysel_globaltimer();
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if ((tid & 31) == 0) {
+    sm.c0[tid >> 5] = dysel_clock64();
+    sm.t0[tid >> 5] = dysel_globaltimer();
   }
+  if (tid == 0) {
+    sm.c_last = sm.c0[0];
+    sm.dominated = 0;
+  }
+}
+
+/* Dominance poll (reading A-32).  Call with ALL threads of the CTA (it holds
+ * one __syncthreads), every few microseconds of work, between
+ * dysel_prof_begin and dysel_prof_end.  Thread 0 adds the cycles elapsed
+ * since its last report to the variant's running sum lb; the variant is
+ * dominated once lb * 64 / (units_total * occupancy) (or lb / units_total
+ * with score_cycles) exceeds the best completed score — its final score can
+ * only be larger — and the first CTA to see it decides the variant (maximal
+ * score).  Returns true when the variant is dominated: a SANDBOX CTA may then
+ * stop (its output is discarded), a productive CTA must finish its tile. */
+__device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof_smem &sm) {
+  if (s.timer == nullptr || s.lb == nullptr) return false;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if (tid == 0 && !sm.dominated) {
+    const unsigned long long now = dysel_clock64();
+    const unsigned long long tot = atomicAdd((unsigned long long *)s.lb, now - sm.c_last) + (now - sm.c_last);
+    sm.c_last = now;
+    int d = *(volatile uint32_t *)s.decided == 2u;
+    if (!d) {
+      const unsigned long long best = *(volatile unsigned long long *)s.best >> 8;
+      const unsigned long long cap = (1ull << 56) - 1;
+      const unsigned long long un = s.units_total ? s.units_total : 1ull;
+      const unsigned long long lbs = s.score_cycles ? tot / un
+                                     : s.occupancy   ? tot * 64ull / (un * (unsigned long long)s.occupancy)
+                                                     : 0ull;   /* makespan scores: no cycle bound */
+      if (best < cap && lbs > best) {
+        d = 1;
+        if (atomicCAS(s.decided, 0u, 2u) == 0u) dysel_variant_decided(s);
+      }
+    }
+    sm.dominated = d;
+  }
+  __syncthreads();
+  return sm.dominated != 0;
 }
 
 /* Call with all threads at the end of the CTA's work.  `units` = units this
@@ -122,7 +175,8 @@ __device__ __forceinline__ void dysel_prof_end(const dysel_slice &s, dysel_prof_
       atomicAdd((unsigned long long *)&slot->units, (unsigned long long)units);
       __threadfence();
       const uint32_t done = atomicAdd(s.ctas_done, 1u) + 1u;
-      if (done == s.ctas_total) {           /* last CTA of this variant */
+      /* last CTA of this variant, unless dominance decided it already */
+      if (done == s.ctas_total && (s.decided == nullptr || atomicCAS(s.decided, 0u, 1u) == 0u)) {
         __threadfence();
         const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
         const unsigned long long b = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
@@ -134,13 +188,7 @@ __device__ __forceinline__ void dysel_prof_end(const dysel_slice &s, dysel_prof_
                            : (b - a);
         if (score > (1ull << 56) - 1) score = (1ull << 56) - 1;
         atomicMin((unsigned long long *)s.best, (score << 8) | (unsigned)s.variant);
-        __threadfence();
-        const uint32_t vd = atomicAdd(s.variants_done, 1u) + 1u;
-        if (vd == s.n_variants) {           /* last variant: publish the selection */
-          __threadfence();
-          const unsigned long long fin = atomicAdd((unsigned long long *)s.best, 0ull);
-          atomicExch((unsigned long long *)s.sel, fin);
-        }
+        dysel_variant_decided(s);
       }
     }
   }

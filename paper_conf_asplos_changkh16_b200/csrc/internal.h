@@ -50,6 +50,8 @@ dysel_status make_plan(dysel_ctx *ctx, const uint64_t U[3], const uint32_t (*wa)
 // Generic (host-launched variants) profiling bookkeeping, one per ctx.
 struct DevProf {
   dysel_timer_slot slot[DYSEL_MAX_VARIANTS];
+  uint64_t lb[DYSEL_MAX_VARIANTS];        // dominance: running cycle sums (A-32)
+  uint32_t decided[DYSEL_MAX_VARIANTS];   // 0 running, 1 completed, 2 dominated
   uint32_t ctas_done[DYSEL_MAX_VARIANTS];
   uint32_t variants_done;
   uint32_t pad;
@@ -93,6 +95,9 @@ struct dysel_ctx {
   cudaEvent_t ev_start = nullptr;
   cudaEvent_t ev_join[DYSEL_MAX_VARIANTS] = {};
   cudaEvent_t ev_fork2 = nullptr;
+  cudaStream_t rem[DYSEL_MAX_VARIANTS] = {};        // gated remainder copies (device path)
+  cudaStream_t wsel = nullptr;                      // wait-for-selection kernel (device path)
+  cudaEvent_t ev_join2[DYSEL_MAX_VARIANTS] = {};
   dysel::DevProf *d_prof = nullptr;
   dysel::DevProf *h_prof = nullptr;  // pinned
   void *d_spmv_state = nullptr;      // persistent-dispatcher state (spmv.cu)

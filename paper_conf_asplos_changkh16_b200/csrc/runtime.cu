@@ -183,12 +183,28 @@ __global__ void init_prof_kernel(DevProf *p, int K, int def) {
     p->slot[i].units = 0;
     p->slot[i].cycles = 0;
     p->ctas_done[i] = 0;
+    p->lb[i] = 0;
+    p->decided[i] = 0;
   }
   if (i == 0) {
     p->variants_done = 0;
     p->best = (((1ull << 56) - 1) << 8) | (uint64_t)def;
     p->sel = ~0ull;
   }
+}
+
+// Device path: stream-order the gated remainder behind the SELECTION rather
+// than behind the profiling kernels' completion — a variant decided by
+// dominance (A-32) may still be finishing productive tiles.  One thread; the
+// selection is always published (every variant is decided by completion or
+// dominance), so the wait ends.
+__global__ void wait_selection_kernel(const uint64_t *sel) {
+  // bounded (5 s): a variant that never calls dysel_prof_end would otherwise
+  // hang the stream; its gated copies then all exit (no variant selected)
+  const uint64_t t0 = dysel_globaltimer();
+  for (uint32_t ns = 64; dysel_ld_acquire_u64(sel) == ~0ull && dysel_globaltimer() - t0 < 5000000000ull;
+       ns = ns < 2048 ? 2 * ns : ns)
+    __nanosleep(ns);
 }
 
 __global__ void gated_copy_kernel(uint4 *dst, const uint4 *src, size_t n16, const uint64_t *gate, int v) {
@@ -358,8 +374,13 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
     if (cudaStreamCreateWithPriority(&ctx->fork[i], cudaStreamNonBlocking, prio_hi) != cudaSuccess)
       return fail(DYSEL_ERR_CUDA);
     if (cudaEventCreateWithFlags(&ctx->ev_join[i], cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+    if (cudaStreamCreateWithPriority(&ctx->rem[i], cudaStreamNonBlocking, prio_lo) != cudaSuccess)
+      return fail(DYSEL_ERR_CUDA);
+    if (cudaEventCreateWithFlags(&ctx->ev_join2[i], cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   }
   if (cudaStreamCreateWithFlags(&ctx->query, cudaStreamNonBlocking) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (cudaStreamCreateWithPriority(&ctx->wsel, cudaStreamNonBlocking, prio_hi) != cudaSuccess)
+    return fail(DYSEL_ERR_CUDA);
   if (cudaEventCreateWithFlags(&ctx->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (cudaEventCreateWithFlags(&ctx->ev_fork2, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (cudaMalloc(&ctx->d_prof, sizeof(DevProf)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
@@ -387,8 +408,11 @@ void dysel_destroy(dysel_ctx *ctx) {
   for (int i = 0; i < DYSEL_MAX_VARIANTS; ++i) {
     if (ctx->fork[i]) cudaStreamDestroy(ctx->fork[i]);
     if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
+    if (ctx->rem[i]) cudaStreamDestroy(ctx->rem[i]);
+    if (ctx->ev_join2[i]) cudaEventDestroy(ctx->ev_join2[i]);
   }
   if (ctx->query) cudaStreamDestroy(ctx->query);
+  if (ctx->wsel) cudaStreamDestroy(ctx->wsel);
   if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
   if (ctx->ev_fork2) cudaEventDestroy(ctx->ev_fork2);
   if (ctx->d_prof) cudaFree(ctx->d_prof);
@@ -560,7 +584,10 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
   const bool score_cycles = (mode & DYSEL_SCORE_CYCLES) != 0;
   // generic ASYNC = the paper's host polling path: heterogeneous user kernels
   // cannot share a device-side ticket scheduler (the SpMV pool does, spmv.cu)
-  const bool host_orch = (mode & DYSEL_HOST_ORCH) != 0 || (mode & DYSEL_ASYNC) != 0;
+  // ASYNC without HOST_ORCH: device path with an eager wave of the default
+  // variant beside the profiling copies (reading A-33); HOST_ORCH: the paper's
+  // host polling + eager chunks
+  const bool host_orch = (mode & DYSEL_HOST_ORCH) != 0;
   const bool async = (mode & DYSEL_ASYNC) != 0;
   // ---- per-variant argument vectors (sandboxes / private outputs, Table 1)
   std::vector<std::vector<void *>> vargs(K, base_args);
@@ -621,6 +648,11 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
     s.score_cycles = score_cycles ? 1u : 0u;
     s.occupancy = variant_occupancy(R, v, mode, ctx->n_sm);
     s.sel = &ctx->d_prof->sel;
+    if (!(mode & DYSEL_NO_ABORT)) {   // reading A-32: dominance
+      s.lb = &ctx->d_prof->lb[v];
+      s.decided = &ctx->d_prof->decided[v];
+      s.units_total = P.c * (uint64_t)P.g[0] * P.g[1] * P.g[2];
+    }
     DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[v], ctx->ev_start, 0));
     DYSEL_TRY(R.v[v].fn(&s, vargs[v].data(), ctx->fork[v], R.v[v].user));
     DYSEL_TRY(check_launch(ctx, "variant profiling copy"));
@@ -632,10 +664,46 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
   const uint64_t rem_end = P.Gn;
   int selected = -1;
   uint64_t eager_units = 0;
+  if (!host_orch && async && rem_begin < rem_end && R.v[R.def].ctas_per_wave > 0) {
+    // ---- eager wave (reading A-33): the default variant fills the
+    // execution slots the profiling copies leave free, on `st`, while they run
+    uint64_t prof_slots = 0;   // profiling CTAs in units of the default's slots
+    for (int v = 0; v < K; ++v)
+      if (R.v[v].ctas_per_wave > 0)
+        prof_slots += (P.c * P.h[v] * R.v[R.def].ctas_per_wave + R.v[v].ctas_per_wave - 1) / R.v[v].ctas_per_wave;
+    const uint64_t free_slots = R.v[R.def].ctas_per_wave > prof_slots ? R.v[R.def].ctas_per_wave - prof_slots : 0;
+    const uint64_t E = std::min<uint64_t>(free_slots / P.h[R.def], rem_end - rem_begin);
+    if (E > 0) {
+      dysel_slice s = base_slice(P);
+      s.variant = R.def;
+      s.role = DYSEL_ROLE_EAGER;
+      s.granule_begin = rem_begin;
+      s.granule_count = E;
+      DYSEL_TRY(R.v[R.def].fn(&s, base_args.data(), st, R.v[R.def].user));
+      DYSEL_TRY(check_launch(ctx, "variant eager wave"));
+      add_slice_rec(rep, s);
+      mark_units(rep, s);
+      rem_begin += E;
+      eager_units = E;
+    }
+  }
   if (!host_orch) {
     // ---- device path: gated remainder, selection never leaves the device
-    for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
-    if (P.mode == DYSEL_SWAP) {
+    const bool dominance = !(mode & DYSEL_NO_ABORT) && P.mode != DYSEL_SWAP;
+    // the remainder is ordered behind the selection only — not behind the
+    // eager wave (its CTAs take the slots the eager ones free) nor, with
+    // dominance, behind dominated variants finishing productive tiles
+    cudaStream_t gate_st = ctx->wsel;
+    DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_start, 0));
+    if (dominance) {
+      wait_selection_kernel<<<1, 1, 0, gate_st>>>(&ctx->d_prof->sel);
+      DYSEL_TRY(check_launch(ctx, "wait_selection_kernel"));
+    } else {
+      for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_join[v], 0));
+    }
+    DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, gate_st));
+    if (P.mode == DYSEL_SWAP) {   // winner's private output copied in (after every private copy is complete)
+      DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_fork2, 0));
       for (int v = 0; v < K; ++v)
         for (size_t k = 0; k < R.sandbox_args[v].size(); ++k) {
           int a = R.sandbox_args[v][k];
@@ -647,9 +715,9 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
             DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync((char *)base_args[a] + n16 * 16, (char *)vargs[v][a] + n16 * 16,
                                                 sandbox_bytes[k] % 16, cudaMemcpyDeviceToDevice, st));
         }
+      DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, st));
     }
     if (rem_begin < rem_end) {
-      DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, st));
       for (int v = 0; v < K; ++v) {
         dysel_slice s = base_slice(P);
         s.variant = v;
@@ -657,13 +725,15 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
         s.granule_begin = rem_begin;
         s.granule_count = rem_end - rem_begin;
         s.gate = &ctx->d_prof->sel;
-        DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[v], ctx->ev_fork2, 0));
-        DYSEL_TRY(R.v[v].fn(&s, base_args.data(), ctx->fork[v], R.v[v].user));
+        DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->rem[v], ctx->ev_fork2, 0));
+        DYSEL_TRY(R.v[v].fn(&s, base_args.data(), ctx->rem[v], R.v[v].user));
         DYSEL_TRY(check_launch(ctx, "variant gated batch"));
-        DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[v], ctx->fork[v]));
+        DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join2[v], ctx->rem[v]));
       }
-      for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
+      for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join2[v], 0));
     }
+    // the call completes with every profiling copy (stream semantics)
+    for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
     // selection for the activation-flag cache: async D2H, resolved lazily
     DYSEL_TRY(push_pending_sel(ctx, sig, &ctx->d_prof->sel, st));
     if (rep) {   // a report costs a D2H copy + sync
@@ -780,7 +850,9 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
       rep->makespan_ns[v] = t.t_end_max - t.t_start_min;
       rep->units[v] = t.units;
       rep->cycles[v] = t.cycles;
-      rep->score[v] = host_score(t, score_cycles, variant_occupancy(R, v, mode, ctx->n_sm));
+      rep->score[v] = ctx->h_prof->decided[v] == 2u   // dominated (A-32): cannot win
+                          ? (1ull << 56) - 1
+                          : host_score(t, score_cycles, variant_occupancy(R, v, mode, ctx->n_sm));
     }
     rep->host_ns = now_ns() - t_host0;
   }

@@ -4,6 +4,7 @@
 // Unit = one 32x32 tile of C; wa = (tile_N/32, tile_M/32) (SURVEY §8 notation).
 #include <cudaTypedefs.h>
 
+#include <algorithm>
 #include <cstring>
 
 #include "internal.h"
@@ -60,6 +61,8 @@ static dysel_status launch_tc(const SgemmArgs &g, float *C, const dysel_slice &s
   return launch_tc_sgemm<BN>(g, C, s, ctas, st);
 }
 
+static uint64_t g_simt_wave[2] = {0, 0};   // resident CTAs (occupancy x #SM) of the two SIMT kernels
+
 template <int VID>
 static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
   const SgemmArgs &g = *(const SgemmArgs *)args[1];
@@ -77,10 +80,13 @@ static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, vo
   }
   const uint64_t ctas = dysel_slice_ctas(*s, wa);
   if (ctas == 0) return DYSEL_OK;
+  // gated remainder of a SIMT variant: one persistent wave (sgemm_simt_kernel)
+  const uint64_t grid = (s->gate && s->timer == nullptr && g_simt_wave[VID & 1] > 0)
+                            ? std::min<uint64_t>(ctas, g_simt_wave[VID & 1]) : ctas;
   if constexpr (VID == DYSEL_SGEMM_S64) {
-    sgemm_simt_kernel<64, 64, 16, 4, 4><<<(unsigned)ctas, 256, 0, st>>>(g, C, *s);
+    sgemm_simt_kernel<64, 64, 16, 4, 4><<<(unsigned)grid, 256, 0, st>>>(g, C, *s);
   } else if constexpr (VID == DYSEL_SGEMM_S128) {
-    sgemm_simt_kernel<128, 128, 8, 8, 8><<<(unsigned)ctas, 256, 0, st>>>(g, C, *s);
+    sgemm_simt_kernel<128, 128, 8, 8, 8><<<(unsigned)grid, 256, 0, st>>>(g, C, *s);
   } else if constexpr (VID == DYSEL_SGEMM_T128x64) {
     DYSEL_TRY(launch_tc<64>(g, C, *s, (unsigned)ctas, st));
   } else {
@@ -105,6 +111,8 @@ dysel_status sgemm_register(dysel_ctx *ctx) {
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[3], sgemm_tma_kernel<128>, 192, TmaCfg<128>::SMEM);
   cudaGetLastError();
   const uint64_t n = (uint64_t)ctx->n_sm;
+  g_simt_wave[0] = (uint64_t)o[0] * n;
+  g_simt_wave[1] = (uint64_t)o[1] * n;
   dysel_variant v[DYSEL_SGEMM_NVARIANTS] = {
       {"simt64x64", sgemm_variant_fn<0>, {2, 2, 1}, sb, 1, 0, nullptr, (uint64_t)o[0] * n},
       {"simt128x128", sgemm_variant_fn<1>, {4, 4, 1}, sb, 1, 0, nullptr, (uint64_t)o[1] * n},
@@ -139,9 +147,6 @@ dysel_status dysel_sgemm(dysel_ctx *ctx, int M, int N, int K, float alpha, const
   if (rep) rep->n_slices = 0;
   if ((int64_t)M * N == 0) return DYSEL_OK;
   SgemmArgs g{M, N, K, alpha, beta, d_A, lda, d_B, ldb, d_C, ldc};
-  // A single-wave SGEMM leaves no room for eager chunks: without HOST_ORCH,
-  // ASYNC runs the device-gated synchronous path (SURVEY §7 hard part 1).
-  if (!(mode & DYSEL_HOST_ORCH)) mode &= ~DYSEL_ASYNC;
   const uint64_t U[3] = {(uint64_t)(N + 31) / 32, (uint64_t)(M + 31) / 32, 1};
   void *args[2] = {d_C, &g};
   const size_t sbytes[1] = {(size_t)M * ldc * sizeof(float)};

@@ -24,8 +24,11 @@ struct SgemmArgs {
 
 // BM x BN tile, TM x TN per thread, BK deep, 256 threads; register-staged
 // double buffering of the next K-slab.
-template <int BM, int BN, int BK, int TM, int TN>
-__device__ __forceinline__ void simt_tile(const SgemmArgs &g, float *__restrict__ C, int m0, int n0) {
+// poll(): called by all threads every 16 K-slabs; true => abandon the tile
+// (a dominated sandbox copy, reading A-32: its output would be discarded).
+template <int BM, int BN, int BK, int TM, int TN, class Poll>
+__device__ __forceinline__ void simt_tile(const SgemmArgs &g, float *__restrict__ C, int m0, int n0,
+                                          const Poll &poll) {
   static_assert((BM / TM) * (BN / TN) == 256, "256 threads");
   constexpr int A_PER = BM * BK / 256, B_PER = BK * BN / 256;
   __shared__ __align__(16) float As[2][BK][BM + 4];
@@ -89,6 +92,7 @@ __device__ __forceinline__ void simt_tile(const SgemmArgs &g, float *__restrict_
     }
     if (kt + 1 < nk) store(buf ^ 1);
     __syncthreads();
+    if ((kt & 15) == 15 && poll()) return;
   }
 #pragma unroll
   for (int i = 0; i < TM; ++i) {
@@ -110,10 +114,25 @@ __global__ void __launch_bounds__(256) sgemm_simt_kernel(SgemmArgs g, float *__r
   __shared__ dysel_prof_smem psm;
   if (!dysel_gate_open(s)) return;
   const uint32_t wa[3] = {BN / 32, BM / 32, 1};
+  if (s.timer == nullptr && s.gate != nullptr) {
+    // gated remainder: a persistent grid of one wave walks the slice's tiles,
+    // so a variant that lost the selection costs one wave of exiting CTAs,
+    // not one per tile (they compete for slots with the winner's grid)
+    const uint64_t n = dysel_slice_ctas(s, wa);
+    for (uint64_t cta = blockIdx.x; cta < n; cta += gridDim.x) {
+      uint64_t u[3];
+      if (dysel_cta_origin(s, wa, cta, u))
+        simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32, []() { return false; });
+      __syncthreads();   // the tile's shared buffers are reused
+    }
+    return;
+  }
   dysel_prof_begin(s, psm);
   uint64_t u[3];
   const bool ok = dysel_cta_origin(s, wa, blockIdx.x, u);
-  if (ok) simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32);
+  if (ok)
+    simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32,
+                                  [&]() { return dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_SANDBOX; });
   dysel_prof_end(s, psm, ok ? wa[0] * wa[1] : 0u);   // units (32x32 tiles) this CTA covered
 }
 
