@@ -211,8 +211,8 @@ def dysel_arm(args, world, rank, local_rank):
     for v in plan.variant_ids:
         for _ in range(2):
             ctx.spmv_variant(plan, v, xd, yl)
-        ts = time_events(lambda: ctx.spmv_variant(plan, v, xd, yl), args.oracle_reps, stream)
-        T_v[D.SPMV_NAMES[v]] = float(np.median(ts))
+        # timed exactly like the DySel steps: back to back between two events
+        T_v[D.SPMV_NAMES[v]] = time_b2b(lambda: ctx.spmv_variant(plan, v, xd, yl), args.oracle_reps, stream)
     best_name = min(T_v, key=T_v.get)
     T_star = T_v[best_name]
     # ---- warmup, then K timed steps (barrier + sync on both sides)
@@ -223,21 +223,18 @@ def dysel_arm(args, world, rank, local_rank):
         dist.barrier()
     launches0 = ctx.kernel_launches()
     with ClockSampler(local_rank) as clk:
-        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
         torch.cuda.synchronize()
+        # K steps back to back between two events on the launching stream
         t_all0 = torch.cuda.Event(enable_timing=True)
         t_all1 = torch.cuda.Event(enable_timing=True)
         t_all0.record(stream)
-        for a, b in ev:
-            a.record(stream)
+        for _ in range(args.steps):
             step()
-            b.record(stream)
         t_all1.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     launches = ctx.kernel_launches() - launches0
-    per_step = [a.elapsed_time(b) * 1e-3 for a, b in ev]
     T_total = t_all0.elapsed_time(t_all1) * 1e-3
     if world > 1:
         t = torch.tensor([T_total], device=dev)
@@ -247,6 +244,12 @@ def dysel_arm(args, world, rank, local_rank):
     value = nbytes_total / T_step / 1e9
     # report of one extra (untimed) launch: selection, scores
     rep = ctx.spmv(plan, xd, yl, f=f, mode=mode, report=True)
+    # selection accuracy over repeated single-shot launches (95%)
+    accuracy = {}
+    for ff in sorted({f, 0.001, 0.005}):
+        sels = [ctx.spmv(plan, xd, yl, f=ff, mode=mode, report=True)["selected_name"] for _ in range(20)]
+        accuracy[str(ff)] = {"exact": round(sum(n == best_name for n in sels) / len(sels), 3),
+                             "within_5pct": round(sum(T_v.get(n, 1e9) <= 1.05 * T_star for n in sels) / len(sels), 3)}
     # ---- amortised: profile once, then the activation flag
     I = args.amortize
     def amort():
@@ -262,6 +265,22 @@ def dysel_arm(args, world, rank, local_rank):
                                                / T_star - 1) * 100, 2)
         ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10, stream)
                                                       / T_star - 1) * 100, 2) for ff in (0.001, 0.005, 0.01, 0.02)}
+        # iterative driver (SURVEY §8f f-3, P:L796-804 / §5.2): 20 power
+        # iterations; profiling on iteration 0 only vs every iteration vs never
+        xi, yi = xd.clone(), torch.empty_like(yl)
+        nit = 20
+        def power(pe, md):
+            xi.copy_(xd)
+            ctx.spmv_power(plan, xi, yi, nit, profile_every=pe, f=f, mode=md)
+        t_never = time_b2b(lambda: power(0, mode | D.NO_PROFILE), 3, stream) / nit
+        t_once = time_b2b(lambda: power(0, mode), 3, stream) / nit
+        t_every = time_b2b(lambda: power(1, mode), 3, stream) / nit
+        ablation["iterative_power_20"] = {
+            "us_per_iter_no_profiling": round(t_never * 1e6, 2),
+            "profile_first_only_overhead_pct": round((t_once / t_never - 1) * 100, 2),
+            "profile_every_iter_overhead_pct": round((t_every / t_never - 1) * 100, 2),
+            "note": "x <- A x / ||A x|| (dysel_spmv_power); reference = the same loop with the activation flag "
+                    "off (default variant = the best pure one on D4)"}
         for dname, dv in (("csr_vector", D.SPMV_CSR_VECTOR), ("jds", D.SPMV_JDS)):
             pd = ctx.spmv_prepare(rp, col, val, A.n_cols, default=dv)
             td = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode), 10, stream)
@@ -318,6 +337,7 @@ def dysel_arm(args, world, rank, local_rank):
                                     "all_ms": {k: round(v * 1e3, 4) for k, v in T_v.items()}},
             "selected": rep["selected_name"], "selection_matches_oracle": rep["selected_name"] == best_name,
             "mode_used": rep["mode_used"], "profiled_units_per_variant": rep["c"],
+            "selection_accuracy_20_launches": accuracy,
             "amortized_overhead_pct": round((ta - T_star) / T_star * 100, 3) if world == 1 else None,
             "amortized_iters": I, "ablation": ablation,
             "e2e": {"value": round(nbytes_total / T_e2e / 1e9, 3), "unit": "GB/s",
@@ -489,7 +509,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="dysel", choices=["dysel", "reference"])
     ap.add_argument("--rows", type=int, default=10_000_000)
-    ap.add_argument("--f", type=float, default=0.002)
+    ap.add_argument("--f", type=float, default=0.001)
     ap.add_argument("--oracle-reps", type=int, default=15)
     ap.add_argument("--amortize", type=int, default=20)
     ap.add_argument("--cpu-reps", type=int, default=5)

@@ -177,6 +177,13 @@ typedef struct {
   uint64_t *lb;
   uint32_t *decided;
   uint64_t units_total;
+  /* wave-quantised score (reading A-34; used when both are non-zero and
+   * score_cycles == 0): predicted full-grid time of the variant =
+   * ceil(grid_ctas / wave_ctas) waves x mean cycles per full CTA
+   * (= sum cycles x units_per_cta / units) */
+  uint64_t grid_ctas;        /* CTAs of the variant's full grid (G_n x CTAs per granule) */
+  uint64_t wave_ctas;        /* CTAs resident at once (occupancy x #SM) */
+  uint32_t units_per_cta;    /* wa[0] x wa[1] x wa[2] */
 } dysel_slice;
 
 /* A variant = a host function that launches its kernel(s) over a slice on
@@ -376,6 +383,35 @@ dysel_status dysel_comm_broadcast(dysel_ctx *ctx, float *d_buf, size_t n, int ro
 dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A,
                                  int lda, const float *d_B, int ldb, float beta, float *d_C, int ldc,
                                  float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+
+/* --------------------------------------------------------- iterative driver */
+/* Iterative use of a DySel kernel: the paper's activation
+ * flag profiles an iterative kernel on its first invocation and reuses the
+ * selection afterwards; §5.2 measures the per-iteration cost of
+ * profiling every iteration instead.  Power iteration on a
+ * square matrix, n_iter times:
+ *     y_k = A x_k  (dysel_spmv),   x_{k+1} = y_k / ||y_k||_2
+ * (x_{k+1} = 0 if y_k = 0).  d_x: device fp32 [n], in x_0, out x_{n_iter}
+ * (overwritten every iteration); d_y: device fp32 [n], out y_{n_iter-1}.
+ * profile_every: 0 = profile iteration 0 only (activation flag off
+ * afterwards: cached selection), p > 0 = profile iterations 0, p, 2p, ...
+ * d_norms: nullable DEVICE fp64 [n_iter], ||y_k||_2 (fp64 two-pass reduction
+ * in a fixed order: deterministic).  rep: report of iteration 0.  Errors:
+ * DYSEL_ERR_INVALID for a non-square plan, n_iter < 0 or profile_every < 0.
+ * Stream-ordered on `stream`; blocks only where dysel_spmv's activation-flag
+ * path waits for iteration 0's selection. */
+dysel_status dysel_spmv_power(dysel_ctx *ctx, dysel_spmv_plan *plan, float *d_x, float *d_y, int n_iter,
+                              int profile_every, float profile_fraction, uint32_t mode, void *stream,
+                              double *d_norms, dysel_report *rep);
+/* Row-sharded power iteration (§8e): every rank holds the full x and y
+ * (n = bounds[world]); each iteration is dysel_spmv_sharded (local rows +
+ * y allgather, the y -> x exchange) followed by the same deterministic
+ * normalisation on every rank.  Arguments as dysel_spmv_power /
+ * dysel_spmv_sharded. */
+dysel_status dysel_spmv_power_sharded(dysel_ctx *ctx, dysel_spmv_plan *local_plan, const int64_t *bounds,
+                                      float *d_x, float *d_y, int64_t n, int n_iter, int profile_every,
+                                      float profile_fraction, uint32_t mode, void *stream, double *d_norms,
+                                      dysel_report *rep);
 
 /* ------------------------------------------------------------------- debug */
 /* Number of dysel kernels launched by this ctx so far (bench.py's gpu_launches). */

@@ -83,6 +83,25 @@ struct dysel_prof_smem {
   int dominated;               /* broadcast of the last dysel_prof_poll result */
 };
 
+/* Score from a cycle sum `cy` over `un` units (cap on un == 0): wave-quantised
+ * full-grid prediction (A-34) when the slice declares its grid and wave,
+ * else occupancy-normalised time per unit per slot (A-6), else cycles/unit. */
+__host__ __device__ __forceinline__ unsigned long long dysel_cycle_score(const dysel_slice &s, unsigned long long cy,
+                                                                         unsigned long long un) {
+  const unsigned long long cap = (1ull << 56) - 1;
+  if (un == 0) return cap;
+  unsigned long long r;
+  if (s.score_cycles)
+    r = cy / un;
+  else if (s.grid_ctas && s.wave_ctas && s.units_per_cta)
+    r = ((s.grid_ctas + s.wave_ctas - 1) / s.wave_ctas) * (cy * (unsigned long long)s.units_per_cta / un);
+  else if (s.occupancy)
+    r = cy * 64ull / (un * (unsigned long long)s.occupancy);
+  else
+    return cap;
+  return r < cap ? r : cap;
+}
+
 /* Packed selection bookkeeping shared by completion and dominance: called
  * once per variant (by whoever decided it); the last variant publishes. */
 __device__ __forceinline__ void dysel_variant_decided(const dysel_slice &s) {
@@ -131,9 +150,10 @@ __device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof
       const unsigned long long best = *(volatile unsigned long long *)s.best >> 8;
       const unsigned long long cap = (1ull << 56) - 1;
       const unsigned long long un = s.units_total ? s.units_total : 1ull;
-      const unsigned long long lbs = s.score_cycles ? tot / un
-                                     : s.occupancy   ? tot * 64ull / (un * (unsigned long long)s.occupancy)
-                                                     : 0ull;   /* makespan scores: no cycle bound */
+      /* a lower bound of the final score (tot <= final cycle sum, un >= final
+       * units); makespan scores have no cycle bound */
+      const bool cyc = s.score_cycles || (s.grid_ctas && s.wave_ctas && s.units_per_cta) || s.occupancy;
+      const unsigned long long lbs = cyc ? dysel_cycle_score(s, tot, un) : 0ull;
       if (best < cap && lbs > best) {
         d = 1;
         if (atomicCAS(s.decided, 0u, 2u) == 0u) dysel_variant_decided(s);
@@ -184,7 +204,7 @@ __device__ __forceinline__ void dysel_prof_end(const dysel_slice &s, dysel_prof_
         const unsigned long long un = atomicAdd((unsigned long long *)&slot->units, 0ull);
         unsigned long long score =
             s.score_cycles ? (un ? cy / un : (1ull << 56) - 1)
-            : s.occupancy  ? (un ? cy * 64ull / (un * (unsigned long long)s.occupancy) : (1ull << 56) - 1)
+            : (s.occupancy || (s.grid_ctas && s.wave_ctas)) ? dysel_cycle_score(s, cy, un)
                            : (b - a);
         if (score > (1ull << 56) - 1) score = (1ull << 56) - 1;
         atomicMin((unsigned long long *)s.best, (score << 8) | (unsigned)s.variant);

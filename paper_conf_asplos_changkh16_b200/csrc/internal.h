@@ -104,6 +104,7 @@ struct dysel_ctx {
   void *h_spmv_rep = nullptr;        // pinned copy of its report area
   dysel::ScratchBuf sandbox[2 * DYSEL_MAX_VARIANTS];
   dysel::ScratchBuf unit_variant;    // device bytes, one per granule
+  dysel::ScratchBuf norm_part;       // iterate.cu: fp64 norm partials
   dysel::PendingSel pending[dysel::kPendingRing];
   uint64_t *h_pending_sel = nullptr;   // pinned + mapped, kPendingRing words
   uint64_t *d_pending_sel = nullptr;   // device alias of h_pending_sel

@@ -271,22 +271,40 @@ static dysel_slice base_slice(const Plan &p) {
   return s;
 }
 
-// same rule as dysel_prof_end (dysel_device.cuh)
-static uint64_t host_score(const dysel_timer_slot &t, bool cycles, uint32_t occupancy) {
-  const uint64_t cap = (1ull << 56) - 1;
-  uint64_t s = cycles      ? (t.units ? t.cycles / t.units : cap)
-               : occupancy ? (t.units ? t.cycles * 64ull / (t.units * (uint64_t)occupancy) : cap)
-                           : (t.t_end_max - t.t_start_min);
-  return std::min(s, cap);
-}
-
 // resident CTAs per SM of variant v, when every variant declares ctas_per_wave
-// (the occupancy-normalised score needs all of them), else 0 (makespan)
+// (the cycle-based scores need all of them), else 0 (makespan)
 static uint32_t variant_occupancy(const Registered &R, int v, uint32_t mode, int n_sm) {
   if (mode & DYSEL_SCORE_MAKESPAN) return 0;
   for (const auto &x : R.v)
     if (x.ctas_per_wave == 0) return 0;
   return (uint32_t)std::max<uint64_t>(1, R.v[v].ctas_per_wave / (uint64_t)std::max(1, n_sm));
+}
+
+// Score parameters of variant v (dysel_slice score fields): cycles/unit
+// (DYSEL_SCORE_CYCLES); else, when every variant declares ctas_per_wave, the
+// wave-quantised full-grid prediction (reading A-34): ceil(grid CTAs / wave)
+// x mean cycles per CTA; else makespan (Fig. 7b).
+static void set_score_params(dysel_slice &s, const Registered &R, const Plan &P, int v, uint32_t mode, int n_sm) {
+  s.score_cycles = (mode & DYSEL_SCORE_CYCLES) ? 1u : 0u;
+  s.occupancy = variant_occupancy(R, v, mode, n_sm);
+  if (!s.score_cycles && s.occupancy) {
+    s.grid_ctas = P.Gn * P.h[v];
+    s.wave_ctas = R.v[v].ctas_per_wave;
+    s.units_per_cta = R.v[v].wa[0] * R.v[v].wa[1] * R.v[v].wa[2];
+  }
+}
+
+// same rule as dysel_prof_end (dysel_device.cuh)
+static uint64_t host_score(const dysel_timer_slot &t, const dysel_slice &sp) {
+  if (sp.score_cycles || sp.occupancy) return dysel_cycle_score(sp, t.cycles, t.units);
+  return std::min<uint64_t>(t.t_end_max - t.t_start_min, (1ull << 56) - 1);
+}
+static uint64_t host_score(const dysel_timer_slot &t, const Registered &R, const Plan &P, int v, uint32_t mode,
+                           int n_sm) {
+  dysel_slice sp;
+  memset(&sp, 0, sizeof(sp));
+  set_score_params(sp, R, P, v, mode, n_sm);
+  return host_score(t, sp);
 }
 
 static void fill_report_common(dysel_report *rep, const Plan &p, int mode_used, int profiled, int selected) {
@@ -423,6 +441,7 @@ void dysel_destroy(dysel_ctx *ctx) {
   for (auto &b : ctx->sandbox)
     if (b.ptr) cudaFree(b.ptr);
   if (ctx->unit_variant.ptr) cudaFree(ctx->unit_variant.ptr);
+  if (ctx->norm_part.ptr) cudaFree(ctx->norm_part.ptr);
   comm_free(ctx);
   delete ctx;
 }
@@ -581,7 +600,6 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
     if (rep) rep->host_ns = now_ns() - t_host0;
     return DYSEL_OK;
   }
-  const bool score_cycles = (mode & DYSEL_SCORE_CYCLES) != 0;
   // generic ASYNC = the paper's host polling path: heterogeneous user kernels
   // cannot share a device-side ticket scheduler (the SpMV pool does, spmv.cu)
   // ASYNC without HOST_ORCH: device path with an eager wave of the default
@@ -645,8 +663,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
     s.best = &ctx->d_prof->best;
     s.variants_done = &ctx->d_prof->variants_done;
     s.n_variants = (uint32_t)K;
-    s.score_cycles = score_cycles ? 1u : 0u;
-    s.occupancy = variant_occupancy(R, v, mode, ctx->n_sm);
+    set_score_params(s, R, P, v, mode, ctx->n_sm);
     s.sel = &ctx->d_prof->sel;
     if (!(mode & DYSEL_NO_ABORT)) {   // reading A-32: dominance
       s.lb = &ctx->d_prof->lb[v];
@@ -772,7 +789,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
                                             cudaMemcpyDeviceToHost, ctx->query));
         DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(ctx->query));
         uint64_t pk =
-            (host_score(ctx->h_prof->slot[v], score_cycles, variant_occupancy(R, v, mode, ctx->n_sm)) << 8) |
+            (host_score(ctx->h_prof->slot[v], R, P, v, mode, ctx->n_sm) << 8) |
             (uint64_t)v;
         if (pk < best_pack) {
           best_pack = pk;
@@ -852,7 +869,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
       rep->cycles[v] = t.cycles;
       rep->score[v] = ctx->h_prof->decided[v] == 2u   // dominated (A-32): cannot win
                           ? (1ull << 56) - 1
-                          : host_score(t, score_cycles, variant_occupancy(R, v, mode, ctx->n_sm));
+                          : host_score(t, R, P, v, mode, ctx->n_sm);
     }
     rep->host_ns = now_ns() - t_host0;
   }

@@ -514,10 +514,11 @@ __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
 
 // All K profiling slices in ONE launch (no forked streams / joins): CTA b runs
 // unit b / K of pool variant b mod K (interleaved start order).  The register
-// cap is generous (1 CTA/SM guaranteed) so each variant's code is compiled as
-// in its own kernel; its slice is far below one wave, so occupancy does not
-// shape the measured per-unit time, and the score is normalised by the plain
-// kernel's occupancy anyway.
+// cap is generous (128 registers): each variant's code is compiled as in its
+// own kernel.  A 4-CTA/SM cap (64 registers, so profiling CTAs leave more
+// room to the eager claim CTAs) measured no better on D4 (+5.0-5.4% vs
+// +4.2% per step, same box).  The score is normalised by the plain kernel's
+// occupancy, so the cap does not bias the selection.
 #ifndef DYSEL_PROF_MINB
 #define DYSEL_PROF_MINB 1
 #endif

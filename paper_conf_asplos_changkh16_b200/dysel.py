@@ -106,6 +106,10 @@ dysel_comm_unique_id = _sig("dysel_comm_unique_id", c_int, P)
 dysel_comm_init = _sig("dysel_comm_init", c_int, P, P, c_int, c_int)
 dysel_partition_rows = _sig("dysel_partition_rows", c_int, P, c_i64, c_int, P)
 dysel_spmv_sharded = _sig("dysel_spmv_sharded", c_int, P, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_spmv_power = _sig("dysel_spmv_power", c_int, P, P, P, P, c_int, c_int, c_float, c_u32, P, P,
+                        ctypes.POINTER(Report))
+dysel_spmv_power_sharded = _sig("dysel_spmv_power_sharded", c_int, P, P, P, P, P, c_i64, c_int, c_int, c_float, c_u32,
+                                P, P, ctypes.POINTER(Report))
 dysel_comm_broadcast = _sig("dysel_comm_broadcast", c_int, P, P, c_size, c_int, P)
 dysel_sgemm_sharded = _sig("dysel_sgemm_sharded", c_int, P, c_int, c_int, c_int, c_float, P, c_int, P, c_int, c_float,
                            P, c_int, c_float, c_u32, P, ctypes.POINTER(Report))
@@ -272,6 +276,16 @@ class Context:
             return None
         return report_dict(rep, SPMV_NAMES, bytes(uv) if uv is not None else None)
 
+    def spmv_power(self, plan, x, y, n_iter, profile_every=0, f=0.02, mode=DEFAULT_MODE, norms=None, report=False,
+                   stream=None):
+        """Power iteration x <- A x / ||A x|| (dysel_spmv_power); x in/out, y = A x of the last iteration,
+        norms: optional device float64 [n_iter] receiving ||A x_k||."""
+        rep, keep, uv = (_make_report(0) if report else (None, None, None))
+        self._check(dysel_spmv_power(self.h, plan.handle, _ptr(x), _ptr(y), int(n_iter), int(profile_every), float(f),
+                                     int(mode), _stream(stream), _ptr(norms) if norms is not None else None,
+                                     ctypes.byref(rep) if rep is not None else None))
+        return report_dict(rep, SPMV_NAMES) if rep is not None else None
+
     def debug_spmv_device_launch(self, plan, variant_id, x, y, how, stream=None, resident=False):
         """Full grid of one variant launched from the host (0) / device fire-and-forget (1) / tail (2);
         resident=True returns the max resident CTAs per SM."""
@@ -351,6 +365,16 @@ class Context:
         rep, keep, uv = (_make_report(0) if report else (None, None, None))
         self._check(dysel_spmv_sharded(self.h, local_plan.handle, b, _ptr(x), _ptr(y), float(f), int(mode),
                                        _stream(stream), ctypes.byref(rep) if rep is not None else None))
+        return report_dict(rep, SPMV_NAMES) if rep is not None else None
+
+    def spmv_power_sharded(self, local_plan, bounds, x, y, n_iter, profile_every=0, f=0.02, mode=DEFAULT_MODE,
+                           norms=None, report=False, stream=None):
+        b = (c_i64 * len(bounds))(*bounds)
+        rep, keep, uv = (_make_report(0) if report else (None, None, None))
+        self._check(dysel_spmv_power_sharded(self.h, local_plan.handle, b, _ptr(x), _ptr(y), int(bounds[-1]),
+                                             int(n_iter), int(profile_every), float(f), int(mode), _stream(stream),
+                                             _ptr(norms) if norms is not None else None,
+                                             ctypes.byref(rep) if rep is not None else None))
         return report_dict(rep, SPMV_NAMES) if rep is not None else None
 
     def sgemm_sharded(self, A, B, C, alpha=1.0, beta=0.0, f=0.02, mode=DEFAULT_MODE, report=False, stream=None):

@@ -18,14 +18,13 @@ A = d4_powerlaw()
 x = torch.from_numpy(uniform_f32(10010, A.n_cols)).cuda()
 rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
 y = torch.empty(A.n_rows, device="cuda")
-for fm, label in ((D.FMT_ALL, "pool4"), (D.FMT_STREAM, "pool3")):
-    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, formats=fm, default=4)
+for fm, label in ((D.FMT_DEFAULT, "pool4"),):
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, formats=fm, default=D.SPMV_DEFAULT_AUTO)
     T = b2b(lambda: ctx.spmv_variant(plan, 4, x, y))
     print(label, "pure csr_stream", round(T, 1), "us", flush=True)
-    for name, mode, f in [("hyb_async", D.AUTO | D.ASYNC, 0.005), ("hyb_async", D.AUTO | D.ASYNC, 0.001),
-                          ("hyb_async", D.AUTO | D.ASYNC, 0.0005),
-                          ("hyb_async_noabort", D.HYBRID | D.ASYNC | D.NO_ABORT, 0.005),
-                          ("fully_async", D.FULLY | D.ASYNC, 0.001), ("hyb_sync", D.AUTO, 0.005)]:
+    for name, mode, f in [("hyb_async", D.AUTO | D.ASYNC, 0.002), ("hyb_async", D.AUTO | D.ASYNC, 0.001),
+                          ("hyb_async", D.AUTO | D.ASYNC, 0.0005), ("no_profile", D.AUTO | D.NO_PROFILE, 0.002),
+                          ("fully_async", D.FULLY | D.ASYNC, 0.002), ("hyb_sync", D.AUTO, 0.002)]:
         t = b2b(lambda: ctx.spmv(plan, x, y, f=f, mode=mode))
         r = ctx.spmv(plan, x, y, f=f, mode=mode, report=True)
         print(f"  {label} {name:18s} f={f:<7} {t:7.1f} us ovh {100*(t/T-1):5.1f}% c={r['c']} eager={r['eager_units']} "

@@ -23,7 +23,7 @@ __all__ = [
     "CSR", "rng", "uniform_f32", "d1_bus", "d3_fem", "d4_powerlaw",
     "powerlaw_alpha", "powerlaw_lengths", "d6_random", "d6_diag", "identity",
     "small_int_csr", "small_int_vector", "sgemm_inputs", "small_int_gemm",
-    "random_lengths_csr", "csr_from_lengths",
+    "random_lengths_csr", "csr_from_lengths", "laplacian_2d",
 ]
 
 
@@ -123,6 +123,30 @@ def d3_fem(grid=383, radius=2, val_seed=383) -> CSR:
     rows = np.concatenate(rows_l)
     cols = np.concatenate(cols_l)
     return _csr_from_pattern(n, n, rows, cols, val_seed)
+
+
+def laplacian_2d(grid: int) -> CSR:
+    """5-point Dirichlet Laplacian on a grid x grid mesh (input for the
+    iterative driver's parity tests): 4 on the diagonal, -1 to
+    the four neighbours, row-major node order, ascending columns."""
+    n = grid * grid
+    i, j = np.divmod(np.arange(n, dtype=np.int64), grid)
+    rows_l, cols_l, vals_l = [], [], []
+    for di, dj, v in ((-1, 0, -1.0), (0, -1, -1.0), (0, 0, 4.0), (0, 1, -1.0), (1, 0, -1.0)):
+        ii, jj = i + di, j + dj
+        ok = (ii >= 0) & (ii < grid) & (jj >= 0) & (jj < grid)
+        rows_l.append(np.nonzero(ok)[0])
+        cols_l.append((ii * grid + jj)[ok])
+        vals_l.append(np.full(int(ok.sum()), v))
+    rows = np.concatenate(rows_l)
+    cols = np.concatenate(cols_l)
+    vals = np.concatenate(vals_l)
+    order = np.lexsort((cols, rows))
+    rows, cols, vals = rows[order], cols[order], vals[order]
+    row_ptr = np.zeros(n + 1, np.int64)
+    np.add.at(row_ptr, rows + 1, 1)
+    np.cumsum(row_ptr, out=row_ptr)
+    return CSR(n, n, row_ptr.astype(np.int32), cols.astype(np.int32), vals.astype(np.float32))
 
 
 # --------------------------------------------------------------------------- D4
