@@ -423,6 +423,34 @@ def secondary_workloads(ctx, D, args, stream):
                      "dysel_forced_us": round(t6 * 1e6, 2), "selected": rep6["selected_name"],
                      "all_us": {k: round(v * 1e6, 2) for k, v in r6.items()}}
         plan6.destroy()
+    # f-4: stencil pool, Parboil-default-shaped 512 x 512 x 64 grid
+    nz, ny, nx = 64, 512, 512
+    a3 = torch.from_numpy(uniform_f32(64, (nz, ny, nx))).cuda()
+    o3 = torch.empty_like(a3)
+    c0, c1 = 0.8125, 0.15625
+    ts3 = {D.STENCIL_NAMES[v]: time_b2b(lambda: ctx.stencil_variant(v, a3, o3, c0, c1), 20, stream) for v in range(3)}
+    b3 = min(ts3, key=ts3.get)
+    td3 = time_b2b(lambda: ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC), 20, stream)
+    r3 = ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC, report=True)
+    tf3 = time_b2b(lambda: ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE), 20, stream)
+    rf3 = ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE, report=True)
+    def amort3():
+        ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE)
+        for _ in range(19):
+            ctx.stencil(a3, o3, c0, c1, mode=D.NO_PROFILE)
+    tam3 = time_b2b(amort3, 3, stream) / 20
+    sb3 = 2 * 4 * nx * ny * nz     # algorithmic: read in once, write out once
+    out["stencil_512x512x64"] = {"best_variant": b3, "best_us": round(ts3[b3] * 1e6, 2),
+                                 "best_gbs": round(sb3 / ts3[b3] / 1e9, 1),
+                                 "dysel_us": round(td3 * 1e6, 2), "selected": r3["selected_name"],
+                                 "profiled": r3["profiled"], "overhead_pct": round((td3 / ts3[b3] - 1) * 100, 2),
+                                 "forced_single_shot_overhead_pct": round((tf3 / ts3[b3] - 1) * 100, 2),
+                                 "forced_selected": rf3["selected_name"],
+                                 "amortized_overhead_pct": round((tam3 / ts3[b3] - 1) * 100, 2),
+                                 "all_us": {k: round(v * 1e6, 2) for k, v in ts3.items()},
+                                 "note": "in + out 134 MB > L2; fully|async, f = 0.02 (profiled unless the default's grid fits one "
+                                         "wave, A-3b); forced: profile once; amortised: forced once + 19 activation-flag "
+                                         "calls"}
     # D2m: Parboil-medium SGEMM 1024 x 992 x 1056
     M, K, N = 1024, 992, 1056
     Ah, Bh, _ = sgemm_inputs(M, K, N)

@@ -360,6 +360,26 @@ dysel_status dysel_sgemm_variant(dysel_ctx *ctx, int variant_id, int M, int N, i
                                  const float *d_A, int lda, const float *d_B, int ldb, float beta,
                                  float *d_C, int ldc, void *stream);
 
+/* ---------------------------------------------------------------- stencil
+ * One 3-D 7-point Jacobi step (the paper's stencil case with
+ * three versions of work-assignment factor 1, 64x and 128x):
+ * fp32 arrays [nz][ny][nx] (x fastest), d_in and d_out distinct device
+ * buffers of nx*ny*nz floats (caller-owned).  Interior points:
+ *   out = c1 * (((((in[z-1] + in[z+1]) + in[y-1]) + in[y+1]) + in[x-1]) + in[x+1]) - c0 * in
+ * (this association order, fp32, round to nearest, no contraction: all
+ * variants are bit-identical); boundary points (any coordinate 0 or n-1):
+ * out = in (reading A-37).  Unit = 32 x 4 x 1 points.  Built-in variants:
+ * 0 base (thread per point, wa 1x1x1), 1 z-march (thread per (x, y) column
+ * over 64 z-planes, wa 1x1x64), 2 tiled (64x4 tile staged plane by plane in
+ * shared memory + z-march, wa 2x1x64).  nx, ny, nz >= 0 (0 volume: no-op);
+ * DYSEL_ERR_INVALID for NULL or aliased buffers. */
+enum { DYSEL_STENCIL_BASE = 0, DYSEL_STENCIL_ZMARCH = 1, DYSEL_STENCIL_TILED = 2, DYSEL_STENCIL_NVARIANTS = 3 };
+dysel_status dysel_stencil(dysel_ctx *ctx, int nx, int ny, int nz, float c0, float c1, const float *d_in,
+                           float *d_out, float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+/* Full-grid run of one stencil variant (exhaustive oracle timing). */
+dysel_status dysel_stencil_variant(dysel_ctx *ctx, int variant_id, int nx, int ny, int nz, float c0, float c1,
+                                   const float *d_in, float *d_out, void *stream);
+
 /* --------------------------------------------------------------- multi-GPU
  * Row-sharded SpMV / M-sharded SGEMM over NCCL (the paper is
  * single-GPU).  nccl_unique_id points to the 128-byte

@@ -129,11 +129,17 @@ int reserve_pending_sel(dysel_ctx *ctx, uint64_t **d_slot);
 dysel_status commit_pending_sel(dysel_ctx *ctx, int slot, const std::string &sig, cudaStream_t st);
 // move landed selections into the cache; block_sig != NULL waits for that sig
 void resolve_pending(dysel_ctx *ctx, const char *block_sig);
+// dysel_launch with a selection-cache key distinct from the registry sig
+dysel_status launch_keyed(dysel_ctx *ctx, const char *sig, const char *key, const uint64_t ndrange_units[3], float f,
+                          uint32_t mode, void *const *args, int n_args, const size_t *sandbox_bytes, void *stream,
+                          dysel_report *rep);
 // spmv.cu
 dysel_status spmv_ctx_init(dysel_ctx *ctx);
 void spmv_ctx_free(dysel_ctx *ctx);
 // sgemm.cu
 dysel_status sgemm_register(dysel_ctx *ctx);
+// stencil.cu
+dysel_status stencil_register(dysel_ctx *ctx);
 // comm.cu
 void comm_free(dysel_ctx *ctx);
 }  // namespace dysel

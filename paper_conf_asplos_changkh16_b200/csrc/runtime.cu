@@ -410,6 +410,7 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
     if (cudaEventCreateWithFlags(&ctx->pending[i].ev, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (spmv_ctx_init(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   if (sgemm_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
+  if (stencil_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   uint64_t tick = 0;
   double cpn = 0;
   if (dysel_timer_calibrate(ctx, 1u << 16, 20000, &tick, &cpn) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
@@ -492,7 +493,10 @@ dysel_status dysel_register_variants(dysel_ctx *ctx, const char *sig, const dyse
   }
   r.def = default_variant;
   ctx->reg[sig] = std::move(r);
-  ctx->sel_cache.erase(sig);
+  // drop cached selections of the sig and of its shape-keyed entries (sig#...)
+  const std::string pre = std::string(sig) + "#";
+  for (auto c = ctx->sel_cache.begin(); c != ctx->sel_cache.end();)
+    c = (c->first == sig || c->first.compare(0, pre.size(), pre) == 0) ? ctx->sel_cache.erase(c) : std::next(c);
   return DYSEL_OK;
 }
 
@@ -541,6 +545,17 @@ dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key) {
 dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrange_units[3], float f, uint32_t mode,
                           void *const *args, int n_args, const size_t *sandbox_bytes, void *stream_v,
                           dysel_report *rep) {
+  return dysel::launch_keyed(ctx, sig, sig, ndrange_units, f, mode, args, n_args, sandbox_bytes, stream_v, rep);
+}
+
+}  // extern "C"
+
+// The selection cache (activation flag) is keyed by `key` (reading A-22):
+// kernel_sig for dysel_launch, sig + problem shape for the built-in SGEMM and
+// stencil pools (a selection made for one shape is not reused for another).
+dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *key, const uint64_t ndrange_units[3],
+                                 float f, uint32_t mode, void *const *args, int n_args, const size_t *sandbox_bytes,
+                                 void *stream_v, dysel_report *rep) {
   const uint64_t t_host0 = now_ns();
   if (!ctx || !sig || !ndrange_units || n_args < 0 || (n_args > 0 && !args)) {
     set_error(ctx, "dysel_launch: invalid arguments");
@@ -585,8 +600,8 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
   std::vector<void *> base_args(args, args + n_args);
   if (!P.active) {   // activation flag off / small workload: one plain batch copy
     int v = R.def;
-    resolve_pending(ctx, sig);
-    auto c = ctx->sel_cache.find(sig);
+    resolve_pending(ctx, key);
+    auto c = ctx->sel_cache.find(key);
     if (c != ctx->sel_cache.end() && c->second < K) v = c->second;
     dysel_slice s = base_slice(P);
     s.granule_count = P.Gn;
@@ -752,12 +767,12 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
     // the call completes with every profiling copy (stream semantics)
     for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
     // selection for the activation-flag cache: async D2H, resolved lazily
-    DYSEL_TRY(push_pending_sel(ctx, sig, &ctx->d_prof->sel, st));
+    DYSEL_TRY(push_pending_sel(ctx, key, &ctx->d_prof->sel, st));
     if (rep) {   // a report costs a D2H copy + sync
       DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(ctx->h_prof, ctx->d_prof, sizeof(DevProf), cudaMemcpyDeviceToHost, st));
       DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
       selected = (int)(ctx->h_prof->sel & 0xff);
-      ctx->sel_cache[sig] = selected;
+      ctx->sel_cache[key] = selected;
     }
   } else if (!async) {
     // ---- paper host path, synchronous
@@ -839,7 +854,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
       add_slice_rec(rep, s);
       mark_units(rep, s);
     }
-    ctx->sel_cache[sig] = selected;
+    ctx->sel_cache[key] = selected;
   }
   if (rep) {
     if (!host_orch && rep) {
@@ -875,5 +890,3 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
   }
   return DYSEL_OK;
 }
-
-}  // extern "C"

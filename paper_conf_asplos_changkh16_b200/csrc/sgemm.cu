@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <cstring>
+#include <string>
 
 #include "internal.h"
 #include "sgemm_simt.cuh"
@@ -150,7 +151,9 @@ dysel_status dysel_sgemm(dysel_ctx *ctx, int M, int N, int K, float alpha, const
   const uint64_t U[3] = {(uint64_t)(N + 31) / 32, (uint64_t)(M + 31) / 32, 1};
   void *args[2] = {d_C, &g};
   const size_t sbytes[1] = {(size_t)M * ldc * sizeof(float)};
-  return dysel_launch(ctx, kSgemmSig, U, f, mode, args, 2, sbytes, stream, rep);
+  const std::string key = std::string(kSgemmSig) + "#" + std::to_string(M) + "x" + std::to_string(N) + "x" +
+                          std::to_string(K);
+  return launch_keyed(ctx, kSgemmSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep);
 }
 
 dysel_status dysel_sgemm_variant(dysel_ctx *ctx, int variant_id, int M, int N, int K, float alpha, const float *d_A,

@@ -41,6 +41,8 @@ FMT_DEFAULT = FMT_ELL | FMT_JDS | FMT_STREAM
 SPMV_DEFAULT_AUTO = -1
 SGEMM_S64, SGEMM_S128, SGEMM_T128x64, SGEMM_T128x128 = range(4)
 SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"]
+STENCIL_NAMES = ["base", "zmarch64", "tiled64x4_zmarch64"]
+STENCIL_BASE, STENCIL_ZMARCH, STENCIL_TILED = range(3)
 
 c_void_p, c_int, c_float, c_u32, c_u64, c_i64, c_size = (ctypes.c_void_p, ctypes.c_int, ctypes.c_float,
                                                         ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int64,
@@ -106,6 +108,9 @@ dysel_comm_unique_id = _sig("dysel_comm_unique_id", c_int, P)
 dysel_comm_init = _sig("dysel_comm_init", c_int, P, P, c_int, c_int)
 dysel_partition_rows = _sig("dysel_partition_rows", c_int, P, c_i64, c_int, P)
 dysel_spmv_sharded = _sig("dysel_spmv_sharded", c_int, P, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_stencil = _sig("dysel_stencil", c_int, P, c_int, c_int, c_int, c_float, c_float, P, P, c_float, c_u32, P,
+                     ctypes.POINTER(Report))
+dysel_stencil_variant = _sig("dysel_stencil_variant", c_int, P, c_int, c_int, c_int, c_int, c_float, c_float, P, P, P)
 dysel_spmv_power = _sig("dysel_spmv_power", c_int, P, P, P, P, c_int, c_int, c_float, c_u32, P, P,
                         ctypes.POINTER(Report))
 dysel_spmv_power_sharded = _sig("dysel_spmv_power_sharded", c_int, P, P, P, P, P, c_i64, c_int, c_int, c_float, c_u32,
@@ -354,6 +359,23 @@ class Context:
         t, c = c_u64(), ctypes.c_double()
         self._check(dysel_timer_calibrate(self.h, samples, spin_ns, ctypes.byref(t), ctypes.byref(c)))
         return t.value, c.value
+
+    # ------------------------------------------------------------ stencil
+    def stencil(self, inp, out, c0, c1, f=0.02, mode=DEFAULT_MODE, report=False, unit_map=False, stream=None):
+        """One 7-point Jacobi step out = c1 * (6-neighbour sum) - c0 * in (boundary copied); inp/out [nz, ny, nx]."""
+        nz, ny, nx = inp.shape
+        G = ((nx + 31) // 32 + 1) // 2 * ((ny + 3) // 4) * ((nz + 63) // 64)
+        rep, keep, uv = (_make_report(G if unit_map else 0) if report else (None, None, None))
+        self._check(dysel_stencil(self.h, nx, ny, nz, float(c0), float(c1), _ptr(inp), _ptr(out), float(f), int(mode),
+                                  _stream(stream), ctypes.byref(rep) if rep is not None else None))
+        if rep is None:
+            return None
+        return report_dict(rep, STENCIL_NAMES, bytes(uv) if uv is not None else None)
+
+    def stencil_variant(self, variant_id, inp, out, c0, c1, stream=None):
+        nz, ny, nx = inp.shape
+        self._check(dysel_stencil_variant(self.h, int(variant_id), nx, ny, nz, float(c0), float(c1), _ptr(inp),
+                                          _ptr(out), _stream(stream)))
 
     # -------------------------------------------------------- multi-GPU
     def comm_init(self, rank, world, uid: bytes):
