@@ -86,37 +86,43 @@ constexpr int kZq = 4;
 template <class Poll>
 __device__ __forceinline__ void zmarch_column(const StencilArgs &g, float *__restrict__ out, int x, int y, int z0,
                                               int z1, const Poll &poll) {
-  const size_t sy = (size_t)g.nx, sz = (size_t)g.nx * g.ny;
   const bool col = x < g.nx && y < g.ny;
   const bool inner_xy = col && x > 0 && y > 0 && x < g.nx - 1 && y < g.ny - 1;
-  const size_t base = col ? (size_t)y * sy + x : 0;
-  float zm = (col && z0 > 0) ? __ldg(g.in + (size_t)(z0 - 1) * sz + base) : 0.0f;
-  float c = col ? __ldg(g.in + (size_t)z0 * sz + base) : 0.0f;
+  const int sy = g.nx;
+  const size_t sz = (size_t)g.nx * g.ny;
+  // running pointers at plane z (64-bit adds only; neighbour offsets are 32-bit)
+  const size_t off0 = (size_t)z0 * sz + (col ? (size_t)y * sy + x : 0);
+  const float *pin = g.in + off0;
+  float *pout = out + off0;
+  float zm = (col && z0 > 0) ? __ldg(pin - sz) : 0.0f;
+  float c = col ? __ldg(pin) : 0.0f;
   for (int z = z0; z < z1; z += kZq) {
     if (((z - z0) & 15) == 15 - (kZq - 1) && poll()) return;
     float up[kZq], ym[kZq], yp[kZq], xm[kZq], xp[kZq];
 #pragma unroll
     for (int q = 0; q < kZq; ++q) {
       const int zz = z + q;
-      const size_t i = (size_t)zz * sz + base;
-      up[q] = (col && zz < z1 && zz + 1 < g.nz) ? __ldg(g.in + i + sz) : 0.0f;
+      const float *pq = pin + (size_t)q * sz;
+      up[q] = (col && zz < z1 && zz + 1 < g.nz) ? __ldg(pq + sz) : 0.0f;
       const bool in = inner_xy && zz < z1 && zz > 0 && zz < g.nz - 1;
-      ym[q] = in ? __ldg(g.in + i - sy) : 0.0f;
-      yp[q] = in ? __ldg(g.in + i + sy) : 0.0f;
-      xm[q] = in ? __ldg(g.in + i - 1) : 0.0f;
-      xp[q] = in ? __ldg(g.in + i + 1) : 0.0f;
+      ym[q] = in ? __ldg(pq - sy) : 0.0f;
+      yp[q] = in ? __ldg(pq + sy) : 0.0f;
+      xm[q] = in ? __ldg(pq - 1) : 0.0f;
+      xp[q] = in ? __ldg(pq + 1) : 0.0f;
     }
 #pragma unroll
     for (int q = 0; q < kZq; ++q) {
       const int zz = z + q;
       if (col && zz < z1) {
-        const size_t i = (size_t)zz * sz + base;
-        out[i] = (inner_xy && zz > 0 && zz < g.nz - 1) ? st_point(c, zm, up[q], ym[q], yp[q], xm[q], xp[q], g.c0, g.c1)
-                                                       : c;
+        pout[(size_t)q * sz] = (inner_xy && zz > 0 && zz < g.nz - 1)
+                                   ? st_point(c, zm, up[q], ym[q], yp[q], xm[q], xp[q], g.c0, g.c1)
+                                   : c;
         zm = c;
         c = up[q];
       }
     }
+    pin += kZq * sz;
+    pout += kZq * sz;
   }
 }
 
