@@ -76,7 +76,8 @@ def test_k_zero(ctx):
         assert np.allclose(C.cpu().numpy(), 2.0 * C0)
 
 
-@pytest.mark.parametrize("mode_name", ["fully_sync", "fully_host_sync", "fully_host_async", "hybrid_sync"])
+@pytest.mark.parametrize("mode_name", ["fully_sync", "fully_host_sync", "fully_host_async", "hybrid_sync",
+                                       "fully_async", "hybrid_async", "fully_sync_noabort"])
 def test_dysel_sgemm_composition(ctx, D, mode_name):
     M, K, N = 1024, 992, 1056
     A, B, C0 = sgemm_inputs(M, K, N, 992, 993, 994)
@@ -89,6 +90,7 @@ def test_dysel_sgemm_composition(ctx, D, mode_name):
     mode = D.FORCE_PROFILE | (D.HYBRID if "hybrid" in mode_name else D.FULLY)
     mode |= D.HOST_ORCH if "host" in mode_name else 0
     mode |= D.ASYNC if "async" in mode_name else 0
+    mode |= D.NO_ABORT if "noabort" in mode_name else 0
     C = dev(C0.copy())
     rep = ctx.sgemm(Ad, Bd, C, alpha=1.5, beta=-0.5, f=0.3, mode=mode, report=True, unit_map=True)
     Ch = C.cpu().numpy()
