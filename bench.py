@@ -263,6 +263,8 @@ def dysel_arm(args, world, rank, local_rank):
     if world == 1 and not args.no_secondary:
         ablation["sync_overhead_pct"] = round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=D.AUTO), 10, stream)
                                                / T_star - 1) * 100, 2)
+        ablation["solo_claim_kernel_overhead_pct"] = round(
+            (time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=mode | D.SOLO), 10, stream) / T_star - 1) * 100, 2)
         ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10, stream)
                                                       / T_star - 1) * 100, 2) for ff in (0.001, 0.005, 0.01, 0.02)}
         # iterative driver (SURVEY §8f f-3, P:L796-804 / §5.2): 20 power

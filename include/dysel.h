@@ -92,6 +92,11 @@ const char *dysel_status_str(dysel_status s);
 #define DYSEL_DEVICE_LAUNCH 4096u /* SpMV device path, round-1 scheme (ablation): eager kernel and remainder
                                      launched from the device (CDP2 fire-and-forget) instead of the
                                      host-launched PDL work kernel */
+#define DYSEL_SOLO 8192u        /* SpMV device path (reading A-38): launch only the default's claim kernel, which
+                                   also runs the winner's remainder slots (through a dispatch over the pool's
+                                   variants at the default's occupancy) — saves the non-winning claim grids
+                                   (~1.6% on D4 when the default wins), costs far more when it does not
+                                   (+44% with a CSR-V default on D4); ignored when the pool holds CSR-T */
 /* Default score: generic launcher = makespan (variants are separate concurrent
  * grids, Fig. 7b); SpMV dispatcher = mean per-unit busy time (%globaltimer end -
  * start of each profiled unit; all variants share one launch and occupancy). */

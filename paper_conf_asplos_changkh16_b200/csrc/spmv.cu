@@ -70,6 +70,7 @@ struct ProfParams {
   uint8_t *unit_variant; // optional debug map (variant id per unit)
   uint32_t pure;         // pure full-grid run of one variant (self-resetting counters, no init kernel)
   uint32_t k_claim;      // claim kernels: max slots per claim (~kClaimNnz nonzeros of work)
+  uint32_t solo;         // one claim kernel (the default's) also runs the winner's remainder (A-38)
 };
 
 __global__ void spmv_state_init_kernel(SpmvState *s, int K, int def) {
@@ -605,6 +606,7 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
                        : (uint64_t)atomicAdd(&st->c2, k);
     return __shfl_sync(FULL, raw, 0);
   };
+  int rem_vid = VID;   // variant of the remainder slots (the winner; solo: any pool variant)
   // a warp's first slot of a pure run / of the remainder is static: measured
   // on D3, claiming it instead cost 30-45% (ELL 15.9 vs 11.0 us)
   const bool stat = true;
@@ -613,7 +615,8 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     uint64_t sw = 0;
     if (lane == 0) sw = wait_published(&st->sw);
     sw = __shfl_sync(FULL, sw, 0);
-    if ((sw & 0xff) != pv) return false;
+    if ((sw & 0xff) != pv && !p.solo) return false;
+    rem_vid = p.vids[sw & 0xff];
     phase = 2;
     S = min((uint32_t)(sw >> 8), n_slots);
     dyn = n_slots - S > n_warps;
@@ -677,8 +680,11 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     }
     for (uint32_t q = t; q < e; ++q) {
       const uint32_t u = p.p_end + q / kSlots;
-      run_slot<VID>(A, u, (int)(q % kSlots), y + (size_t)u * kUnitRows);
-      if (lane == 0 && p.unit_variant && q % kSlots == 0) p.unit_variant[u] = (uint8_t)VID;
+      if (phase != 2 || rem_vid == VID)
+        run_slot<VID>(A, u, (int)(q % kSlots), y + (size_t)u * kUnitRows);
+      else
+        run_slot_dyn(rem_vid, A, u, (int)(q % kSlots), y + (size_t)u * kUnitRows);
+      if (lane == 0 && p.unit_variant && q % kSlots == 0) p.unit_variant[u] = (uint8_t)(phase == 2 ? rem_vid : VID);
     }
     t = e;
   }
@@ -1071,6 +1077,13 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.def = (uint32_t)pl->def;
   p.k_claim = claim_batch(pl);
   const bool cdp = (mode & DYSEL_DEVICE_LAUNCH) != 0;   // round-1 scheme: eager + remainder launched on the device
+  {   // reading A-38 (opt-in): one claim kernel (the default's) runs every
+      // remainder slot, whichever variant wins — not with CSR-T in the pool
+      // (its staging buffers live in its own kernel's shared memory)
+    bool tma = false;
+    for (int i = 0; i < pl->K; ++i) tma |= pl->vids[i] == DYSEL_SPMV_CSR_TMA;
+    p.solo = (!tma && (mode & DYSEL_SOLO)) ? 1u : 0u;
+  }
   p.tail = (cdp && !(mode & DYSEL_NO_TAIL)) ? 1u : 0u;
   p.abort = ((mode & DYSEL_NO_ABORT) || p.score_mode == 1) ? 0u : 1u;   // dominance needs busy or makespan
   for (int i = 0; i < pl->K; ++i) {
@@ -1114,11 +1127,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
     // launch lets them start while profiling runs (not after NO_TAIL or a
     // sequential profile: then they follow in stream order)
     const bool pdl = !(mode & DYSEL_NO_TAIL) && !sequential;
-#ifdef DYSEL_EXP_DEF_ONLY
-    for (int k = 0; k < 1; ++k) {
-#else
-    for (int k = 0; k < pl->K; ++k) {
-#endif
+    for (int k = 0; k < (p.solo ? 1 : pl->K); ++k) {
       const uint32_t i = (uint32_t)(k == 0 ? pl->def : (k <= pl->def ? k - 1 : k));
       const int v = pl->vids[i];
       const uint64_t g = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[v]) * ctx->n_sm,

@@ -586,6 +586,19 @@ __device__ __forceinline__ void run_unit(const SpmvDev &A, uint32_t j, float *ou
   run_slot<VID, Poll>(A, j, (int)(threadIdx.x >> 5), out, poll);
 }
 
+// One warp slot of any pool variant but CSR-T (which needs the staging
+// buffers): the solo claim kernel's remainder when the winner is not the
+// kernel's own variant (reading A-38).
+static __device__ __noinline__ void run_slot_dyn(int vid, const SpmvDev &A, uint32_t j, int w, float *out) {
+  switch (vid) {
+    case 0: run_slot<0>(A, j, w, out); break;
+    case 1: run_slot<1>(A, j, w, out); break;
+    case 2: run_slot<2>(A, j, w, out); break;
+    case 3: run_slot<3>(A, j, w, out); break;
+    default: run_slot<4>(A, j, w, out); break;
+  }
+}
+
 template <class Poll>
 __device__ __forceinline__ void run_unit_dyn(int vid, const SpmvDev &A, uint32_t j, float *out, const Poll &poll) {
   switch (vid) {

@@ -122,7 +122,7 @@ def test_identity_and_diagonal_exact(ctx):
 
 MODES = ["fully_sync", "fully_async", "hybrid_sync", "hybrid_async", "fully_sync_host", "fully_async_host",
          "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles", "hybrid_async_cdp", "fully_sync_cdp",
-         "hybrid_async_notail", "fully_sync_seq"]
+         "hybrid_async_notail", "fully_sync_seq", "hybrid_async_solo", "fully_sync_solo"]
 
 
 def mode_bits(D, m):
@@ -135,6 +135,7 @@ def mode_bits(D, m):
     b |= D.DEVICE_LAUNCH if "cdp" in m else 0
     b |= D.NO_TAIL if "notail" in m else 0
     b |= D.SEQUENTIAL if "seq" in m else 0
+    b |= D.SOLO if "solo" in m else 0
     return b
 
 
@@ -146,7 +147,9 @@ def test_dysel_composition(ctx, D, name, m):
     import torch
     A = MATS[name]()
     x = uniform_f32(7, A.n_cols)
-    plan = prepared(ctx, A, default=0)
+    # solo (A-38) needs a pool without CSR-T; its remainder then runs the winner
+    # through the default's (CSR-S's) claim kernel
+    plan = prepared(ctx, A, default=0, formats=D.FMT_DEFAULT if "solo" in m else None)
     xd = vec(x)
     full = {}
     for v in plan.variant_ids:
