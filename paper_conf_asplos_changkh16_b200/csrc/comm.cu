@@ -81,7 +81,8 @@ dysel_status dysel_comm_init(dysel_ctx *ctx, const void *uid, int rank, int worl
   comm_free(ctx);
   ctx->rank = rank;
   ctx->world = world;
-  if (world == 1) return DYSEL_OK;
+  // world == 1 still builds a (one-rank) communicator, so the collective
+  // calls below run — and are tested — on a single GPU
   ncclUniqueId id;
   memcpy(&id, uid, sizeof(id));
   ncclComm_t comm;
@@ -119,7 +120,7 @@ dysel_status dysel_partition_rows(const int32_t *rp, int64_t n, int world, int64
 
 static dysel_status allgatherv(dysel_ctx *ctx, float *buf, const int64_t *offs, const int64_t *counts,
                                cudaStream_t st) {
-  if (ctx->world == 1 || !ctx->nccl_comm) return DYSEL_OK;
+  if (!ctx->nccl_comm) return DYSEL_OK;
   ncclComm_t comm = (ncclComm_t)ctx->nccl_comm;
   DYSEL_NCCL_TRY(ctx, nccl().GroupStart());
   for (int r = 0; r < ctx->world; ++r)
@@ -131,7 +132,7 @@ static dysel_status allgatherv(dysel_ctx *ctx, float *buf, const int64_t *offs, 
 
 dysel_status dysel_comm_broadcast(dysel_ctx *ctx, float *d_buf, size_t n, int root, void *stream) {
   if (!ctx || (n > 0 && !d_buf) || root < 0 || root >= ctx->world) return DYSEL_ERR_INVALID;
-  if (ctx->world == 1 || !ctx->nccl_comm || n == 0) return DYSEL_OK;
+  if (!ctx->nccl_comm || n == 0) return DYSEL_OK;
   DYSEL_NCCL_TRY(ctx, nccl().Broadcast(d_buf, d_buf, n, ncclFloat, root, (ncclComm_t)ctx->nccl_comm,
                                     (cudaStream_t)stream));
   return DYSEL_OK;

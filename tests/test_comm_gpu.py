@@ -1,0 +1,71 @@
+"""The NCCL path of the multi-GPU calls on one GPU: a one-rank
+communicator runs the real grouped-broadcast allgatherv / broadcast code;
+results checked against the fp64 oracles.  (N > 1 needs more GPUs than
+gpurun provides; the partition / assembly host logic is covered by the gloo
+world-2 tests.)"""
+import numpy as np
+import pytest
+
+from gpu_helpers import spmv_err, to_dev, vec
+from oracle import iterative, sgemm as osg
+from workloads import d4_powerlaw, laplacian_2d, sgemm_inputs, uniform_f32
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def cctx(gpu):
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+    c = D.Context(0)
+    c.comm_init(0, 1, D.comm_unique_id())
+    yield c
+    c.close()
+
+
+def test_spmv_sharded_one_rank(cctx):
+    import torch
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+    A = d4_powerlaw(n=300_000, lmax=4096)
+    bounds = D.partition_rows(A.row_ptr, 1)
+    assert list(bounds) == [0, A.n_rows]
+    rp, col, val = to_dev(A)
+    plan = cctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO)
+    x = uniform_f32(21, A.n_cols)
+    xd = vec(x)
+    cctx.comm_broadcast(xd, 0)
+    y = torch.full((A.n_rows,), float("nan"), device="cuda")
+    cctx.spmv_sharded(plan, list(bounds), xd, y, f=0.01, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE)
+    torch.cuda.synchronize()
+    assert spmv_err(A, x, y) <= 1e-5
+    plan.destroy()
+
+
+def test_power_sharded_one_rank(cctx):
+    import torch
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+    L = laplacian_2d(80)
+    x0 = uniform_f32(3, L.n_cols, 0.0, 1.0)
+    rp, col, val = to_dev(L)
+    plan = cctx.spmv_prepare(rp, col, val, L.n_cols, default=D.SPMV_CSR_VECTOR)
+    x = vec(x0)
+    y = torch.empty_like(x)
+    norms = torch.zeros(12, dtype=torch.float64, device="cuda")
+    cctx.spmv_power_sharded(plan, [0, L.n_rows], x, y, 12, profile_every=4, f=0.5,
+                            mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE, norms=norms)
+    torch.cuda.synchronize()
+    _, _, no = iterative.power_iteration(L.row_ptr, L.col, L.val, x0, 12)
+    assert np.max(np.abs(norms.cpu().numpy() - no) / no) <= 1e-5
+    plan.destroy()
+
+
+def test_sgemm_sharded_one_rank(cctx):
+    import torch
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+    M, K, N = 1024, 992, 1056
+    A, B, C0 = sgemm_inputs(M, K, N, 992, 993, 994)
+    C = torch.from_numpy(C0.copy()).cuda()
+    cctx.sgemm_sharded(torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda(), C, 1.5, -0.5, f=0.06,
+                       mode=D.FULLY | D.FORCE_PROFILE)
+    torch.cuda.synchronize()
+    ref, den = osg.sgemm(A, B, C0, 1.5, -0.5), osg.sgemm_abs(A, B, C0, 1.5, -0.5)
+    assert float((np.abs(C.cpu().numpy() - ref) / den).max()) <= osg.SGEMM_TOL
