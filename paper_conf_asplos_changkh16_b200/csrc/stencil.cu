@@ -78,9 +78,10 @@ __global__ void __launch_bounds__(128) stencil_base_kernel(StencilArgs g, float 
 // z-march in chunks of kZq planes: all loads of a chunk (the next kZq centre
 // values and the 4 in-plane neighbours of each plane) are issued before its
 // first point is computed, so a thread waits once per chunk, not once per
-// plane (64 dependent plane steps per thread otherwise bound the kernel by
-// latency: 56 us -> see DESIGN.md).
-constexpr int kZq = 4;
+// plane.  kZq = 2 fits the 32-register budget of 16 CTAs/SM without spills
+// (512 x 512 x 64: 43 us at 16/SM vs 50 us with kZq = 4 at 10/SM and 60 us
+// with kZq = 4 squeezed to 32 registers).
+constexpr int kZq = 2;
 // poll(): called by all threads every 16 planes (A-32 dominance; productive
 // copies only report, sandbox copies stop when it returns true)
 template <class Poll>
@@ -126,13 +127,19 @@ __device__ __forceinline__ void zmarch_column(const StencilArgs &g, float *__res
   }
 }
 
-__global__ void __launch_bounds__(128) stencil_zmarch_kernel(StencilArgs g, float *__restrict__ out, dysel_slice s) {
+// Untimed launches (full grid, gated remainder) use a lean instantiation with
+// no timing / dominance code and a 16-CTA/SM register cap, so a 2,048-CTA grid
+// (512 x 512 x 64) is resident in one wave; timed (profiling) copies keep the
+// timing code.
+template <bool TIMED>
+__global__ void __launch_bounds__(128, TIMED ? 1 : 16)
+    stencil_zmarch_kernel(StencilArgs g, float *__restrict__ out, dysel_slice s) {
   __shared__ dysel_prof_smem psm;
   if (!dysel_gate_open(s)) return;
   const uint32_t wa[3] = {1, 1, 64};
-  const bool persistent = s.timer == nullptr && s.gate != nullptr;   // gated remainder: one wave walks the tiles
+  const bool persistent = !TIMED && s.gate != nullptr;   // gated remainder: one wave walks the tiles
   const uint64_t n_cta = persistent ? dysel_slice_ctas(s, wa) : (uint64_t)blockIdx.x + 1;
-  dysel_prof_begin(s, psm);
+  if constexpr (TIMED) dysel_prof_begin(s, psm);
   uint32_t units = 0;
   for (uint64_t cta = blockIdx.x; cta < n_cta; cta += gridDim.x) {
   uint64_t u[3];
@@ -140,12 +147,15 @@ __global__ void __launch_bounds__(128) stencil_zmarch_kernel(StencilArgs g, floa
   if (ok) {
     const int x = (int)u[0] * 32 + (threadIdx.x & 31), y = (int)u[1] * 4 + (threadIdx.x >> 5);
     const int z0 = (int)u[2], z1 = min(z0 + 64, g.nz);
-    zmarch_column(g, out, x, y, z0, z1,
-                  [&]() { return dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_SANDBOX; });
+    if constexpr (TIMED)
+      zmarch_column(g, out, x, y, z0, z1,
+                    [&]() { return dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_SANDBOX; });
+    else
+      zmarch_column(g, out, x, y, z0, z1, []() { return false; });
     units = (uint32_t)(z1 - z0);
   }
   }
-  dysel_prof_end(s, psm, units);
+  if constexpr (TIMED) dysel_prof_end(s, psm, units);
 }
 
 // ------------------------------------------------------------------- V2
@@ -241,7 +251,10 @@ static dysel_status stencil_variant_fn(const dysel_slice *s, void *const *args, 
   if constexpr (VID == DYSEL_STENCIL_BASE)
     stencil_base_kernel<<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
   else if constexpr (VID == DYSEL_STENCIL_ZMARCH)
-    stencil_zmarch_kernel<<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
+    if (s->timer)
+      stencil_zmarch_kernel<true><<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
+    else
+      stencil_zmarch_kernel<false><<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
   else
     stencil_tiled_kernel<<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
@@ -254,7 +267,7 @@ dysel_status stencil_register(dysel_ctx *ctx) {
   static const int sb[1] = {0};
   int o[3] = {0, 0, 0};
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[0], stencil_base_kernel, 128, 0);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[1], stencil_zmarch_kernel, 128, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[1], stencil_zmarch_kernel<false>, 128, 0);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], stencil_tiled_kernel, 128, 0);
   cudaGetLastError();
   const uint64_t n = (uint64_t)ctx->n_sm;
