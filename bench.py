@@ -140,7 +140,7 @@ def reference_arm(args, world, rank):
     line = {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(T * 1e3, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": config(A, world),
+            "data": "synthetic", "config": config(A, world, args.f),
             "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
                              "sample": f"full D4 matrix ({A.nnz} nnz), one fp64 SpMV per step"},
             "e2e": {"value": round(v, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -150,10 +150,10 @@ def reference_arm(args, world, rank):
 METRIC = "DySel SpMV GB/s (power-law 1e7 rows, profiling on every call) + overhead % vs best-variant oracle"
 
 
-def config(A, world):
+def config(A, world, f):
     return {"workload": "D4 power-law SpMV: 10^7 rows, p(L)~L^-1.761 on [1,16384], uniform cols, fp32 CSR",
             "n_rows": int(A.n_rows), "nnz": int(A.nnz), "parallelism": f"row-shard{world}",
-            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": "AUTO|ASYNC (hybrid), f=0.002",
+            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": f"AUTO|ASYNC (hybrid), f={f}",
             "default_variant": "DYSEL_SPMV_DEFAULT_AUTO (A-30)"}
 
 
@@ -374,7 +374,7 @@ def dysel_arm(args, world, rank, local_rank):
             "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(T_step * 1e3, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": config(A, world),
+            "config": config(A, world, args.f),
             "default_variant": default_name,
             "overhead_pct_vs_best_variant": round((T_step - T_star) / T_star * 100, 3) if world == 1 else None,
             "best_variant_oracle": {"variant": best_name, "ms": round(T_star * 1e3, 4),
