@@ -132,7 +132,7 @@ void resolve_pending(dysel_ctx *ctx, const char *block_sig);
 // dysel_launch with a selection-cache key distinct from the registry sig
 dysel_status launch_keyed(dysel_ctx *ctx, const char *sig, const char *key, const uint64_t ndrange_units[3], float f,
                           uint32_t mode, void *const *args, int n_args, const size_t *sandbox_bytes, void *stream,
-                          dysel_report *rep);
+                          dysel_report *rep, int def_override = -1);
 // spmv.cu
 dysel_status spmv_ctx_init(dysel_ctx *ctx);
 void spmv_ctx_free(dysel_ctx *ctx);

@@ -545,7 +545,7 @@ dysel_status dysel_reset_selection(dysel_ctx *ctx, const char *key) {
 dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrange_units[3], float f, uint32_t mode,
                           void *const *args, int n_args, const size_t *sandbox_bytes, void *stream_v,
                           dysel_report *rep) {
-  return dysel::launch_keyed(ctx, sig, sig, ndrange_units, f, mode, args, n_args, sandbox_bytes, stream_v, rep);
+  return dysel::launch_keyed(ctx, sig, sig, ndrange_units, f, mode, args, n_args, sandbox_bytes, stream_v, rep, -1);
 }
 
 }  // extern "C"
@@ -555,7 +555,7 @@ dysel_status dysel_launch(dysel_ctx *ctx, const char *sig, const uint64_t ndrang
 // stencil pools (a selection made for one shape is not reused for another).
 dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *key, const uint64_t ndrange_units[3],
                                  float f, uint32_t mode, void *const *args, int n_args, const size_t *sandbox_bytes,
-                                 void *stream_v, dysel_report *rep) {
+                                 void *stream_v, dysel_report *rep, int def_override) {
   const uint64_t t_host0 = now_ns();
   if (!ctx || !sig || !ndrange_units || n_args < 0 || (n_args > 0 && !args)) {
     set_error(ctx, "dysel_launch: invalid arguments");
@@ -568,6 +568,9 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
   }
   const Registered &R = it->second;
   const int K = (int)R.v.size();
+  // initial ("default") version: the registered one, or a per-call choice of
+  // a built-in pool (reading A-39)
+  const int def = (def_override >= 0 && def_override < K) ? def_override : R.def;
   uint32_t wa[DYSEL_MAX_VARIANTS][3], vflags[DYSEL_MAX_VARIANTS];
   for (int v = 0; v < K; ++v) {
     for (int d = 0; d < 3; ++d) wa[v][d] = R.v[v].wa[d];
@@ -580,13 +583,13 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
         return DYSEL_ERR_INVALID;
       }
   Plan P;
-  DYSEL_TRY(make_plan(ctx, ndrange_units, wa, K, f, ctx->n_sm, R.def, mode, vflags, &P));
+  DYSEL_TRY(make_plan(ctx, ndrange_units, wa, K, f, ctx->n_sm, def, mode, vflags, &P));
   resolve_pending(ctx, nullptr);
-  if (P.active && !(mode & DYSEL_FORCE_PROFILE) && R.v[R.def].ctas_per_wave > 0) {
+  if (P.active && !(mode & DYSEL_FORCE_PROFILE) && R.v[def].ctas_per_wave > 0) {
     // reading A-3b: the default variant's whole grid runs in one wave
     uint64_t def_ctas = 1;
-    for (int d = 0; d < 3; ++d) def_ctas *= (P.U[d] + wa[R.def][d] - 1) / wa[R.def][d];
-    if (def_ctas <= R.v[R.def].ctas_per_wave) {
+    for (int d = 0; d < 3; ++d) def_ctas *= (P.U[d] + wa[def][d] - 1) / wa[def][d];
+    if (def_ctas <= R.v[def].ctas_per_wave) {
       P.active = false;
       P.c = 0;
     }
@@ -594,12 +597,12 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
   cudaStream_t st = (cudaStream_t)stream_v;
   if (rep) rep->n_slices = 0;
   if (P.Gn == 0) {
-    fill_report_common(rep, P, P.mode, 0, R.def);
+    fill_report_common(rep, P, P.mode, 0, def);
     return DYSEL_OK;
   }
   std::vector<void *> base_args(args, args + n_args);
   if (!P.active) {   // activation flag off / small workload: one plain batch copy
-    int v = R.def;
+    int v = def;
     resolve_pending(ctx, key);
     auto c = ctx->sel_cache.find(key);
     if (c != ctx->sel_cache.end() && c->second < K) v = c->second;
@@ -633,7 +636,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
   if (P.mode == DYSEL_HYBRID || P.mode == DYSEL_SWAP) {
     int slot = 0;
     for (int v = 0; v < K; ++v) {
-      if (P.mode == DYSEL_HYBRID && v == R.def) continue;       // ≤ K-1 sandboxes
+      if (P.mode == DYSEL_HYBRID && v == def) continue;       // ≤ K-1 sandboxes
       for (size_t k = 0; k < R.sandbox_args[v].size(); ++k) {
         if ((size_t)slot >= sizeof(ctx->sandbox) / sizeof(ctx->sandbox[0])) {
           set_error(ctx, "too many sandbox buffers");
@@ -651,7 +654,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     }
   }
   // ---- profiling copies, concurrently on forked streams
-  init_prof_kernel<<<1, 32, 0, st>>>(ctx->d_prof, K, R.def);
+  init_prof_kernel<<<1, 32, 0, st>>>(ctx->d_prof, K, def);
   DYSEL_TRY(check_launch(ctx, "init_prof_kernel"));
   DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_start, st));
   fill_report_common(rep, P, P.mode | (async ? DYSEL_ASYNC : 0), 1, -1);
@@ -668,7 +671,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
       }
       s.role = DYSEL_ROLE_PRODUCTIVE;
     } else if (P.mode == DYSEL_HYBRID) {
-      s.role = v == R.def ? DYSEL_ROLE_PRODUCTIVE : DYSEL_ROLE_SANDBOX;
+      s.role = v == def ? DYSEL_ROLE_PRODUCTIVE : DYSEL_ROLE_SANDBOX;
     } else {
       s.role = DYSEL_ROLE_PRIVATE;
     }
@@ -696,22 +699,22 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
   const uint64_t rem_end = P.Gn;
   int selected = -1;
   uint64_t eager_units = 0;
-  if (!host_orch && async && rem_begin < rem_end && R.v[R.def].ctas_per_wave > 0) {
+  if (!host_orch && async && rem_begin < rem_end && R.v[def].ctas_per_wave > 0) {
     // ---- eager wave (reading A-33): the default variant fills the
     // execution slots the profiling copies leave free, on `st`, while they run
     uint64_t prof_slots = 0;   // profiling CTAs in units of the default's slots
     for (int v = 0; v < K; ++v)
       if (R.v[v].ctas_per_wave > 0)
-        prof_slots += (P.c * P.h[v] * R.v[R.def].ctas_per_wave + R.v[v].ctas_per_wave - 1) / R.v[v].ctas_per_wave;
-    const uint64_t free_slots = R.v[R.def].ctas_per_wave > prof_slots ? R.v[R.def].ctas_per_wave - prof_slots : 0;
-    const uint64_t E = std::min<uint64_t>(free_slots / P.h[R.def], rem_end - rem_begin);
+        prof_slots += (P.c * P.h[v] * R.v[def].ctas_per_wave + R.v[v].ctas_per_wave - 1) / R.v[v].ctas_per_wave;
+    const uint64_t free_slots = R.v[def].ctas_per_wave > prof_slots ? R.v[def].ctas_per_wave - prof_slots : 0;
+    const uint64_t E = std::min<uint64_t>(free_slots / P.h[def], rem_end - rem_begin);
     if (E > 0) {
       dysel_slice s = base_slice(P);
-      s.variant = R.def;
+      s.variant = def;
       s.role = DYSEL_ROLE_EAGER;
       s.granule_begin = rem_begin;
       s.granule_count = E;
-      DYSEL_TRY(R.v[R.def].fn(&s, base_args.data(), st, R.v[R.def].user));
+      DYSEL_TRY(R.v[def].fn(&s, base_args.data(), st, R.v[def].user));
       DYSEL_TRY(check_launch(ctx, "variant eager wave"));
       add_slice_rec(rep, s);
       mark_units(rep, s);
@@ -785,7 +788,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     bool done[DYSEL_MAX_VARIANTS] = {};
     int ndone = 0;
     uint64_t best_pack = ~0ull;
-    int best_v = R.def;
+    int best_v = def;
     cudaEvent_t chunk_ev = nullptr;
     cudaEventCreateWithFlags(&chunk_ev, cudaEventDisableTiming);
     bool chunk_inflight = false;

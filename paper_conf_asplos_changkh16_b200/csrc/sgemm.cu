@@ -63,6 +63,7 @@ static dysel_status launch_tc(const SgemmArgs &g, float *C, const dysel_slice &s
 }
 
 static uint64_t g_simt_wave[2] = {0, 0};   // resident CTAs (occupancy x #SM) of the two SIMT kernels
+static uint64_t g_tc128_wave = 0;          // ... of the 128x128 tcgen05 kernel
 
 template <int VID>
 static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
@@ -114,6 +115,7 @@ dysel_status sgemm_register(dysel_ctx *ctx) {
   const uint64_t n = (uint64_t)ctx->n_sm;
   g_simt_wave[0] = (uint64_t)o[0] * n;
   g_simt_wave[1] = (uint64_t)o[1] * n;
+  g_tc128_wave = (uint64_t)o[3] * n;
   dysel_variant v[DYSEL_SGEMM_NVARIANTS] = {
       {"simt64x64", sgemm_variant_fn<0>, {2, 2, 1}, sb, 1, 0, nullptr, (uint64_t)o[0] * n},
       {"simt128x128", sgemm_variant_fn<1>, {4, 4, 1}, sb, 1, 0, nullptr, (uint64_t)o[1] * n},
@@ -153,7 +155,12 @@ dysel_status dysel_sgemm(dysel_ctx *ctx, int M, int N, int K, float alpha, const
   const size_t sbytes[1] = {(size_t)M * ldc * sizeof(float)};
   const std::string key = std::string(kSgemmSig) + "#" + std::to_string(M) + "x" + std::to_string(N) + "x" +
                           std::to_string(K);
-  return launch_keyed(ctx, kSgemmSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep);
+  // reading A-39: the initial version is the 128x128 tcgen05 tiling when its
+  // grid spans at least two waves (large GEMMs: fewest passes over A and B),
+  // else the 128x64 tiling (more CTAs: fills the SMs of a small GEMM)
+  const uint64_t t128 = (uint64_t)((M + 127) / 128) * (uint64_t)((N + 127) / 128);
+  const int def = (g_tc128_wave > 0 && t128 >= 2 * g_tc128_wave) ? DYSEL_SGEMM_T128x128 : DYSEL_SGEMM_T128x64;
+  return launch_keyed(ctx, kSgemmSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep, def);
 }
 
 dysel_status dysel_sgemm_variant(dysel_ctx *ctx, int variant_id, int M, int N, int K, float alpha, const float *d_A,
