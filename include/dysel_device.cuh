@@ -138,10 +138,13 @@ __device__ __forceinline__ void dysel_prof_begin(const dysel_slice &s, dysel_pro
  * only be larger — and the first CTA to see it decides the variant (maximal
  * score).  Returns true when the variant is dominated: a SANDBOX CTA may then
  * stop (its output is discarded), a productive CTA must finish its tile. */
-__device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof_smem &sm) {
+/* Single-thread form (no barrier), for warp-specialised kernels: the calling
+ * thread (the one that ran dysel_prof_begin's thread-0 part, i.e. tid 0)
+ * reports and checks; it returns the dominated flag but nothing stops the
+ * CTA — it only lets the selection be published without waiting for it. */
+__device__ __forceinline__ bool dysel_prof_poll_thread(const dysel_slice &s, dysel_prof_smem &sm) {
   if (s.timer == nullptr || s.lb == nullptr) return false;
-  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
-  if (tid == 0 && !sm.dominated) {
+  if (!sm.dominated) {
     const unsigned long long now = dysel_clock64();
     const unsigned long long tot = atomicAdd((unsigned long long *)s.lb, now - sm.c_last) + (now - sm.c_last);
     sm.c_last = now;
@@ -161,6 +164,13 @@ __device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof
     }
     sm.dominated = d;
   }
+  return sm.dominated != 0;
+}
+
+__device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof_smem &sm) {
+  if (s.timer == nullptr || s.lb == nullptr) return false;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if (tid == 0) dysel_prof_poll_thread(s, sm);
   __syncthreads();
   return sm.dominated != 0;
 }

@@ -97,6 +97,7 @@ struct dysel_ctx {
   cudaEvent_t ev_fork2 = nullptr;
   cudaStream_t rem[DYSEL_MAX_VARIANTS] = {};        // gated remainder copies (device path)
   cudaStream_t wsel = nullptr;                      // wait-for-selection kernel (device path)
+  cudaStream_t rem_hi = nullptr;                    // the default variant's gated remainder (high priority)
   cudaEvent_t ev_join2[DYSEL_MAX_VARIANTS] = {};
   dysel::DevProf *d_prof = nullptr;
   dysel::DevProf *h_prof = nullptr;  // pinned

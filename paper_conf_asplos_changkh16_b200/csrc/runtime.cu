@@ -399,6 +399,8 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
   if (cudaStreamCreateWithFlags(&ctx->query, cudaStreamNonBlocking) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (cudaStreamCreateWithPriority(&ctx->wsel, cudaStreamNonBlocking, prio_hi) != cudaSuccess)
     return fail(DYSEL_ERR_CUDA);
+  if (cudaStreamCreateWithPriority(&ctx->rem_hi, cudaStreamNonBlocking, prio_hi) != cudaSuccess)
+    return fail(DYSEL_ERR_CUDA);
   if (cudaEventCreateWithFlags(&ctx->ev_start, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (cudaEventCreateWithFlags(&ctx->ev_fork2, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
   if (cudaMalloc(&ctx->d_prof, sizeof(DevProf)) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
@@ -432,6 +434,7 @@ void dysel_destroy(dysel_ctx *ctx) {
   }
   if (ctx->query) cudaStreamDestroy(ctx->query);
   if (ctx->wsel) cudaStreamDestroy(ctx->wsel);
+  if (ctx->rem_hi) cudaStreamDestroy(ctx->rem_hi);
   if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
   if (ctx->ev_fork2) cudaEventDestroy(ctx->ev_fork2);
   if (ctx->d_prof) cudaFree(ctx->d_prof);
@@ -753,17 +756,22 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
       DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, st));
     }
     if (rem_begin < rem_end) {
-      for (int v = 0; v < K; ++v) {
+      // the default's gated copy goes first and on a high-priority stream: when
+      // it wins (the usual case with a good initial version), the block
+      // scheduler dispatches its CTAs ahead of the exiting CTAs of the losers
+      for (int k = 0; k < K; ++k) {
+        const int v = k == 0 ? def : (k <= def ? k - 1 : k);
+        cudaStream_t rs = k == 0 ? ctx->rem_hi : ctx->rem[v];
         dysel_slice s = base_slice(P);
         s.variant = v;
         s.role = DYSEL_ROLE_BATCH;
         s.granule_begin = rem_begin;
         s.granule_count = rem_end - rem_begin;
         s.gate = &ctx->d_prof->sel;
-        DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->rem[v], ctx->ev_fork2, 0));
-        DYSEL_TRY(R.v[v].fn(&s, base_args.data(), ctx->rem[v], R.v[v].user));
+        DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(rs, ctx->ev_fork2, 0));
+        DYSEL_TRY(R.v[v].fn(&s, base_args.data(), rs, R.v[v].user));
         DYSEL_TRY(check_launch(ctx, "variant gated batch"));
-        DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join2[v], ctx->rem[v]));
+        DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join2[v], rs));
       }
       for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join2[v], 0));
     }
