@@ -215,6 +215,16 @@ def dysel_arm(args, world, rank, local_rank):
         T_v[D.SPMV_NAMES[v]] = time_b2b(lambda: ctx.spmv_variant(plan, v, xd, yl), args.oracle_reps, stream)
     best_name = min(T_v, key=T_v.get)
     T_star = T_v[best_name]
+    # ---- practical floor: the matrix's CSR traffic with no row structure
+    # (dysel_spmv_gather_probe; flavour 0 = gather at col, 1 = sequential x)
+    probe = {}
+    try:
+        for fl, nm in ((0, "gather"), (1, "stream")):
+            for _ in range(2):
+                ctx.spmv_gather_probe(plan, fl, xd, yl)
+            probe[nm] = time_b2b(lambda: ctx.spmv_gather_probe(plan, fl, xd, yl), args.oracle_reps, stream)
+    except Exception as e:   # unaligned col / val: no probe
+        probe = {"error": str(e)}
     # ---- warmup, then K timed steps (barrier + sync on both sides)
     for _ in range(args.warmup):
         step()
@@ -402,7 +412,16 @@ def dysel_arm(args, world, rank, local_rank):
                          "kernel": f"dysel::spmv_claim_kernel<{sel_name}> (pure full grid, event-timed back to back)",
                          "peak_source": src,
                          "note": "D4 gathers x at uniform-random columns: bound in practice by the L1TEX/L2 "
-                                 "random-sector rate (DESIGN.md §Roofline), not HBM"},
+                                 "random-sector rate (DESIGN.md §Roofline), not HBM",
+                         "floor": ({"gather_probe_ms": round(probe["gather"] * 1e3, 4),
+                                    "gather_probe_gbs": round(kern_bytes / probe["gather"] / 1e9, 2),
+                                    "stream_probe_ms": round(probe["stream"] * 1e3, 4),
+                                    "stream_probe_gbs": round(kern_bytes / probe["stream"] / 1e9, 2),
+                                    "frac_of_gather_floor": round(probe["gather"] / T_v[sel_name], 4),
+                                    "what": "dysel_spmv_gather_probe: the same col/val stream + x[col] gathers + "
+                                            "row_ptr/y traffic with no row structure (gather), and with x read "
+                                            "sequentially instead (stream); frac = probe time / kernel time"}
+                                   if "gather" in probe else probe)},
             "gpu_launches": int(launches), "clocks": clk.summary(),
             "cpu_baseline": cpu, "secondary": secondary,
         }

@@ -306,6 +306,8 @@ typedef struct {
   uint64_t prep_ns;              /* device time of format preparation (a-1) */
   uint64_t ell_bytes, jds_bytes; /* extra device memory held by the plan */
   int32_t default_variant;       /* DYSEL_SPMV_* id of the initial version (resolved when AUTO) */
+  int32_t n_heavy;               /* units the claim kernels run first: >= max(8192, 4 x mean) nonzeros,
+                                    by nonzeros descending (longest-processing-time order, A-40) */
 } dysel_spmv_plan_info;
 
 /* Build the variant pool for one CSR matrix: CSR -> ELL and CSR -> block JDS
@@ -348,6 +350,18 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x,
  * and what DYSEL_NO_PROFILE runs. */
 dysel_status dysel_spmv_variant(dysel_ctx *ctx, dysel_spmv_plan *plan, int variant_id, const float *d_x,
                                 float *d_y, void *stream);
+
+/* Measurement only (not part of the method): one launch that generates the
+ * memory traffic every CSR SpMV of the plan's matrix must generate -- col / val
+ * streamed once (128-bit), x gathered at col (flavour 0) or read sequentially
+ * (flavour 1), one fma per nonzero, row_ptr read and d_out [n_rows] written
+ * once -- with no row structure.  Its duration is the practical floor the
+ * variant kernels are judged against (SURVEY §8d roofline);
+ * d_out receives meaningless values.  Grid = #SM x occupancy, stream-ordered
+ * on `stream`.  DYSEL_ERR_UNSUPPORTED if col / val are not 16-byte aligned;
+ * DYSEL_ERR_INVALID for a bad flavour or NULL pointers. */
+dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *plan, int flavour, const float *d_x,
+                                     float *d_out, void *stream);
 
 /* ------------------------------------------------------------------ SGEMM
  * C = alpha * A B + beta * C, fp32, row-major, no transposes (Parboil sgemm,

@@ -71,6 +71,12 @@ struct ProfParams {
   uint32_t pure;         // pure full-grid run of one variant (self-resetting counters, no init kernel)
   uint32_t k_claim;      // claim kernels: max slots per claim (~kClaimNnz nonzeros of work)
   uint32_t solo;         // one claim kernel (the default's) also runs the winner's remainder (A-38)
+  // claim kernels, heavy-first order (A-40): tickets [0, 8 n_heavy) are the
+  // slots of heavy[] (skipped if profiled: unit < p_end), the rest the
+  // remainder units in order (skipped if heavy)
+  uint32_t n_heavy;
+  const int32_t *heavy;
+  const uint32_t *heavy_bits;
 };
 
 __global__ void spmv_state_init_kernel(SpmvState *s, int K, int def) {
@@ -488,7 +494,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
   {   // claim kernels: close the eager ticket range; the default keeps whole
       // units only, so the switch point S is rounded up to a unit boundary
     const uint64_t old = atomicOr((unsigned long long *)&st->c1, 1ull << 32);
-    const uint64_t n_slots = (uint64_t)(p.n_units - p.p_end) * kSlots;
+    const uint64_t n_slots = (uint64_t)(p.n_units - p.p_end + p.n_heavy) * kSlots;   // claim tickets (A-40)
     const uint64_t S = min(((uint64_t)(uint32_t)old + kSlots - 1) / kSlots * kSlots, n_slots);
     atomicExch((unsigned long long *)&st->sw, (S << 8) | win);
   }
@@ -578,7 +584,8 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const uint32_t FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
-  const uint32_t n_slots = (p.n_units - p.p_end) * kSlots;
+  const uint32_t n_hs = p.n_heavy * kSlots;
+  const uint32_t n_slots = (p.n_units - p.p_end) * kSlots + n_hs;   // tickets
   const uint32_t n_warps = gridDim.x * (kUnitRows / 32);
   const uint32_t gid = blockIdx.x * (kUnitRows / 32) + (threadIdx.x >> 5);
   // Claims.  A warp's first slot of a pure run or of the remainder is static
@@ -679,7 +686,14 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
       done += e - t;
     }
     for (uint32_t q = t; q < e; ++q) {
-      const uint32_t u = p.p_end + q / kSlots;
+      uint32_t u;
+      if (q < n_hs) {   // heavy-first (A-40); a profiled heavy unit is done
+        u = (uint32_t)__ldg(p.heavy + q / kSlots);
+        if (u < p.p_end) continue;
+      } else {
+        u = p.p_end + (q - n_hs) / kSlots;
+        if (n_hs && ((__ldg(p.heavy_bits + (u >> 5)) >> (u & 31)) & 1u)) continue;
+      }
       if (phase != 2 || rem_vid == VID)
         run_slot<VID>(A, u, (int)(q % kSlots), y + (size_t)u * kUnitRows);
       else
@@ -860,6 +874,12 @@ typedef dysel_status (*ClaimLauncher)(const SpmvDev &, float *, SpmvState *, con
 static const ClaimLauncher kClaim[DYSEL_SPMV_NVARIANTS] = {launch_claim<0>, launch_claim<1>, launch_claim<2>,
                                                            launch_claim<3>, launch_claim<4>, launch_claim<5>};
 
+static void set_heavy(ProfParams &p, const dysel_spmv_plan *pl) {
+  p.n_heavy = pl->n_heavy;
+  p.heavy = pl->heavy;
+  p.heavy_bits = pl->heavy_bits;
+}
+
 // Slots per claim: about kClaimNnz nonzeros of work (at least 1, at most a unit).
 constexpr int64_t kClaimNnz = 1024;
 static uint32_t claim_batch(const dysel_spmv_plan *pl) {
@@ -881,6 +901,7 @@ static dysel_status launch_variant_full(dysel_ctx *ctx, dysel_spmv_plan *pl, int
   p.n_units = pl->n_units;
   p.pure = 1;
   p.k_claim = claim_batch(pl);
+  set_heavy(p, pl);
   const uint64_t grid = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[vid]) * ctx->n_sm, pl->n_units);
   SpmvDev A = pl->dev;
   A.x = x;
@@ -896,11 +917,86 @@ typedef void (*ProfLauncher)(const SpmvDev &, float *, SpmvState *, const ProfPa
 static const ProfLauncher kProf[DYSEL_SPMV_NVARIANTS] = {launch_prof<0>, launch_prof<1>, launch_prof<2>, launch_prof<3>,
                                                          launch_prof<4>, launch_prof<5>};
 
+// ------------------------------------------------------------ gather probe
+// Measurement only (dysel_spmv_gather_probe): the memory traffic
+// every CSR SpMV of this matrix must generate and nothing else -- col / val
+// streamed with 128-bit evict_first loads, x[col] gathered (evict_last), one
+// fma per nonzero, row_ptr read and y written once -- with no row structure
+// (no segmented sums, no per-row work imbalance).  Its time is the practical
+// floor of the variant kernels on this box; the result is not y = Ax.
+// FLAV 0: x gathered at col (the matrix's access pattern); FLAV 1: x read at
+// the nonzero's own index modulo a power of two <= n_cols (same bytes,
+// sequential: the stream floor).
+template <int FLAV>
+__global__ void __launch_bounds__(kUnitRows) spmv_gather_probe_kernel(SpmvDev A, float *out, int64_t nnz, int64_t xmask) {
+  const uint64_t ps = policy_evict_first(), px = policy_evict_last();
+  const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t n4 = nnz >> 2;
+  float acc = 0.0f;
+  auto xat = [&](int c, int64_t k) -> float {
+    if (FLAV == 0) return ld_x(A.x + c, px);
+    return ld_x(A.x + ((k ^ (int64_t)(c & 1)) & xmask), px);   // keeps the col stream live
+  };
+  for (int64_t q = t; q < n4; q += 2 * nthr) {
+    const int64_t q1 = q + nthr;
+    const bool h1 = q1 < n4;
+    const int4 c0 = ld_stream4(A.col + 4 * q, ps);
+    const float4 v0 = ld_stream4(A.val + 4 * q, ps);
+    const int4 c1 = h1 ? ld_stream4(A.col + 4 * q1, ps) : make_int4(0, 0, 0, 0);
+    const float4 v1 = h1 ? ld_stream4(A.val + 4 * q1, ps) : make_float4(0.f, 0.f, 0.f, 0.f);
+    const float x0 = xat(c0.x, 4 * q), x1 = xat(c0.y, 4 * q + 1), x2 = xat(c0.z, 4 * q + 2), x3 = xat(c0.w, 4 * q + 3);
+    const float z0 = xat(c1.x, 4 * q1), z1 = xat(c1.y, 4 * q1 + 1), z2 = xat(c1.z, 4 * q1 + 2),
+                z3 = xat(c1.w, 4 * q1 + 3);
+    acc = __fmaf_rn(v0.x, x0, acc);
+    acc = __fmaf_rn(v0.y, x1, acc);
+    acc = __fmaf_rn(v0.z, x2, acc);
+    acc = __fmaf_rn(v0.w, x3, acc);
+    acc = __fmaf_rn(v1.x, z0, acc);
+    acc = __fmaf_rn(v1.y, z1, acc);
+    acc = __fmaf_rn(v1.z, z2, acc);
+    acc = __fmaf_rn(v1.w, z3, acc);
+  }
+  for (int64_t k = 4 * n4 + t; k < nnz; k += nthr) acc = __fmaf_rn(ld_stream(A.val + k, ps), xat(ld_stream(A.col + k, ps), k), acc);
+  for (int64_t i = t; i < A.n_rows; i += nthr) out[i] = acc + (float)__ldg(A.row_ptr + i + (i == A.n_rows - 1));
+}
+
 }  // namespace dysel
 
 using namespace dysel;
 
 extern "C" {
+
+dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *pl, int flavour, const float *d_x, float *d_out,
+                                     void *stream) {
+  if (!ctx || !pl || (flavour != 0 && flavour != 1) || (pl->dev.n_rows > 0 && !d_out) ||
+      (pl->info.nnz > 0 && !d_x)) {
+    set_error(ctx, "dysel_spmv_gather_probe: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  if (pl->info.nnz > 0 && !pl->dev.vec_ok) {
+    set_error(ctx, "dysel_spmv_gather_probe: col / val not 16-byte aligned");
+    return DYSEL_ERR_UNSUPPORTED;
+  }
+  if (pl->dev.n_rows == 0) return DYSEL_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  SpmvDev A = pl->dev;
+  A.x = d_x;
+  int occ = 0;
+  if (flavour == 0)
+    DYSEL_CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, spmv_gather_probe_kernel<0>, kUnitRows, 0));
+  else
+    DYSEL_CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, spmv_gather_probe_kernel<1>, kUnitRows, 0));
+  const unsigned grid = (unsigned)std::max(1, occ) * (unsigned)ctx->n_sm;
+  int64_t xmask = 1;
+  while (xmask * 2 <= pl->dev.n_cols) xmask *= 2;
+  xmask -= 1;
+  if (flavour == 0)
+    spmv_gather_probe_kernel<0><<<grid, kUnitRows, 0, st>>>(A, d_out, (int64_t)pl->info.nnz, xmask);
+  else
+    spmv_gather_probe_kernel<1><<<grid, kUnitRows, 0, st>>>(A, d_out, (int64_t)pl->info.nnz, xmask);
+  return check_launch(ctx, "spmv_gather_probe_kernel");
+}
 
 dysel_status dysel_spmv_variant(dysel_ctx *ctx, dysel_spmv_plan *pl, int variant_id, const float *d_x, float *d_y,
                                 void *stream) {
@@ -1076,6 +1172,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   if (sequential) p.async = 0;   // a variant profiled alone: no eager work beside it
   p.def = (uint32_t)pl->def;
   p.k_claim = claim_batch(pl);
+  set_heavy(p, pl);
   const bool cdp = (mode & DYSEL_DEVICE_LAUNCH) != 0;   // round-1 scheme: eager + remainder launched on the device
   {   // reading A-38 (opt-in): one claim kernel (the default's) runs every
       // remainder slot, whichever variant wins — not with CSR-T in the pool

@@ -335,8 +335,8 @@ __device__ __forceinline__ void unit_jds(const SpmvDev &A, uint32_t j, int w, fl
 // takes the scan value at the last lane of its segment.  The per-row order
 // depends only on the row's offset inside its group: deterministic (c-6).
 template <class Poll>
-__device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
-                                                const Poll &poll) {
+__device__ __forceinline__ void unit_csr_stream_s(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
+                                                  const Poll &poll) {
   const uint32_t FULL = 0xffffffffu;
   const int lane = threadIdx.x & 31;
   const int64_t base = (int64_t)j * kUnitRows + w * 32;
@@ -431,6 +431,168 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, in
       if (has) acc += got;
       const int nb = cb + 32;
       o = open_row(nb);
+      oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
+    }
+    if (Poll::active && __any_sync(FULL, poll.warp())) break;   // warp-uniform exit
+  }
+  float P = part;
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
+  if (lane == o) acc += P;
+  if (lane < nr) out[w * 32 + lane] = acc;
+}
+
+// CSR-W, 128-bit form (col / val 16-byte aligned, vec_ok): the group's
+// nonzeros are walked from a = s & ~3 in 128-entry chunks, lane l loading
+// entries cb + 4l .. cb + 4l + 3 with one 128-bit col and one 128-bit val load
+// (4x fewer load requests than 32-bit chunks; the x gathers are the same).
+// Entries outside [s, e) contribute +0.  A chunk wholly inside the open row
+// adds its 4 products to the lane partial; otherwise the row sums come from a
+// two-level segmented scan: sequential within the lane's 4 entries, then a
+// Hillis-Steele scan of the lane totals (segment starts = lanes holding a row
+// start, from a ballot), so a chunk costs ~20 shuffles instead of ~12 per 32
+// entries.  The order of every row's additions depends only on the row's
+// offset inside its group and on s mod 4: deterministic (c-6).
+constexpr int kStreamVec = 2;   // 128-entry chunks in flight per warp (8 x gathers per lane)
+template <class Poll>
+__device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
+                                                const Poll &poll) {
+#ifndef DYSEL_EXP_CSRW_SCALAR
+#define DYSEL_EXP_CSRW_SCALAR 0   // experiment knob (scripts/build_exp.py): force the 32-bit form
+#endif
+  if (!A.vec_ok || DYSEL_EXP_CSRW_SCALAR) {
+    unit_csr_stream_s(A, j, w, out, poll);
+    return;
+  }
+  const uint32_t FULL = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int64_t base = (int64_t)j * kUnitRows + w * 32;
+  const int nr = (int)min((int64_t)32, (int64_t)A.n_rows - base);
+  if (nr <= 0) return;
+  const uint64_t ps = policy_evict_first(), px = policy_evict_last();
+  const int gend = __ldg(A.row_ptr + base + nr);
+  const int re = lane < nr ? __ldg(A.row_ptr + base + lane + 1) : gend;
+  const int rs = lane < nr ? __ldg(A.row_ptr + base + lane) : gend;
+  const int s = __shfl_sync(FULL, rs, 0);
+  const int e = gend;
+  float acc = 0.0f, part = 0.0f;
+  auto open_row = [&](int cb) -> int {
+    const uint32_t m = __ballot_sync(FULL, rs <= cb && cb < re);
+    return m ? __ffs(m) - 1 : -1;
+  };
+  int o = open_row(s);
+  int oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
+  const uint32_t lane_mask_le = (lane == 31) ? FULL : ((2u << lane) - 1u);
+  const bool starts = rs < re;   // this lane's row is non-empty
+  for (int c0 = s & ~3; c0 < e; c0 += 128 * kStreamVec) {
+    // long stretch of the open row ahead (c0 >= s: no foreign entries)
+    if (c0 >= s && oe - c0 >= kStreamLong) {
+      const int a = c0;   // 16-byte aligned here
+      const int body_end = a + ((oe - a) & ~255);
+      bool stop = false;
+      for (int b0 = a; b0 < body_end; b0 += 256) {
+        const int k0 = b0 + 4 * lane, k1 = k0 + 128;
+        const int4 q0 = ld_stream4(A.col + k0, ps), q1 = ld_stream4(A.col + k1, ps);
+        const float4 v0 = ld_stream4(A.val + k0, ps), v1 = ld_stream4(A.val + k1, ps);
+        const float x0 = ld_x(A.x + q0.x, px), x1 = ld_x(A.x + q0.y, px), x2 = ld_x(A.x + q0.z, px),
+                    x3 = ld_x(A.x + q0.w, px);
+        const float z0 = ld_x(A.x + q1.x, px), z1 = ld_x(A.x + q1.y, px), z2 = ld_x(A.x + q1.z, px),
+                    z3 = ld_x(A.x + q1.w, px);
+        part = __fmaf_rn(v0.x, x0, part);
+        part = __fmaf_rn(v0.y, x1, part);
+        part = __fmaf_rn(v0.z, x2, part);
+        part = __fmaf_rn(v0.w, x3, part);
+        part = __fmaf_rn(v1.x, z0, part);
+        part = __fmaf_rn(v1.y, z1, part);
+        part = __fmaf_rn(v1.z, z2, part);
+        part = __fmaf_rn(v1.w, z3, part);
+        if (Poll::active && __any_sync(FULL, poll.warp())) {
+          stop = true;
+          break;
+        }
+      }
+      if (stop) break;
+      c0 = body_end;
+      if (c0 >= e) break;
+    }
+    float p[kStreamVec][4];
+#pragma unroll
+    for (int u = 0; u < kStreamVec; ++u) {
+      const int k = c0 + 128 * u + 4 * lane;
+      int cc[4] = {-1, -1, -1, -1};
+      float vv[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+      if (k + 3 < e) {
+        const int4 q = ld_stream4(A.col + k, ps);
+        const float4 v = ld_stream4(A.val + k, ps);
+        cc[0] = q.x; cc[1] = q.y; cc[2] = q.z; cc[3] = q.w;
+        vv[0] = v.x; vv[1] = v.y; vv[2] = v.z; vv[3] = v.w;
+      } else {
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          if (k + i < e) {
+            cc[i] = ld_stream(A.col + k + i, ps);
+            vv[i] = ld_stream(A.val + k + i, ps);
+          }
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const bool ok = k + i >= s && k + i < e;
+        p[u][i] = ok ? vv[i] * ld_x(A.x + cc[i], px) : 0.0f;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kStreamVec; ++u) {
+      const int cb = c0 + 128 * u;
+      if (cb >= e) break;
+      if (oe >= cb + 128) {   // whole chunk inside the open row
+        part += (p[u][0] + p[u][1]) + (p[u][2] + p[u][3]);
+        continue;
+      }
+      // fold the open row's per-lane partials
+      float P = part;
+#pragma unroll
+      for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
+      if (lane == o) acc += P;
+      part = 0.0f;
+      // head bits of the chunk's 128 entries (word q: entries 32q .. 32q+31);
+      // entry 0 always starts a segment
+      const int off = rs - cb;
+      const bool in = starts && off >= 0 && off < 128;
+      uint32_t hw[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) hw[q] = __reduce_or_sync(FULL, (in && (off >> 5) == q) ? 1u << (off & 31) : 0u);
+      hw[0] |= 1u;
+      const uint32_t word = lane < 8 ? hw[0] : lane < 16 ? hw[1] : lane < 24 ? hw[2] : hw[3];
+      const uint32_t h = (word >> ((4 * lane) & 31)) & 0xfu;
+      // level 1: sequential segmented sums within the lane's 4 entries
+      float v0 = p[u][0];
+      float v1 = (h & 2u) ? p[u][1] : v0 + p[u][1];
+      float v2 = (h & 4u) ? p[u][2] : v1 + p[u][2];
+      float v3 = (h & 8u) ? p[u][3] : v2 + p[u][3];
+      // level 2: segmented inclusive scan of the lane totals
+      const uint32_t H = __ballot_sync(FULL, h != 0u) | 1u;
+      const int seg_start = 31 - __clz(H & lane_mask_le);
+      float c = v3;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const float t = __shfl_up_sync(FULL, c, d);
+        if (lane - d >= seg_start) c += t;
+      }
+      float cin = __shfl_up_sync(FULL, c, 1);
+      if (lane == 0) cin = 0.0f;
+      if (!(h & 1u)) v0 += cin;
+      if (!(h & 3u)) v1 += cin;
+      if (!(h & 7u)) v2 += cin;
+      if (!(h & 15u)) v3 += cin;
+      // each row takes the value at its last entry inside the chunk
+      const int lo = max(rs, cb), hi = min(re, cb + 128);
+      const bool has = lo < hi;
+      const int src = has ? hi - 1 - cb : 0;
+      const float g0 = __shfl_sync(FULL, v0, src >> 2), g1 = __shfl_sync(FULL, v1, src >> 2),
+                  g2 = __shfl_sync(FULL, v2, src >> 2), g3 = __shfl_sync(FULL, v3, src >> 2);
+      const int si = src & 3;
+      if (has) acc += si == 0 ? g0 : si == 1 ? g1 : si == 2 ? g2 : g3;
+      o = open_row(cb + 128);
       oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
     }
     if (Poll::active && __any_sync(FULL, poll.warp())) break;   // warp-uniform exit

@@ -20,10 +20,16 @@ struct dysel_spmv_plan {
   int vids[DYSEL_SPMV_NVARIANTS] = {};  // pool index -> DYSEL_SPMV_* id
   int def = 0;                        // pool index of the default (initial) variant
   uint32_t n_units = 0;               // 256-row units
+  // heavy-first claim order (reading A-40): units with >= 4x the mean and
+  // >= kHeavyUnitNnz nonzeros, by nonzeros descending; bitmap over units
+  int32_t *heavy = nullptr;
+  uint32_t *heavy_bits = nullptr;
+  uint32_t n_heavy = 0;
   std::string sig;                    // generic-registry signature (host path)
 };
 
 namespace dysel {
+constexpr int64_t kHeavyUnitNnz = 8192;   // heavy-first order: minimum nonzeros of a heavy unit (A-40)
 int spmv_pool_index(const dysel_spmv_plan *pl, int vid);
 // register the plan's pool with the generic launcher (host-orchestrated path)
 dysel_status spmv_register_pool(dysel_ctx *ctx, dysel_spmv_plan *pl);

@@ -7,6 +7,7 @@
 //   JDS  per 256-row block b: rows stably sorted by length (descending, ties by
 //        row), perm[b*256+p] = row, jds_len[b*256+p] = its length,
 //        jd_ptr_b[k] = sum_p min(len_p, k), entry (p, k) at blk_off[b] + jd_ptr_b[k] + p.
+#include <vector>
 #include <cub/device/device_scan.cuh>
 
 #include <algorithm>
@@ -38,6 +39,12 @@ __global__ void ell_fill_kernel(const int32_t *__restrict__ rp, const int32_t *_
 }
 
 // phase 1: per block, stable sort by length (rank counting), W_b + 1
+// row_ptr at the 256-row unit boundaries (heavy-first order, reading A-40)
+__global__ void unit_bounds_kernel(const int32_t *__restrict__ rp, int64_t n, int64_t nu, int32_t *__restrict__ ub) {
+  const int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (u <= nu) ub[u] = rp[min(u * kUnitRows, n)];
+}
+
 __global__ void __launch_bounds__(kUnitRows) jds_sort_kernel(const int32_t *__restrict__ rp, int64_t n,
                                                              int32_t *__restrict__ perm,
                                                              int32_t *__restrict__ jds_len,
@@ -232,6 +239,45 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
   if (formats_mask & DYSEL_FMT_STREAM) pl->vids[pl->K++] = DYSEL_SPMV_CSR_STREAM;
   if (formats_mask & DYSEL_FMT_TMA) pl->vids[pl->K++] = DYSEL_SPMV_CSR_TMA;
   if (cudaStreamSynchronize(st) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  {   // heavy-first claim order (reading A-40): the claim kernels run the
+      // heaviest units first (longest-processing-time order), so no warp
+      // starts a 10^4-entry row in the last microseconds of a launch
+    const int64_t nu = pl->n_units;
+    const int64_t mean = nu > 0 ? nnz / nu : 0;
+    const int64_t thr = std::max<int64_t>(kHeavyUnitNnz, 4 * mean);
+#ifndef DYSEL_EXP_NO_HEAVY
+#define DYSEL_EXP_NO_HEAVY 0   // experiment knob (scripts/build_exp.py): rows-in-order claims
+#endif
+    // (single-wave grids -- fewer than 4 units per SM -- keep the plain order:
+    // every slot starts at once; measured 39 vs 41 us at 235 units)
+    if (!DYSEL_EXP_NO_HEAVY && nu >= 4 * (int64_t)ctx->n_sm && nnz >= 2 * thr) {
+      std::vector<int32_t> ub(nu + 1);
+      int32_t *d_ub = nullptr;
+      if (cudaMalloc(&d_ub, (nu + 1) * 4) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+      unit_bounds_kernel<<<(unsigned)((nu + 256) / 256), 256, 0, st>>>(d_row_ptr, n_rows, nu, d_ub);
+      const bool ok = cudaMemcpyAsync(ub.data(), d_ub, (nu + 1) * 4, cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+                      cudaStreamSynchronize(st) == cudaSuccess;
+      cudaFree(d_ub);
+      if (!ok) return fail(DYSEL_ERR_CUDA);
+      std::vector<int32_t> hv;
+      for (int64_t u = 0; u < nu; ++u)
+        if ((int64_t)ub[u + 1] - ub[u] >= thr) hv.push_back((int32_t)u);
+      std::stable_sort(hv.begin(), hv.end(),
+                       [&](int32_t a, int32_t b) { return ub[a + 1] - ub[a] > ub[b + 1] - ub[b]; });
+      if (!hv.empty()) {
+        std::vector<uint32_t> bits((nu + 31) / 32, 0u);
+        for (int32_t u : hv) bits[u >> 5] |= 1u << (u & 31);
+        if (cudaMalloc(&pl->heavy, hv.size() * 4) != cudaSuccess ||
+            cudaMalloc(&pl->heavy_bits, bits.size() * 4) != cudaSuccess)
+          return fail(DYSEL_ERR_NOMEM);
+        if (cudaMemcpy(pl->heavy, hv.data(), hv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+            cudaMemcpy(pl->heavy_bits, bits.data(), bits.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
+          return fail(DYSEL_ERR_CUDA);
+        pl->n_heavy = (uint32_t)hv.size();
+        I.n_heavy = (int32_t)hv.size();
+      }
+    }
+  }
   if (default_variant == DYSEL_SPMV_DEFAULT_AUTO) {   // reading A-30: initial version from row statistics
     if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
     else if (spmv_pool_index(pl, DYSEL_SPMV_CSR_STREAM) >= 0) default_variant = DYSEL_SPMV_CSR_STREAM;
@@ -308,6 +354,8 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *pl) {
   cudaFree(pl->jds_val);
   cudaFree(pl->blk_off);
   cudaFree(pl->jd_off);
+  cudaFree(pl->heavy);
+  cudaFree(pl->heavy_bits);
   cudaGetLastError();
   delete pl;
 }

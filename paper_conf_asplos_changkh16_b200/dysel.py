@@ -70,7 +70,7 @@ class PlanInfo(ctypes.Structure):
     _fields_ = [("n_rows", c_i64), ("n_cols", c_i64), ("nnz", c_i64), ("n_variants", ctypes.c_int32),
                 ("variant_ids", ctypes.c_int32 * SPMV_NVARIANTS), ("ell_width", ctypes.c_int32), ("uniform", ctypes.c_int32),
                 ("max_row_len", ctypes.c_int32), ("prep_ns", c_u64), ("ell_bytes", c_u64), ("jds_bytes", c_u64),
-                ("default_variant", ctypes.c_int32)]
+                ("default_variant", ctypes.c_int32), ("n_heavy", ctypes.c_int32)]
 
 
 def _sig(name, res, *args):
@@ -100,6 +100,7 @@ dysel_spmv_plan_destroy = _sig("dysel_spmv_plan_destroy", None, P)
 dysel_spmv_plan_copy_array = _sig("dysel_spmv_plan_copy_array", c_int, P, c_int, P, ctypes.POINTER(c_size))
 dysel_spmv = _sig("dysel_spmv", c_int, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
 dysel_spmv_variant = _sig("dysel_spmv_variant", c_int, P, P, c_int, P, P, P)
+dysel_spmv_gather_probe = _sig("dysel_spmv_gather_probe", c_int, P, P, c_int, P, P, P)
 dysel_sgemm = _sig("dysel_sgemm", c_int, P, c_int, c_int, c_int, c_float, P, c_int, P, c_int, c_float, P, c_int,
                    c_float, c_u32, P, ctypes.POINTER(Report))
 dysel_sgemm_variant = _sig("dysel_sgemm_variant", c_int, P, c_int, c_int, c_int, c_int, c_float, P, c_int, P, c_int,
@@ -302,6 +303,10 @@ class Context:
 
     def spmv_variant(self, plan, variant_id, x, y, stream=None):
         self._check(dysel_spmv_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), _stream(stream)))
+
+    def spmv_gather_probe(self, plan, flavour, x, out, stream=None):
+        """Measurement only: the plan's CSR traffic with no row structure (include/dysel.h)."""
+        self._check(dysel_spmv_gather_probe(self.h, plan.handle, int(flavour), _ptr(x), _ptr(out), _stream(stream)))
 
     # ------------------------------------------------------------ SGEMM
     def sgemm(self, A, B, C, alpha=1.0, beta=0.0, f=0.02, mode=DEFAULT_MODE, report=False, unit_map=False,

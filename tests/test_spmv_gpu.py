@@ -17,6 +17,8 @@ MATS = {
     "d3small": lambda: d3_fem(grid=101),
     "powerlaw": lambda: d4_powerlaw(n=60_000, lmax=4000),
     "diag": lambda: d6_diag(n=70_000),
+    # 16,384-entry rows: heavy units, run first by the claim kernels (A-40)
+    "heavy": lambda: d4_powerlaw(n=300_000, lmax=16384),
 }
 
 
@@ -87,7 +89,7 @@ def test_variants_parity(ctx, D, name):
     plan.destroy()
 
 
-@pytest.mark.parametrize("name", ["d1", "ragged", "powerlaw"])
+@pytest.mark.parametrize("name", ["d1", "ragged", "powerlaw", "heavy"])
 def test_small_integer_bit_exact(ctx, name):
     import torch
     A = small_int_csr(MATS[name](), 5)
@@ -140,7 +142,7 @@ def mode_bits(D, m):
 
 
 @pytest.mark.parametrize("m", MODES)
-@pytest.mark.parametrize("name", ["ragged", "powerlaw", "d3small"])
+@pytest.mark.parametrize("name", ["ragged", "powerlaw", "d3small", "heavy"])
 def test_dysel_composition(ctx, D, name, m):
     """c-6: y_dysel restricted to unit u == y_full[v(u)] restricted to u, bitwise;
     every unit productively computed exactly once; parity vs oracle."""
@@ -375,4 +377,52 @@ def test_csr_tma_multi_slot(ctx, D, name):
         outs[v] = y.cpu().numpy()
     assert spmv_err(A, x, torch.from_numpy(outs[D.SPMV_CSR_TMA])) <= SPMV_TOL
     assert np.array_equal(outs[D.SPMV_CSR_TMA].view(np.uint32), outs[D.SPMV_CSR_SCALAR].view(np.uint32))
+    plan.destroy()
+
+
+def test_gather_probe_runs_and_validates(ctx, D):
+    """dysel_spmv_gather_probe (measurement only): both flavours
+    run on an aligned plan and write every one of d_out's n_rows floats; a bad
+    flavour is rejected with DYSEL_ERR_INVALID."""
+    import torch
+    A = MATS["powerlaw"]()
+    plan = prepared(ctx, A)
+    x = vec(uniform_f32(5, A.n_cols))
+    for fl in (0, 1):
+        out = torch.full((A.n_rows,), float("nan"), device="cuda")
+        ctx.spmv_gather_probe(plan, fl, x, out)
+        torch.cuda.synchronize()
+        assert bool(torch.isfinite(out).all())
+    with pytest.raises(Exception):
+        ctx.spmv_gather_probe(plan, 2, x, out)
+    plan.destroy()
+
+
+@pytest.mark.parametrize("name", ["heavy", "powerlaw", "d3small"])
+def test_heavy_first_units(ctx, D, name):
+    """Reading A-40: the plan's heavy units are exactly those with at least
+    max(8192, 4 x mean) nonzeros when the grid spans >= 4 units per SM (rule
+    restated here); every pure variant's heavy-first claim run is within
+    tolerance of the oracle, and CSR-S / ELL / JDS stay bit-identical."""
+    import torch
+    A = MATS[name]()
+    plan = prepared(ctx, A)
+    nu = (A.n_rows + 255) // 256
+    ub = A.row_ptr[np.minimum(np.arange(nu + 1) * 256, A.n_rows)].astype(np.int64)
+    thr = max(8192, 4 * (A.nnz // nu))
+    want = int((np.diff(ub) >= thr).sum()) if (A.nnz >= 2 * thr and nu >= 4 * ctx.n_sm) else 0
+    assert plan.info.n_heavy == want
+    if name == "heavy":
+        assert want > 0
+    x = uniform_f32(9, A.n_cols)
+    xd = vec(x)
+    ys = {}
+    for v in plan.variant_ids:
+        y = torch.full((A.n_rows,), float("nan"), device="cuda")
+        ctx.spmv_variant(plan, v, xd, y)
+        ys[v] = y.cpu().numpy()
+        assert spmv_err(A, x, y) <= SPMV_TOL, v
+    for v in (0, 2, 3):   # CSR-S, ELL, JDS: bit-identical by construction
+        if v in ys:
+            assert np.array_equal(ys[v], ys[0]), v
     plan.destroy()
