@@ -275,6 +275,9 @@ def dysel_arm(args, world, rank, local_rank):
                                                / T_star - 1) * 100, 2)
         ablation["solo_claim_kernel_overhead_pct"] = round(
             (time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=mode | D.SOLO), 10, stream) / T_star - 1) * 100, 2)
+        ablation["all_claim_kernels_overhead_pct"] = round(
+            (time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=mode | D.ALL_CLAIMS), 10, stream) / T_star - 1) * 100,
+            2)
         ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10, stream)
                                                       / T_star - 1) * 100, 2) for ff in (0.001, 0.005, 0.01, 0.02)}
         # iterative driver (SURVEY §8f f-3, P:L796-804 / §5.2): 20 power
@@ -297,7 +300,9 @@ def dysel_arm(args, world, rank, local_rank):
             pd = ctx.spmv_prepare(rp, col, val, A.n_cols, default=dv)
             td = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode), 10, stream)
             rd = ctx.spmv(pd, xd, yl, f=f, mode=mode, report=True)
+            tda = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode | D.ALL_CLAIMS), 10, stream)
             ablation[f"default_{dname}"] = {"overhead_pct": round((td / T_star - 1) * 100, 2),
+                                            "all_claims_overhead_pct": round((tda / T_star - 1) * 100, 2),
                                             "selected": rd["selected_name"], "eager_units": rd["eager_units"]}
             pd.destroy()
     xh = torch.from_numpy(x).pin_memory()
@@ -405,8 +410,9 @@ def dysel_arm(args, world, rank, local_rank):
                      "aborted_sandbox_units": {D.SPMV_NAMES[v]: rep["aborted"][v] for v in plan.variant_ids},
                      "busy_us_per_unit": {D.SPMV_NAMES[v]: round(rep["busy_ns"][v] / max(1, rep["units"][v]) / 1e3, 2)
                                           for v in plan.variant_ids},
-                     "kernels": "init + one profiling kernel (K variants) + K claim kernels (PDL-chained, "
-                                "default first: eager, then the winner's remainder)"},
+                     "kernels": "init + one profiling kernel (K variants) + the default's claim kernel (eager, "
+                                "then the remainder if it wins) + a one-warp switch kernel that device-launches "
+                                "the winner's claim kernel only when the default lost (A-42), PDL-chained"},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": pk["hbm_gbs"], "unit": "GB/s",
                          "frac": round(achieved / pk["hbm_gbs"], 4), "traffic": traffic,
                          "kernel": f"dysel::spmv_claim_kernel<{sel_name}> (pure full grid, event-timed back to back)",

@@ -97,6 +97,10 @@ const char *dysel_status_str(dysel_status s);
                                    variants at the default's occupancy) — saves the non-winning claim grids
                                    (~1.6% on D4 when the default wins), costs far more when it does not
                                    (+44% with a CSR-V default on D4); ignored when the pool holds CSR-T */
+#define DYSEL_ALL_CLAIMS 16384u /* SpMV device path (ablation of reading A-42): host-launch every pool variant's
+                                   claim kernel (PDL-chained, default first) instead of the default's claim kernel
+                                   plus a one-warp switch kernel that device-launches the winner's claim kernel
+                                   only when the default lost */
 /* Default score: generic launcher = makespan (variants are separate concurrent
  * grids, Fig. 7b); SpMV dispatcher = mean per-unit busy time (%globaltimer end -
  * start of each profiled unit; all variants share one launch and occupancy). */

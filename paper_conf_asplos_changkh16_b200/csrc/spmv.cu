@@ -711,6 +711,32 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
 // debug: selection preset to pool index pv with no eager range (claim kernel alone)
 // eager_all: the eager range stays open (c1 unpublished) and S = n_slots, so
 // the default's eager phase runs the whole grid
+// Switch kernel (reading A-42, the default SpMV device path): instead of one
+// host-launched claim kernel per non-default variant -- K - 1 full grids that,
+// when the default wins, only drain as exiting CTAs at the end of the step --
+// one 32-thread CTA queued behind the default's claim kernel waits for the
+// selection and, only if another variant won, launches that variant's claim
+// kernel from the device (fire-and-forget: stream order is kept, the parent
+// grid completes with its child).  The child enters the remainder at the
+// published switch point S like a host-launched one.
+__global__ void spmv_switch_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p) {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  if (threadIdx.x != 0) return;
+  const uint64_t sw = wait_published(&st->sw);
+  const uint32_t w = (uint32_t)(sw & 0xff);
+  if (w == p.def || w >= p.K || p.p_end >= p.n_units) return;
+  const unsigned g = (unsigned)min((uint64_t)p.occ[w] * p.n_sm, (uint64_t)(p.n_units - p.p_end));
+  const cudaStream_t ff = cudaStreamFireAndForget;
+  switch (p.vids[w]) {
+    case 0: spmv_claim_kernel<0><<<g, kUnitRows, dyn_smem(0), ff>>>(A, y, st, p, w); break;
+    case 1: spmv_claim_kernel<1><<<g, kUnitRows, dyn_smem(1), ff>>>(A, y, st, p, w); break;
+    case 2: spmv_claim_kernel<2><<<g, kUnitRows, dyn_smem(2), ff>>>(A, y, st, p, w); break;
+    case 3: spmv_claim_kernel<3><<<g, kUnitRows, dyn_smem(3), ff>>>(A, y, st, p, w); break;
+    case 4: spmv_claim_kernel<4><<<g, kUnitRows, dyn_smem(4), ff>>>(A, y, st, p, w); break;
+    default: spmv_claim_kernel<5><<<g, kUnitRows, dyn_smem(5), ff>>>(A, y, st, p, w); break;
+  }
+}
+
 __global__ void spmv_state_preset_kernel(SpmvState *s, uint32_t pv, int eager_all, uint64_t n_slots) {
   s->sel = pv;
   s->c1 = eager_all ? 0ull : 1ull << 32;
@@ -1224,13 +1250,29 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
     // launch lets them start while profiling runs (not after NO_TAIL or a
     // sequential profile: then they follow in stream order)
     const bool pdl = !(mode & DYSEL_NO_TAIL) && !sequential;
-    for (int k = 0; k < (p.solo ? 1 : pl->K); ++k) {
+    // reading A-42: the default's claim kernel + the switch kernel, unless
+    // DYSEL_ALL_CLAIMS (every variant's claim kernel from the host)
+    const bool sw_k = pdl && !p.solo && !(mode & DYSEL_ALL_CLAIMS) && pl->K > 1;
+    for (int k = 0; k < (p.solo || sw_k ? 1 : pl->K); ++k) {
       const uint32_t i = (uint32_t)(k == 0 ? pl->def : (k <= pl->def ? k - 1 : k));
       const int v = pl->vids[i];
       const uint64_t g = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[v]) * ctx->n_sm,
                                             p.n_units - p.p_end);
       DYSEL_TRY(kClaim[v](A, d_y, dst, p, i, (unsigned)g, st, pdl));
       DYSEL_TRY(check_launch(ctx, "spmv_claim_kernel"));
+    }
+    if (sw_k) {
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(1);
+      cfg.blockDim = dim3(32);
+      cfg.stream = st;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      DYSEL_CUDA_TRY(ctx, cudaLaunchKernelEx(&cfg, spmv_switch_kernel, A, d_y, dst, p));
+      DYSEL_TRY(check_launch(ctx, "spmv_switch_kernel"));
     }
   } else if (cdp && !p.tail && !p.async && p.p_end < p.n_units) {   // CDP scheme, NO_TAIL: winner via claim kernels
     for (int i = 0; i < pl->K; ++i) {

@@ -27,6 +27,7 @@ FULLY, HYBRID, SWAP, AUTO = 0, 1, 2, 3
 SYNC, ASYNC = 0, 4
 NO_PROFILE, HOST_ORCH, FORCE_PROFILE, CONTIGUOUS, SCORE_CYCLES = 8, 16, 32, 64, 128
 SCORE_MAKESPAN, NO_TAIL, NO_ABORT, SEQUENTIAL, DEVICE_LAUNCH, SOLO = 256, 512, 1024, 2048, 4096, 8192
+ALL_CLAIMS = 16384
 DEFAULT_MODE = FULLY | ASYNC
 V_ATOMICS, V_NONUNIFORM = 1, 2
 ROLE_PRODUCTIVE, ROLE_SANDBOX, ROLE_BATCH, ROLE_PRIVATE, ROLE_EAGER = range(5)

@@ -124,7 +124,8 @@ def test_identity_and_diagonal_exact(ctx):
 
 MODES = ["fully_sync", "fully_async", "hybrid_sync", "hybrid_async", "fully_sync_host", "fully_async_host",
          "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles", "hybrid_async_cdp", "fully_sync_cdp",
-         "hybrid_async_notail", "fully_sync_seq", "hybrid_async_solo", "fully_sync_solo"]
+         "hybrid_async_notail", "fully_sync_seq", "hybrid_async_solo", "fully_sync_solo", "hybrid_async_allclaims",
+         "fully_async_allclaims"]
 
 
 def mode_bits(D, m):
@@ -138,6 +139,7 @@ def mode_bits(D, m):
     b |= D.NO_TAIL if "notail" in m else 0
     b |= D.SEQUENTIAL if "seq" in m else 0
     b |= D.SOLO if "solo" in m else 0
+    b |= D.ALL_CLAIMS if "allclaims" in m else 0
     return b
 
 
@@ -255,8 +257,10 @@ def test_edge_cases(ctx, D):
 
 @pytest.mark.parametrize("asy", [False, True])
 def test_remainder_hand_off(ctx, D, asy):
-    """The remainder goes to the winner in every launch scheme: host-launched
-    claim kernels started beside profiling (PDL, default), the same after
+    """The remainder goes to the winner in every launch scheme: the default's
+    claim kernel + the switch kernel that device-launches a non-default
+    winner's claim kernel (A-42, default), every variant's claim kernel
+    host-launched beside profiling (PDL, ALL_CLAIMS), the same after
     profiling completes (NO_TAIL), and the round-1 device-launched scheme
     (DEVICE_LAUNCH: CDP2 eager + remainder, with and without NO_TAIL).
     Sync: every remainder unit is the winner's (eager = 0); async: the
@@ -266,7 +270,7 @@ def test_remainder_hand_off(ctx, D, asy):
     x = uniform_f32(11, A.n_cols)
     plan = prepared(ctx, A, default=1)
     K = len(plan.variant_ids)
-    for extra in (0, D.NO_TAIL, D.DEVICE_LAUNCH, D.DEVICE_LAUNCH | D.NO_TAIL):
+    for extra in (0, D.ALL_CLAIMS, D.NO_TAIL, D.DEVICE_LAUNCH, D.DEVICE_LAUNCH | D.NO_TAIL):
         mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0) | extra
         y = torch.full((A.n_rows,), float("nan"), device="cuda")
         r = ctx.spmv(plan, vec(x), y, f=0.05, mode=mode, report=True, unit_map=True)
