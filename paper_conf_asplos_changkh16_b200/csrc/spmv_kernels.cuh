@@ -35,7 +35,10 @@ constexpr int kVecMin = 128;   // CSR-V: rows at least this long use 128-bit loa
 constexpr int kRowBatch = 4;   // CSR-V: rows in flight per warp
 constexpr int kChunk = 8;      // CSR-S / ELL / JDS: entries per thread in flight
 constexpr int kStreamUnroll = 4;   // CSR-W: 32-entry chunks in flight per warp
-constexpr int kStreamLong = 512;   // CSR-W: open-row stretch that switches to 128-bit loads
+#ifndef DYSEL_STREAM_LONG
+#define DYSEL_STREAM_LONG 512
+#endif
+constexpr int kStreamLong = DYSEL_STREAM_LONG;   // CSR-W: open-row stretch that switches to the 256-entry loop
 
 struct SpmvDev {
   int32_t n_rows, n_cols;
@@ -453,7 +456,10 @@ __device__ __forceinline__ void unit_csr_stream_s(const SpmvDev &A, uint32_t j, 
 // start, from a ballot), so a chunk costs ~20 shuffles instead of ~12 per 32
 // entries.  The order of every row's additions depends only on the row's
 // offset inside its group and on s mod 4: deterministic (c-6).
-constexpr int kStreamVec = 2;   // 128-entry chunks in flight per warp (8 x gathers per lane)
+#ifndef DYSEL_STREAM_VEC
+#define DYSEL_STREAM_VEC 2
+#endif
+constexpr int kStreamVec = DYSEL_STREAM_VEC;   // 128-entry chunks in flight per warp (8 x gathers per lane)
 template <class Poll>
 __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
                                                 const Poll &poll) {
