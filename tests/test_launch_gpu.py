@@ -110,3 +110,31 @@ def test_timer_calibration(ctx):
     tick, cpn = ctx.timer_calibrate()
     assert 0 < tick <= 2000
     assert 0.3 < cpn < 3.0      # SM clock 0.3-3 GHz
+
+
+def test_timer_makespan_vs_cuda_events(ctx, D):
+    """c-9: a variant's device-measured makespan (earliest %globaltimer CTA
+    start .. latest CTA end over its slice) matches the known spin cost of a
+    unit (its c CTAs run side by side), and a full one-wave launch of the
+    same spin variant timed by CUDA events on the launching stream takes that
+    cost plus launch latency (slices >= 100 us, SURVEY c-9)."""
+    import torch
+    costs = [150_000, 100_000, 300_000, 250_000]
+    rep, _ = run(ctx, D, "spin.c9", 600, D.FULLY, costs=costs)
+    assert rep["profiled"] and rep["selected"] == 1
+    for v, c in enumerate(costs):
+        ms = rep["makespan_ns"][v]
+        assert c <= ms <= 1.2 * c + 30_000, (v, c, ms)
+    out = torch.zeros(100, dtype=torch.int32, device="cuda")
+    s = torch.cuda.current_stream()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ctx.launch("spin.c9", (100,), [out], mode=D.NO_PROFILE)   # warm
+    torch.cuda.synchronize()
+    a.record(s)
+    ctx.launch("spin.c9", (100,), [out], mode=D.NO_PROFILE)   # cached winner: 100 us per unit
+    b.record(s)
+    torch.cuda.synchronize()
+    ev_ns = a.elapsed_time(b) * 1e6
+    assert costs[1] <= ev_ns <= 1.2 * costs[1] + 30_000, ev_ns
+    assert abs(ev_ns - rep["makespan_ns"][1]) <= 0.2 * costs[1] + 30_000
+    assert set(np.unique(out.cpu().numpy())) == {2}
