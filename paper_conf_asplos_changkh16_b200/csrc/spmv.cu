@@ -80,6 +80,9 @@ struct ProfParams {
 };
 
 __global__ void spmv_state_init_kernel(SpmvState *s, int K, int def) {
+  // the profiling kernel behind it (PDL) may launch now; it waits for this
+  // grid's completion (griddepcontrol.wait) before touching the state
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int v = threadIdx.x;
   if (v < DYSEL_MAX_VARIANTS) {
     s->ctas_done[v] = 0;
@@ -533,6 +536,9 @@ template <bool CDP>
 __global__ void __launch_bounds__(kUnitRows, DYSEL_PROF_MINB)
     spmv_prof_all_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p) {
   tma_stage_prologue();
+  // launched behind the init kernel with PDL: wait for its state reset (a
+  // no-op when launched without the attribute)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   // programmatic dependent launch: the claim kernels queued behind this one
   // may start as soon as every profiling CTA is resident
   if constexpr (!CDP) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -1239,10 +1245,24 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       DYSEL_TRY(check_launch(ctx, "spmv_prof_kernel"));
     }
   } else {   // all K profiling slices in one launch on the stream
-    if (cdp)
+    if (cdp) {
       spmv_prof_all_kernel<true><<<p.K * p.c, kUnitRows, pool_dyn_smem(p), st>>>(A, d_y, dst, p);
-    else
-      spmv_prof_all_kernel<false><<<p.K * p.c, kUnitRows, pool_dyn_smem(p), st>>>(A, d_y, dst, p);
+    } else {   // PDL behind the init kernel: launch latency overlaps the reset
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(p.K * p.c);
+      cfg.blockDim = dim3(kUnitRows);
+      cfg.dynamicSmemBytes = pool_dyn_smem(p);
+      cfg.stream = st;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = attr;
+#ifndef DYSEL_EXP_NO_PDL_INIT
+#define DYSEL_EXP_NO_PDL_INIT 0   // experiment knob (scripts/build_exp.py): plain stream order
+#endif
+      cfg.numAttrs = DYSEL_EXP_NO_PDL_INIT ? 0 : 1;
+      DYSEL_CUDA_TRY(ctx, cudaLaunchKernelEx(&cfg, spmv_prof_all_kernel<false>, A, d_y, dst, p));
+    }
     DYSEL_TRY(check_launch(ctx, "spmv_prof_all_kernel"));
   }
   if (!cdp && p.p_end < p.n_units) {

@@ -21,7 +21,7 @@ y = torch.empty(A.n_rows, device="cuda")
 for fm, label, dflt in ((D.FMT_DEFAULT, "pool4", D.SPMV_DEFAULT_AUTO), (D.FMT_DEFAULT, "pool4_defV", 1)):
     plan = ctx.spmv_prepare(rp, col, val, A.n_cols, formats=fm, default=dflt)
     T = b2b(lambda: ctx.spmv_variant(plan, 4, x, y))
-    print(label, "pure csr_stream", round(T, 1), "us", flush=True)
+    print(os.environ.get("DYSEL_LIB", "default"), label, "pure csr_stream", round(T, 1), "us", flush=True)
     for name, mode, f in [("hyb_async", D.AUTO | D.ASYNC, 0.002), ("hyb_async", D.AUTO | D.ASYNC, 0.001),
                           ("hyb_async", D.AUTO | D.ASYNC, 0.0005), ("no_profile", D.AUTO | D.NO_PROFILE, 0.002),
                           ("fully_async", D.FULLY | D.ASYNC, 0.002), ("hyb_sync", D.AUTO, 0.002),
