@@ -17,6 +17,8 @@
 //      profiles run; publishing the selection grabs the unclaimed tickets for
 //      the tail launch, so eager work stops and the winner takes over.
 // Hybrid sandbox units of a provably losing variant stop early (dominance).
+#include <cudaTypedefs.h>
+
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
@@ -993,6 +995,103 @@ __global__ void __launch_bounds__(kUnitRows) spmv_gather_probe_kernel(SpmvDev A,
   for (int64_t i = t; i < A.n_rows; i += nthr) out[i] = acc + (float)__ldg(A.row_ptr + i + (i == A.n_rows - 1));
 }
 
+// FLAV 2 (experiment, same contract): x gathered by the TMA unit instead of
+// the LSU -- each lane issues one cp.async.bulk.tensor tile::gather4 per 4
+// nonzeros (x viewed as rows of 4 floats; the 4 rows col >> 2 land in a
+// 128-byte shared slot), two 128-entry chunks in flight per warp (mbarrier
+// per stage), then reads x[col] from shared memory.  Tests whether moving
+// the gathers off the L1TEX pipe lowers the floor.
+constexpr int kG4Warps = kUnitRows / 32;
+struct G4Smem {
+  float buf[kG4Warps][2][32][32];   // warp, stage, lane: 128-byte slot (4 rows x 16 B used)
+  unsigned long long bar[kG4Warps][2];
+};
+template <bool VERIFY>
+__global__ void __launch_bounds__(kUnitRows) spmv_gather4_probe_kernel(const __grid_constant__ CUtensorMap tmX,
+                                                                      SpmvDev A, float *out, int64_t nnz,
+                                                                      uint32_t *err) {
+  extern __shared__ __align__(1024) unsigned char g4_smem[];
+  G4Smem &S = *reinterpret_cast<G4Smem *>(g4_smem);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint64_t ps = policy_evict_first(), px = policy_evict_last();
+  if (lane < 2)
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(spmv_smem_u32(&S.bar[w][lane])) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncwarp();
+  uint32_t phase[2] = {0u, 0u};
+  const int64_t nch = nnz / 128;
+  const int64_t nw = (int64_t)gridDim.x * kG4Warps;
+  const int64_t gw = (int64_t)blockIdx.x * kG4Warps + w;
+  auto issue = [&](int64_t ch, int st, int4 &c, float4 &v) {
+    const int64_t k = ch * 128 + 4 * lane;
+    c = ld_stream4(A.col + k, ps);
+    v = ld_stream4(A.val + k, ps);
+    const uint32_t bar = spmv_smem_u32(&S.bar[w][st]);
+    if (lane == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(32 * 64) : "memory");
+    }
+    __syncwarp();
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%3, %4, %5, %6, %7}], [%2], %8;" ::"r"(spmv_smem_u32(&S.buf[w][st][lane][0])),
+        "l"(&tmX), "r"(bar), "r"(0), "r"(c.x >> 2), "r"(c.y >> 2), "r"(c.z >> 2), "r"(c.w >> 2), "l"(px)
+        : "memory");
+  };
+  float acc = 0.0f;
+  int4 cc = make_int4(0, 0, 0, 0), cn = cc;
+  float4 vc = make_float4(0.f, 0.f, 0.f, 0.f), vn = vc;
+  int st = 0;
+  if (gw < nch) issue(gw, 0, cc, vc);
+  for (int64_t ch = gw; ch < nch; ch += nw, st ^= 1) {
+    if (ch + nw < nch) issue(ch + nw, st ^ 1, cn, vn);
+    const uint32_t bar = spmv_smem_u32(&S.bar[w][st]);
+    uint32_t ok = 0;
+    for (uint32_t spins = 0; !ok; ++spins) {
+      asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                   : "=r"(ok)
+                   : "r"(bar), "r"(phase[st])
+                   : "memory");
+      if (!ok && spins > (1u << 22)) {   // a mis-sized transfer must not hang the box
+        atomicExch(err, 1u);
+        return;
+      }
+    }
+    phase[st] ^= 1u;
+    const float *b = S.buf[w][st][lane];
+    if (VERIFY) {   // flavour 3: the TMA-gathered values must be x[col]
+      const bool bad = b[0 + (cc.x & 3)] != A.x[cc.x] || b[4 + (cc.y & 3)] != A.x[cc.y] ||
+                       b[8 + (cc.z & 3)] != A.x[cc.z] || b[12 + (cc.w & 3)] != A.x[cc.w];
+      if (bad) atomicOr(err, 2u);
+    }
+    acc = __fmaf_rn(vc.x, b[0 + (cc.x & 3)], acc);
+    acc = __fmaf_rn(vc.y, b[4 + (cc.y & 3)], acc);
+    acc = __fmaf_rn(vc.z, b[8 + (cc.z & 3)], acc);
+    acc = __fmaf_rn(vc.w, b[12 + (cc.w & 3)], acc);
+    __syncwarp();   // stage st read by every lane before it is refilled
+    cc = cn;
+    vc = vn;
+  }
+  const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  for (int64_t k = nch * 128 + t; k < nnz; k += nthr)
+    acc = __fmaf_rn(ld_stream(A.val + k, ps), ld_x(A.x + ld_stream(A.col + k, ps), px), acc);
+  for (int64_t i = t; i < A.n_rows; i += nthr) out[i] = acc + (float)__ldg(A.row_ptr + i + (i == A.n_rows - 1));
+}
+
+static PFN_cuTensorMapEncodeTiled_v12000 spmv_tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+    cudaGetLastError();
+  }
+  return fn;
+}
+
 }  // namespace dysel
 
 using namespace dysel;
@@ -1001,7 +1100,7 @@ extern "C" {
 
 dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *pl, int flavour, const float *d_x, float *d_out,
                                      void *stream) {
-  if (!ctx || !pl || (flavour != 0 && flavour != 1) || (pl->dev.n_rows > 0 && !d_out) ||
+  if (!ctx || !pl || flavour < 0 || flavour > 3 || (pl->dev.n_rows > 0 && !d_out) ||
       (pl->info.nnz > 0 && !d_x)) {
     set_error(ctx, "dysel_spmv_gather_probe: invalid arguments");
     return DYSEL_ERR_INVALID;
@@ -1014,6 +1113,50 @@ dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *pl, int fl
   cudaStream_t st = (cudaStream_t)stream;
   SpmvDev A = pl->dev;
   A.x = d_x;
+  if (flavour >= 2) {
+    if ((uintptr_t)d_x & 15) {
+      set_error(ctx, "dysel_spmv_gather_probe: x not 16-byte aligned (TMA)");
+      return DYSEL_ERR_UNSUPPORTED;
+    }
+    auto enc = spmv_tensor_map_encoder();
+    CUtensorMap tm;
+    const cuuint64_t dims[2] = {4, (cuuint64_t)((pl->dev.n_cols + 3) / 4)};
+    const cuuint64_t strides[1] = {16};
+    const cuuint32_t box[2] = {4, 1};
+    const cuuint32_t estr[2] = {1, 1};
+    if (!enc || enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)d_x, dims, strides, box, estr,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      set_error(ctx, "dysel_spmv_gather_probe: tensor map encode failed");
+      return DYSEL_ERR_CUDA;
+    }
+    const size_t smem = sizeof(G4Smem);
+    const void *kfn = flavour == 3 ? (const void *)spmv_gather4_probe_kernel<true>
+                                   : (const void *)spmv_gather4_probe_kernel<false>;
+    DYSEL_CUDA_TRY(ctx, cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int occ2 = 0;
+    DYSEL_CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, kfn, kUnitRows, smem));
+    uint32_t *d_err = nullptr;
+    DYSEL_CUDA_TRY(ctx, cudaMallocAsync(&d_err, 4, st));
+    DYSEL_CUDA_TRY(ctx, cudaMemsetAsync(d_err, 0, 4, st));
+    const unsigned g4 = (unsigned)std::max(1, occ2) * (unsigned)ctx->n_sm;
+    if (flavour == 3)
+      spmv_gather4_probe_kernel<true><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
+    else
+      spmv_gather4_probe_kernel<false><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
+    dysel_status ls = check_launch(ctx, "spmv_gather4_probe_kernel");
+    uint32_t h_err = 0;
+    DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&h_err, d_err, 4, cudaMemcpyDeviceToHost, st));
+    DYSEL_CUDA_TRY(ctx, cudaFreeAsync(d_err, st));
+    DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+    if (ls != DYSEL_OK) return ls;
+    if (h_err) {
+      set_error(ctx, (h_err & 1u) ? "dysel_spmv_gather_probe: gather4 transfer never completed (bounded wait)"
+                                  : "dysel_spmv_gather_probe: gather4 delivered values != x[col]");
+      return DYSEL_ERR_CUDA;
+    }
+    return DYSEL_OK;
+  }
   int occ = 0;
   if (flavour == 0)
     DYSEL_CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, spmv_gather_probe_kernel<0>, kUnitRows, 0));

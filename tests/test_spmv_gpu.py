@@ -392,13 +392,13 @@ def test_gather_probe_runs_and_validates(ctx, D):
     A = MATS["powerlaw"]()
     plan = prepared(ctx, A)
     x = vec(uniform_f32(5, A.n_cols))
-    for fl in (0, 1):
+    for fl in (0, 1, 2, 3):   # 3: TMA gather4 values checked against x[col] on the device
         out = torch.full((A.n_rows,), float("nan"), device="cuda")
         ctx.spmv_gather_probe(plan, fl, x, out)
         torch.cuda.synchronize()
         assert bool(torch.isfinite(out).all())
     with pytest.raises(Exception):
-        ctx.spmv_gather_probe(plan, 2, x, out)
+        ctx.spmv_gather_probe(plan, 4, x, out)
     plan.destroy()
 
 
