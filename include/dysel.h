@@ -360,7 +360,8 @@ dysel_status dysel_spmv_variant(dysel_ctx *ctx, dysel_spmv_plan *plan, int varia
  * streamed once (128-bit), x gathered at col (flavour 0) or read sequentially
  * (flavour 1) or gathered by the TMA unit (flavour 2: cp.async.bulk.tensor
  * tile::gather4 into shared memory; flavour 3 = 2 + a check that every
- * gathered value equals x[col], DYSEL_ERR_CUDA if not; flavours 2/3 need a
+ * gathered value equals x[col], DYSEL_ERR_CUDA if not; flavour 4: a quarter of
+ * the chunks through the TMA unit, the rest through the LSU; flavours 2-4 need a
  * 16-byte aligned x and synchronise `stream`), one fma per nonzero, row_ptr read and d_out [n_rows] written
  * once -- with no row structure.  Its duration is the practical floor the
  * variant kernels are judged against (SURVEY §8d roofline);

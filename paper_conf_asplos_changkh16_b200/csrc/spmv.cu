@@ -1006,7 +1006,11 @@ struct G4Smem {
   float buf[kG4Warps][2][32][32];   // warp, stage, lane: 128-byte slot (4 rows x 16 B used)
   unsigned long long bar[kG4Warps][2];
 };
-template <bool VERIFY>
+// HYBRID (flavour 4): warps 0-1 of each CTA gather the first quarter of the
+// chunks through the TMA unit, warps 2-7 the rest through the LSU (both gather
+// engines at once).
+constexpr int kG4TmaWarps = 2;
+template <bool VERIFY, bool HYBRID>
 __global__ void __launch_bounds__(kUnitRows) spmv_gather4_probe_kernel(const __grid_constant__ CUtensorMap tmX,
                                                                       SpmvDev A, float *out, int64_t nnz,
                                                                       uint32_t *err) {
@@ -1019,9 +1023,35 @@ __global__ void __launch_bounds__(kUnitRows) spmv_gather4_probe_kernel(const __g
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncwarp();
   uint32_t phase[2] = {0u, 0u};
-  const int64_t nch = nnz / 128;
-  const int64_t nw = (int64_t)gridDim.x * kG4Warps;
-  const int64_t gw = (int64_t)blockIdx.x * kG4Warps + w;
+  const int64_t nch_all = nnz / 128;
+  const int64_t nch = HYBRID ? nch_all / 4 : nch_all;   // TMA chunks [0, nch)
+  const int64_t nw = (int64_t)gridDim.x * (HYBRID ? kG4TmaWarps : kG4Warps);
+  const int64_t gw = (int64_t)blockIdx.x * (HYBRID ? kG4TmaWarps : kG4Warps) + w;
+  float acc = 0.0f;
+  if (HYBRID && w >= kG4TmaWarps) {   // LSU warps: chunks [nch, nch_all), two in flight
+    const int64_t nl = (int64_t)gridDim.x * (kG4Warps - kG4TmaWarps);
+    for (int64_t ch = nch + (int64_t)blockIdx.x * (kG4Warps - kG4TmaWarps) + (w - kG4TmaWarps); ch < nch_all;
+         ch += 2 * nl) {
+      const int64_t ch1 = ch + nl;
+      const bool h1 = ch1 < nch_all;
+      const int4 c0 = ld_stream4(A.col + ch * 128 + 4 * lane, ps);
+      const float4 v0 = ld_stream4(A.val + ch * 128 + 4 * lane, ps);
+      const int4 c1 = h1 ? ld_stream4(A.col + ch1 * 128 + 4 * lane, ps) : make_int4(0, 0, 0, 0);
+      const float4 v1 = h1 ? ld_stream4(A.val + ch1 * 128 + 4 * lane, ps) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float x0 = ld_x(A.x + c0.x, px), x1 = ld_x(A.x + c0.y, px), x2 = ld_x(A.x + c0.z, px),
+                  x3 = ld_x(A.x + c0.w, px);
+      const float z0 = ld_x(A.x + c1.x, px), z1 = ld_x(A.x + c1.y, px), z2 = ld_x(A.x + c1.z, px),
+                  z3 = ld_x(A.x + c1.w, px);
+      acc = __fmaf_rn(v0.x, x0, acc);
+      acc = __fmaf_rn(v0.y, x1, acc);
+      acc = __fmaf_rn(v0.z, x2, acc);
+      acc = __fmaf_rn(v0.w, x3, acc);
+      acc = __fmaf_rn(v1.x, z0, acc);
+      acc = __fmaf_rn(v1.y, z1, acc);
+      acc = __fmaf_rn(v1.z, z2, acc);
+      acc = __fmaf_rn(v1.w, z3, acc);
+    }
+  }
   auto issue = [&](int64_t ch, int st, int4 &c, float4 &v) {
     const int64_t k = ch * 128 + 4 * lane;
     c = ld_stream4(A.col + k, ps);
@@ -1038,12 +1068,11 @@ __global__ void __launch_bounds__(kUnitRows) spmv_gather4_probe_kernel(const __g
         "l"(&tmX), "r"(bar), "r"(0), "r"(c.x >> 2), "r"(c.y >> 2), "r"(c.z >> 2), "r"(c.w >> 2), "l"(px)
         : "memory");
   };
-  float acc = 0.0f;
   int4 cc = make_int4(0, 0, 0, 0), cn = cc;
   float4 vc = make_float4(0.f, 0.f, 0.f, 0.f), vn = vc;
   int st = 0;
-  if (gw < nch) issue(gw, 0, cc, vc);
-  for (int64_t ch = gw; ch < nch; ch += nw, st ^= 1) {
+  if ((!HYBRID || w < kG4TmaWarps) && gw < nch) issue(gw, 0, cc, vc);
+  for (int64_t ch = (!HYBRID || w < kG4TmaWarps) ? gw : nch; ch < nch; ch += nw, st ^= 1) {
     if (ch + nw < nch) issue(ch + nw, st ^ 1, cn, vn);
     const uint32_t bar = spmv_smem_u32(&S.bar[w][st]);
     uint32_t ok = 0;
@@ -1074,7 +1103,7 @@ __global__ void __launch_bounds__(kUnitRows) spmv_gather4_probe_kernel(const __g
   }
   const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
   const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  for (int64_t k = nch * 128 + t; k < nnz; k += nthr)
+  for (int64_t k = nch_all * 128 + t; k < nnz; k += nthr)
     acc = __fmaf_rn(ld_stream(A.val + k, ps), ld_x(A.x + ld_stream(A.col + k, ps), px), acc);
   for (int64_t i = t; i < A.n_rows; i += nthr) out[i] = acc + (float)__ldg(A.row_ptr + i + (i == A.n_rows - 1));
 }
@@ -1100,7 +1129,7 @@ extern "C" {
 
 dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *pl, int flavour, const float *d_x, float *d_out,
                                      void *stream) {
-  if (!ctx || !pl || flavour < 0 || flavour > 3 || (pl->dev.n_rows > 0 && !d_out) ||
+  if (!ctx || !pl || flavour < 0 || flavour > 4 || (pl->dev.n_rows > 0 && !d_out) ||
       (pl->info.nnz > 0 && !d_x)) {
     set_error(ctx, "dysel_spmv_gather_probe: invalid arguments");
     return DYSEL_ERR_INVALID;
@@ -1131,8 +1160,9 @@ dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *pl, int fl
       return DYSEL_ERR_CUDA;
     }
     const size_t smem = sizeof(G4Smem);
-    const void *kfn = flavour == 3 ? (const void *)spmv_gather4_probe_kernel<true>
-                                   : (const void *)spmv_gather4_probe_kernel<false>;
+    const void *kfn = flavour == 3   ? (const void *)spmv_gather4_probe_kernel<true, false>
+                      : flavour == 4 ? (const void *)spmv_gather4_probe_kernel<false, true>
+                                     : (const void *)spmv_gather4_probe_kernel<false, false>;
     DYSEL_CUDA_TRY(ctx, cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int occ2 = 0;
     DYSEL_CUDA_TRY(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, kfn, kUnitRows, smem));
@@ -1141,9 +1171,11 @@ dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *pl, int fl
     DYSEL_CUDA_TRY(ctx, cudaMemsetAsync(d_err, 0, 4, st));
     const unsigned g4 = (unsigned)std::max(1, occ2) * (unsigned)ctx->n_sm;
     if (flavour == 3)
-      spmv_gather4_probe_kernel<true><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
+      spmv_gather4_probe_kernel<true, false><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
+    else if (flavour == 4)
+      spmv_gather4_probe_kernel<false, true><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
     else
-      spmv_gather4_probe_kernel<false><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
+      spmv_gather4_probe_kernel<false, false><<<g4, kUnitRows, smem, st>>>(tm, A, d_out, (int64_t)pl->info.nnz, d_err);
     dysel_status ls = check_launch(ctx, "spmv_gather4_probe_kernel");
     uint32_t h_err = 0;
     DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&h_err, d_err, 4, cudaMemcpyDeviceToHost, st));

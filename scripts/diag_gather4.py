@@ -26,7 +26,7 @@ def one(fl):
     b.record(s)
     torch.cuda.synchronize()
     return a.elapsed_time(b) * 1e3
-for fl in (0, 2, 0, 2, 1):
+for fl in (0, 2, 4, 0, 2, 4, 1):
     try:
         ts = sorted(one(fl) for _ in range(7))
         print(f"flavour {fl}: median {ts[3]:.1f} us (min {ts[0]:.1f})", flush=True)
