@@ -215,7 +215,13 @@ struct SandboxPoll {
 
 // resident CTAs per SM each plain variant kernel is compiled for (register cap)
 // (CSR-V at 6/SM spills and measured slower on D4: 1.44 vs 1.35 ms)
-constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 8, 6, 5, 3};
+#ifndef DYSEL_ELL_MINB
+#define DYSEL_ELL_MINB 4
+#endif
+#ifndef DYSEL_ELL_CLAIM_MINB
+#define DYSEL_ELL_CLAIM_MINB 4
+#endif
+constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, DYSEL_ELL_MINB, 6, 5, 3};
 constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
 // dynamic shared memory of each variant's kernels (CSR-T's staging buffers)
 __host__ __device__ constexpr size_t dyn_smem(int vid) { return vid == DYSEL_SPMV_CSR_TMA ? sizeof(TmaStageBufs) : 0; }
@@ -225,7 +231,7 @@ inline size_t pool_dyn_smem(const ProfParams &p) {
   return b;
 }
 // claim kernels: CTAs per SM (CSR-S / ELL at 8 spilled ~200 B in the claim loop)
-constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {6, 4, 6, 6, 5, 3};
+constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {6, 4, DYSEL_ELL_CLAIM_MINB, 6, 5, 3};
 
 // Plain kernel of one variant over a slice: the exhaustive oracle's pure
 // version, the activation-flag-off path, the tail-launched remainder, the

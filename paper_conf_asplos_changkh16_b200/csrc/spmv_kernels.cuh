@@ -33,7 +33,11 @@ namespace dysel {
 constexpr int kUnitRows = 256;
 constexpr int kVecMin = 128;   // CSR-V: rows at least this long use 128-bit loads
 constexpr int kRowBatch = 4;   // CSR-V: rows in flight per warp
-constexpr int kChunk = 8;      // CSR-S / ELL / JDS: entries per thread in flight
+constexpr int kChunk = 8;      // CSR-S / JDS: entries per thread in flight
+#ifndef DYSEL_ELL_CHUNK
+#define DYSEL_ELL_CHUNK 16
+#endif
+constexpr int kEllChunk = DYSEL_ELL_CHUNK;   // ELL: slots per thread in flight
 constexpr int kStreamUnroll = 4;   // CSR-W: 32-entry chunks in flight per warp
 #ifndef DYSEL_STREAM_LONG
 #define DYSEL_STREAM_LONG 512
@@ -270,22 +274,22 @@ __device__ __forceinline__ void unit_ell(const SpmvDev &A, uint32_t j, int w, fl
   const float *vp = A.ell_val + r;
   const int W = A.ell_W;
   float s = 0.0f;
-  for (int k = 0; k < W; k += kChunk) {
-    int c[kChunk];
-    float v[kChunk], xv[kChunk];
+  for (int k = 0; k < W; k += kEllChunk) {
+    int c[kEllChunk];
+    float v[kEllChunk], xv[kEllChunk];
 #pragma unroll
-    for (int u = 0; u < kChunk; ++u) {
+    for (int u = 0; u < kEllChunk; ++u) {
       const bool ok = k + u < W;
       c[u] = ok ? ld_stream(cp + (int64_t)(k + u) * A.n_pad, ps) : -1;
       v[u] = ok ? ld_stream(vp + (int64_t)(k + u) * A.n_pad, ps) : 0.0f;
     }
 #pragma unroll
-    for (int u = 0; u < kChunk; ++u) xv[u] = c[u] >= 0 ? ld_x(A.x + c[u], px) : 0.0f;
+    for (int u = 0; u < kEllChunk; ++u) xv[u] = c[u] >= 0 ? ld_x(A.x + c[u], px) : 0.0f;
 #pragma unroll
-    for (int u = 0; u < kChunk; ++u)
+    for (int u = 0; u < kEllChunk; ++u)
       if (c[u] >= 0) s = __fmaf_rn(v[u], xv[u], s);
-    if (c[kChunk - 1] < 0) break;
-    if (Poll::active && (k & 63) >= 64 - kChunk && poll()) break;
+    if (c[kEllChunk - 1] < 0) break;
+    if (Poll::active && (k & 63) >= 64 - kEllChunk && poll()) break;
   }
   out[i] = s;
 }

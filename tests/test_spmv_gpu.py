@@ -385,20 +385,20 @@ def test_csr_tma_multi_slot(ctx, D, name):
 
 
 def test_gather_probe_runs_and_validates(ctx, D):
-    """dysel_spmv_gather_probe (measurement only): both flavours
+    """dysel_spmv_gather_probe (measurement only): every flavour
     run on an aligned plan and write every one of d_out's n_rows floats; a bad
     flavour is rejected with DYSEL_ERR_INVALID."""
     import torch
     A = MATS["powerlaw"]()
     plan = prepared(ctx, A)
     x = vec(uniform_f32(5, A.n_cols))
-    for fl in (0, 1, 2, 3):   # 3: TMA gather4 values checked against x[col] on the device
+    for fl in (0, 1, 2, 3, 4):   # 3: TMA gather4 values checked against x[col] on the device
         out = torch.full((A.n_rows,), float("nan"), device="cuda")
         ctx.spmv_gather_probe(plan, fl, x, out)
         torch.cuda.synchronize()
         assert bool(torch.isfinite(out).all())
     with pytest.raises(Exception):
-        ctx.spmv_gather_probe(plan, 4, x, out)
+        ctx.spmv_gather_probe(plan, 5, x, out)
     plan.destroy()
 
 
