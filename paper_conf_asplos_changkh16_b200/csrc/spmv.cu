@@ -221,7 +221,13 @@ struct SandboxPoll {
 #ifndef DYSEL_ELL_CLAIM_MINB
 #define DYSEL_ELL_CLAIM_MINB 4
 #endif
-constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, DYSEL_ELL_MINB, 6, 5, 3};
+#ifndef DYSEL_SJ_MINB
+#define DYSEL_SJ_MINB 8
+#endif
+#ifndef DYSEL_SJ_CLAIM_MINB
+#define DYSEL_SJ_CLAIM_MINB 6
+#endif
+constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {DYSEL_SJ_MINB, 4, DYSEL_ELL_MINB, (DYSEL_SJ_MINB < 6 ? DYSEL_SJ_MINB : 6), 5, 3};
 constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
 // dynamic shared memory of each variant's kernels (CSR-T's staging buffers)
 __host__ __device__ constexpr size_t dyn_smem(int vid) { return vid == DYSEL_SPMV_CSR_TMA ? sizeof(TmaStageBufs) : 0; }
@@ -231,7 +237,7 @@ inline size_t pool_dyn_smem(const ProfParams &p) {
   return b;
 }
 // claim kernels: CTAs per SM (CSR-S / ELL at 8 spilled ~200 B in the claim loop)
-constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {6, 4, DYSEL_ELL_CLAIM_MINB, 6, 5, 3};
+constexpr int kClaimMinBlocks[DYSEL_SPMV_NVARIANTS] = {DYSEL_SJ_CLAIM_MINB, 4, DYSEL_ELL_CLAIM_MINB, DYSEL_SJ_CLAIM_MINB, 5, 3};
 
 // Plain kernel of one variant over a slice: the exhaustive oracle's pure
 // version, the activation-flag-off path, the tail-launched remainder, the

@@ -33,7 +33,10 @@ namespace dysel {
 constexpr int kUnitRows = 256;
 constexpr int kVecMin = 128;   // CSR-V: rows at least this long use 128-bit loads
 constexpr int kRowBatch = 4;   // CSR-V: rows in flight per warp
-constexpr int kChunk = 8;      // CSR-S / JDS: entries per thread in flight
+#ifndef DYSEL_CHUNK
+#define DYSEL_CHUNK 8
+#endif
+constexpr int kChunk = DYSEL_CHUNK;   // CSR-S / JDS: entries per thread in flight
 #ifndef DYSEL_ELL_CHUNK
 #define DYSEL_ELL_CHUNK 16
 #endif

@@ -21,7 +21,8 @@ for name, A in (("d3", d3_fem()), ("d6r", d6_random()), ("d6d", d6_diag()), ("fe
     rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
     y = torch.empty(A.n_rows, device="cuda")
     plan = ctx.spmv_prepare(rp, col, val, A.n_cols)
-    if 2 in plan.variant_ids:
-        out.append(f"{name}:ell={b2b(lambda: ctx.spmv_variant(plan, 2, x, y)):.1f}us")
+    for v in (0, 2, 3):
+        if v in plan.variant_ids:
+            out.append(f"{name}:{D.SPMV_NAMES[v]}={b2b(lambda: ctx.spmv_variant(plan, v, x, y)):.1f}us")
     plan.destroy()
 print(os.environ.get("DYSEL_LIB", "default"), " ".join(out), flush=True)
