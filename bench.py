@@ -575,6 +575,11 @@ def secondary_workloads(ctx, D, args, stream):
             ctx.sgemm(Ad, Bd, C, mode=D.NO_PROFILE)
     tam4 = time_b2b(amort4, 2, stream) / I4
     b4 = min(t4, key=t4.get)
+    # the amortised run is 40 back-to-back 4096^3 calls (~25 ms at full power):
+    # compare it with the best variant over the same number of calls, so the
+    # power/clock state of both timed regions matches
+    bv4 = D.SGEMM_NAMES.index(b4)
+    tb4_long = time_b2b(lambda: ctx.sgemm_variant(bv4, Ad, Bd, C), 2 * I4, stream)
     fl4 = 2.0 * M * N * K
     out["sgemm_4096"] = {"best_variant": b4, "best_tflops": round(fl4 / t4[b4] / 1e12, 1),
                          "all_tflops": {k: round(fl4 / v / 1e12, 1) for k, v in t4.items()},
@@ -584,7 +589,9 @@ def secondary_workloads(ctx, D, args, stream):
                          "hybrid_async_overhead_pct": round((th4 / t4[b4] - 1) * 100, 2),
                          "hybrid_async_selected": reph4["selected_name"], "hybrid_async_eager_granules": reph4["eager_units"],
                          "host_async_overhead_pct": round((ta4 / t4[b4] - 1) * 100, 2),
-                         "amortized_overhead_pct": round((tam4 / t4[b4] - 1) * 100, 2),
+                         "amortized_overhead_pct": round((tam4 / tb4_long - 1) * 100, 2),
+                         "amortized_ref": "best variant, %d back-to-back calls (same count as the amortised run)" % (2 * I4),
+                         "amortized_overhead_pct_vs_5_call_best": round((tam4 / t4[b4] - 1) * 100, 2),
                          "tensor_roofline_note": "3xTF32 = 3 tf32 MMAs per fp32 product; ceiling ~ tf32 peak / 3"}
     return out
 
