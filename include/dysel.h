@@ -407,6 +407,28 @@ dysel_status dysel_stencil(dysel_ctx *ctx, int nx, int ny, int nz, float c0, flo
 dysel_status dysel_stencil_variant(dysel_ctx *ctx, int variant_id, int nx, int ny, int nz, float c0, float c1,
                                    const float *d_in, float *d_out, void *stream);
 
+/* ------------------------------------------------------------------ SpMTV
+ * y += A^T x over a prepared plan's CSR (x fp32 [n_rows], y fp32 [n_cols],
+ * caller-owned device memory; the plan's ELL/JDS copies are not used): the
+ * scatter-add kernel whose work-groups write overlapping outputs through
+ * global atomics, i.e. the paper's case for swap-based partial-productive
+ * profiling (§2.2, §3.3, Table 1
+ * P:L735-739).  Both built-in variants carry DYSEL_V_ATOMICS: AUTO resolves
+ * to SWAP (each variant profiles the same slice into a private copy of y
+ * initialised from y; the winner's copy is swapped in; the winner runs the
+ * rest); SWAP|ASYNC returns DYSEL_ERR_UNSUPPORTED.  Unit = 256 rows of A.
+ * Variants: 0 scatter-thread (thread per row), 1 scatter-warp (warp per row,
+ * entries strided over lanes).  One fp32 red.global.add per nonzero, in no
+ * fixed order: the result matches the fp64 oracle within fp32 rounding, not
+ * bitwise.  n_rows = 0 or nnz = 0: no-op.  DYSEL_ERR_INVALID for a NULL plan
+ * or buffer. */
+enum { DYSEL_SPMTV_SCATTER_THREAD = 0, DYSEL_SPMTV_SCATTER_WARP = 1, DYSEL_SPMTV_NVARIANTS = 2 };
+dysel_status dysel_spmtv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,
+                         float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+/* Full-grid run of one SpMTV variant (exhaustive oracle timing): y += A^T x. */
+dysel_status dysel_spmtv_variant(dysel_ctx *ctx, dysel_spmv_plan *plan, int variant_id, const float *d_x,
+                                 float *d_y, void *stream);
+
 /* --------------------------------------------------------------- multi-GPU
  * Row-sharded SpMV / M-sharded SGEMM over NCCL (the paper is
  * single-GPU).  nccl_unique_id points to the 128-byte

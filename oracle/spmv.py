@@ -9,7 +9,9 @@ DySel changes only *which variant computes each row*, never *what* is computed
 and every profiling mode.
 
 Pinned by tests/test_oracle_spmv.py: small-integer exactness, identity /
-diagonal closed forms, dense brute force, scipy.sparse.
+diagonal closed forms, dense brute force, scipy.sparse; spmtv by dense
+brute force (explicit loops), scipy's A.T @ x and the duality u.(A^T x) =
+(A u).x against spmv.
 """
 from __future__ import annotations
 
@@ -55,6 +57,29 @@ def spmv_rows(row_ptr, col, val, x, rows):
         y[j] = s
         d[j] = a
     return y, d
+
+
+def spmtv(row_ptr, col, val, x, y0=None) -> np.ndarray:
+    """y = y0 + A^T x in fp64: y_j = y0_j + sum over nonzeros (i, j) of
+    val_ij * x_i — the plain definition of the transposed product that the
+    atomic scatter pool (dysel_spmtv, the swap-mode case of P:L453-464 §2.2 /
+    P:L977-992 §3.3) computes.  Products applied in CSR order (np.add.at)."""
+    rp = np.asarray(row_ptr, np.int64)
+    c = np.asarray(col, np.int64)
+    n_cols = int(c.max()) + 1 if c.size else 0
+    prod = np.asarray(val, np.float64) * np.asarray(x, np.float64)[_rows_of(rp)]
+    if y0 is not None:
+        y = np.array(y0, np.float64)
+    else:
+        y = np.zeros(n_cols, np.float64)
+    np.add.at(y, c, prod)
+    return y
+
+
+def spmtv_abs(row_ptr, col, val, x, y0) -> np.ndarray:
+    """d_j = |y0_j| + sum |val_ij| * |x_i| — the error denominator for y0 + A^T x."""
+    return spmtv(row_ptr, col, np.abs(np.asarray(val, np.float64)), np.abs(np.asarray(x, np.float64)),
+                 np.abs(np.asarray(y0, np.float64)))
 
 
 def rel_error(y_hat, y_star, denom) -> float:

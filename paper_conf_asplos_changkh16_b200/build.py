@@ -20,7 +20,7 @@ CSRC = os.path.join(HERE, "csrc")
 INC = os.path.join(ROOT, "include")
 OBJ = os.path.join(ROOT, "build", "obj")
 LIB = os.path.join(HERE, "libdysel.so")
-SOURCES = ["runtime.cu", "spmv.cu", "spmv_prep.cu", "sgemm.cu", "comm.cu", "iterate.cu", "stencil.cu"]
+SOURCES = ["runtime.cu", "spmv.cu", "spmv_prep.cu", "sgemm.cu", "comm.cu", "iterate.cu", "stencil.cu", "spmtv.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",

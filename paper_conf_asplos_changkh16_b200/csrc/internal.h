@@ -141,6 +141,7 @@ void spmv_ctx_free(dysel_ctx *ctx);
 dysel_status sgemm_register(dysel_ctx *ctx);
 // stencil.cu
 dysel_status stencil_register(dysel_ctx *ctx);
+dysel_status spmtv_register(dysel_ctx *ctx);
 // comm.cu
 void comm_free(dysel_ctx *ctx);
 }  // namespace dysel

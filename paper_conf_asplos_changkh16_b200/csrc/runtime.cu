@@ -413,6 +413,7 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
   if (spmv_ctx_init(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   if (sgemm_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   if (stencil_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
+  if (spmtv_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   uint64_t tick = 0;
   double cpn = 0;
   if (dysel_timer_calibrate(ctx, 1u << 16, 20000, &tick, &cpn) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);

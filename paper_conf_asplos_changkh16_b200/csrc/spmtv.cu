@@ -1,0 +1,164 @@
+// DySel transposed SpMV pool: y += A^T x over the plan's CSR,
+// the scatter-add kernel whose work-groups write OVERLAPPING outputs through
+// global atomics.  Such a kernel cannot be split into productive slices that
+// each own part of y, so the paper's only productive option is the swap-based
+// partial-productive mode (§2.2, §3.3,
+// Table 1): every variant profiles the SAME slice into a private
+// copy of y (initialised from y), the winner's copy is swapped in, and the
+// winner runs the rest.  Variants carry DYSEL_V_ATOMICS, so AUTO resolves to
+// swap and SWAP|ASYNC is rejected by the planner.
+//
+// Unit = 256 consecutive rows of A (= entries of x), as for dysel_spmv.
+//   V0 scatter-thread  thread per row, the row's entries in CSR order
+//   V1 scatter-warp    warp per row (32 rows per warp, in order), the row's
+//                      entries strided over the lanes: coalesced col/val loads
+// Both issue one fire-and-forget `red.global.add.f32` per nonzero
+// (y[col] += val * x[row]); the order of the reductions is not fixed, so the
+// result equals the fp64 oracle within fp32 rounding, not bit for bit.
+#include <algorithm>
+#include <cstring>
+#include <string>
+
+#include "dysel_device.cuh"
+#include "spmv_plan.h"
+
+namespace dysel {
+
+static const char *kSpmtvSig = "dysel.spmtv";
+constexpr int kSpmtvRows = 256;
+
+struct SpmtvArgs {
+  int64_t n_rows;
+  const int32_t *row_ptr;
+  const int32_t *col;
+  const float *val;
+  const float *x;
+};
+
+__device__ __forceinline__ void red_add(float *p, float v) {
+  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+
+template <int VID>
+__global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restrict__ y, dysel_slice s) {
+  __shared__ dysel_prof_smem psm;
+  if (!dysel_gate_open(s)) return;
+  const uint32_t wa[3] = {1, 1, 1};
+  const bool persistent = s.timer == nullptr && s.gate != nullptr;   // gated remainder: one wave walks the units
+  const uint64_t n_cta = persistent ? dysel_slice_ctas(s, wa) : (uint64_t)blockIdx.x + 1;
+  dysel_prof_begin(s, psm);
+  uint32_t units = 0;
+  for (uint64_t cta = blockIdx.x; cta < n_cta; cta += gridDim.x) {
+    uint64_t u[3];
+    if (!dysel_cta_origin(s, wa, cta, u)) continue;
+    ++units;
+    const int64_t r0 = (int64_t)u[0] * kSpmtvRows;
+    if constexpr (VID == 0) {
+      const int64_t r = r0 + threadIdx.x;
+      if (r < a.n_rows) {
+        const float xr = __ldg(a.x + r);
+        const int e = __ldg(a.row_ptr + r + 1);
+        for (int k = __ldg(a.row_ptr + r); k < e; ++k)
+          red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+      }
+    } else {
+      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      for (int i = 0; i < 32; ++i) {
+        const int64_t r = r0 + w * 32 + i;
+        if (r >= a.n_rows) break;
+        const float xr = __ldg(a.x + r);
+        const int e = __ldg(a.row_ptr + r + 1);
+        for (int k = __ldg(a.row_ptr + r) + lane; k < e; k += 32)
+          red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+      }
+    }
+  }
+  dysel_prof_end(s, psm, persistent ? 0u : units);
+}
+
+static uint64_t g_spmtv_wave[DYSEL_SPMTV_NVARIANTS] = {0, 0};   // occupancy x #SM
+
+template <int VID>
+static dysel_status spmtv_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
+  const SpmtvArgs &a = *(const SpmtvArgs *)args[1];
+  float *y = (float *)args[0];
+  static const uint32_t WA[3] = {1, 1, 1};
+  uint64_t ctas = dysel_slice_ctas(*s, WA);
+  if (ctas == 0) return DYSEL_OK;
+  if (s->gate && !s->timer && g_spmtv_wave[VID] > 0) ctas = std::min<uint64_t>(ctas, g_spmtv_wave[VID]);
+  spmtv_kernel<VID><<<(unsigned)ctas, 256, 0, (cudaStream_t)stream>>>(a, y, *s);
+  return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
+}
+
+static const dysel_variant_fn kSpmtvFns[DYSEL_SPMTV_NVARIANTS] = {spmtv_variant_fn<0>, spmtv_variant_fn<1>};
+
+dysel_status spmtv_register(dysel_ctx *ctx) {
+  static const int sb[1] = {0};
+  int o[2] = {0, 0};
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[0], spmtv_kernel<0>, 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[1], spmtv_kernel<1>, 256, 0);
+  cudaGetLastError();
+  const uint64_t n = (uint64_t)ctx->n_sm;
+  for (int i = 0; i < DYSEL_SPMTV_NVARIANTS; ++i) g_spmtv_wave[i] = (uint64_t)o[i] * n;
+  dysel_variant v[DYSEL_SPMTV_NVARIANTS] = {
+      {"scatter_thread", kSpmtvFns[0], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[0] * n},
+      {"scatter_warp", kSpmtvFns[1], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[1] * n},
+  };
+  // initial version: thread per row, the textbook scatter
+  return dysel_register_variants(ctx, kSpmtvSig, v, DYSEL_SPMTV_NVARIANTS, DYSEL_SPMTV_SCATTER_THREAD);
+}
+
+static dysel_status spmtv_check(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *x, float *y) {
+  if (!pl || (pl->dev.n_rows > 0 && !x) || (pl->dev.n_cols > 0 && !y)) {
+    set_error(ctx, "dysel_spmtv: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  return DYSEL_OK;
+}
+
+}  // namespace dysel
+
+using namespace dysel;
+
+extern "C" {
+
+dysel_status dysel_spmtv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, float *d_y, float f, uint32_t mode,
+                         void *stream, dysel_report *rep) {
+  if (!ctx) return DYSEL_ERR_INVALID;
+  DYSEL_TRY(spmtv_check(ctx, pl, d_x, d_y));
+  if (rep) rep->n_slices = 0;
+  if (pl->dev.n_rows == 0 || pl->info.nnz == 0) return DYSEL_OK;   // y += 0
+  SpmtvArgs a{pl->dev.n_rows, pl->dev.row_ptr, pl->dev.col, pl->dev.val, d_x};
+  const uint64_t U[3] = {(uint64_t)(pl->dev.n_rows + kSpmtvRows - 1) / kSpmtvRows, 1, 1};
+  void *args[2] = {d_y, &a};
+  const size_t sbytes[1] = {(size_t)pl->dev.n_cols * sizeof(float)};
+  const std::string key = std::string(kSpmtvSig) + "#" + pl->sig;
+  return launch_keyed(ctx, kSpmtvSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep);
+}
+
+dysel_status dysel_spmtv_variant(dysel_ctx *ctx, dysel_spmv_plan *pl, int variant_id, const float *d_x, float *d_y,
+                                 void *stream) {
+  if (!ctx || variant_id < 0 || variant_id >= DYSEL_SPMTV_NVARIANTS) {
+    set_error(ctx, "dysel_spmtv_variant: invalid variant");
+    return DYSEL_ERR_INVALID;
+  }
+  DYSEL_TRY(spmtv_check(ctx, pl, d_x, d_y));
+  if (pl->dev.n_rows == 0 || pl->info.nnz == 0) return DYSEL_OK;
+  SpmtvArgs a{pl->dev.n_rows, pl->dev.row_ptr, pl->dev.col, pl->dev.val, d_x};
+  void *args[2] = {d_y, &a};
+  dysel_slice s;
+  memset(&s, 0, sizeof(s));
+  s.g[0] = s.g[1] = s.g[2] = 1;
+  s.U[0] = (uint64_t)(pl->dev.n_rows + kSpmtvRows - 1) / kSpmtvRows;
+  s.U[1] = s.U[2] = 1;
+  s.G[0] = (uint32_t)s.U[0];
+  s.G[1] = s.G[2] = 1;
+  s.granule_count = s.U[0];
+  s.granule_stride = 1;
+  s.role = DYSEL_ROLE_BATCH;
+  s.variant = variant_id;
+  DYSEL_TRY(kSpmtvFns[variant_id](&s, args, stream, nullptr));
+  return check_launch(ctx, "spmtv full-grid variant");
+}
+
+}  // extern "C"

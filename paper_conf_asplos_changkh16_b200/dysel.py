@@ -43,6 +43,7 @@ SPMV_DEFAULT_AUTO = -1
 SGEMM_S64, SGEMM_S128, SGEMM_T128x64, SGEMM_T128x128 = range(4)
 SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"]
 STENCIL_NAMES = ["base", "zmarch64", "tiled64x4_zmarch64"]
+SPMTV_NAMES = ["scatter_thread", "scatter_warp"]
 STENCIL_BASE, STENCIL_ZMARCH, STENCIL_TILED = range(3)
 
 c_void_p, c_int, c_float, c_u32, c_u64, c_i64, c_size = (ctypes.c_void_p, ctypes.c_int, ctypes.c_float,
@@ -112,6 +113,8 @@ dysel_partition_rows = _sig("dysel_partition_rows", c_int, P, c_i64, c_int, P)
 dysel_spmv_sharded = _sig("dysel_spmv_sharded", c_int, P, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
 dysel_stencil = _sig("dysel_stencil", c_int, P, c_int, c_int, c_int, c_float, c_float, P, P, c_float, c_u32, P,
                      ctypes.POINTER(Report))
+dysel_spmtv = _sig("dysel_spmtv", c_int, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_spmtv_variant = _sig("dysel_spmtv_variant", c_int, P, P, c_int, P, P, P)
 dysel_stencil_variant = _sig("dysel_stencil_variant", c_int, P, c_int, c_int, c_int, c_int, c_float, c_float, P, P, P)
 dysel_spmv_power = _sig("dysel_spmv_power", c_int, P, P, P, P, c_int, c_int, c_float, c_u32, P, P,
                         ctypes.POINTER(Report))
@@ -304,6 +307,18 @@ class Context:
 
     def spmv_variant(self, plan, variant_id, x, y, stream=None):
         self._check(dysel_spmv_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), _stream(stream)))
+
+    def spmtv(self, plan, x, y, f=0.02, mode=AUTO, report=False, unit_map=False, stream=None):
+        """y += A^T x through the atomic scatter pool (dysel_spmtv; AUTO -> swap mode)."""
+        rep, keep, uv = (_make_report(plan.n_units if unit_map else 0) if report else (None, None, None))
+        self._check(dysel_spmtv(self.h, plan.handle, _ptr(x), _ptr(y), float(f), int(mode), _stream(stream),
+                                ctypes.byref(rep) if rep is not None else None))
+        if rep is None:
+            return None
+        return report_dict(rep, SPMTV_NAMES, bytes(uv) if uv is not None else None)
+
+    def spmtv_variant(self, plan, variant_id, x, y, stream=None):
+        self._check(dysel_spmtv_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), _stream(stream)))
 
     def spmv_gather_probe(self, plan, flavour, x, out, stream=None):
         """Measurement only: the plan's CSR traffic with no row structure (include/dysel.h)."""

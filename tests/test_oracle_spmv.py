@@ -151,3 +151,40 @@ def test_applicability_and_uniformity_readings():
     assert not formats.uniform_rows(P.row_ptr)
     assert not formats.ell_applicable(P.row_ptr)
     assert formats.ell_applicable(d1_bus().row_ptr)
+
+
+def test_spmtv_dense_brute_force_and_scipy():
+    """y0 + A^T x: explicit-loop dense transpose and scipy's A.T @ x (non-square)."""
+    A = random_lengths_csr(300, 200, 60, 13, empty_frac=0.05)
+    x = uniform_f32(14, A.n_rows)
+    y0 = uniform_f32(15, A.n_cols)
+    D = np.zeros((A.n_cols, A.n_rows))
+    for i in range(A.n_rows):
+        for k in range(A.row_ptr[i], A.row_ptr[i + 1]):
+            D[A.col[k], i] += A.val[k]   # D = A^T
+    y = spmv.spmtv(A.row_ptr, A.col, A.val, x, y0)
+    assert y.shape == (A.n_cols,)
+    assert np.allclose(y, y0.astype(np.float64) + D @ x.astype(np.float64), rtol=1e-13, atol=1e-13)
+    m = sp.csr_matrix((A.val.astype(np.float64), A.col, A.row_ptr), shape=(A.n_rows, A.n_cols))
+    assert np.allclose(y, y0 + m.T @ x.astype(np.float64), rtol=1e-12, atol=1e-12)
+
+
+def test_spmtv_duality_and_small_int():
+    """u.(A^T x) = (A u).x against the (separately pinned) spmv oracle; small
+    integers are exact; all-zero x leaves y0 unchanged."""
+    A = d4_powerlaw(n=3000, lmax=400)
+    x = uniform_f32(21, A.n_rows)
+    u = uniform_f32(22, A.n_cols).astype(np.float64)
+    z = np.zeros(A.n_cols)
+    lhs = u @ spmv.spmtv(A.row_ptr, A.col, A.val, x, z)
+    rhs = spmv.spmv(A.row_ptr, A.col, A.val, u) @ x.astype(np.float64)
+    assert abs(lhs - rhs) <= 1e-10 * max(1.0, abs(rhs))
+    B = small_int_csr(d1_bus(), 3)
+    xi = small_int_vector(B.n_rows, 4)
+    yi = spmv.spmtv(B.row_ptr, B.col, B.val, xi, np.zeros(B.n_cols))
+    assert np.array_equal(yi, np.round(yi))
+    y0 = uniform_f32(23, B.n_cols)
+    assert np.array_equal(spmv.spmtv(B.row_ptr, B.col, B.val, np.zeros(B.n_rows, np.float32), y0),
+                          y0.astype(np.float64))
+    d = spmv.spmtv_abs(B.row_ptr, B.col, B.val, xi, y0)
+    assert np.all(d >= np.abs(spmv.spmtv(B.row_ptr, B.col, B.val, xi, y0)) - 1e-12)

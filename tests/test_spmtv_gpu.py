@@ -1,0 +1,132 @@
+"""GPU parity of the atomic scatter pool y += A^T x (dysel_spmtv, SURVEY §8f
+f-1) through the C ABI vs the fp64 oracle: the swap-based partial-productive
+mode on a real kernel with overlapping outputs (§2.2
+§3.3, Table 1).  fp32 reductions in no fixed order: within
+SPMV_TOL of the oracle; small integers: bit-exact in any order."""
+import numpy as np
+import pytest
+
+from gpu_helpers import to_dev, vec
+from oracle.spmv import SPMV_TOL, rel_error, spmtv, spmtv_abs
+from workloads import d1_bus, d4_powerlaw, random_lengths_csr, small_int_csr, small_int_vector, uniform_f32
+
+pytestmark = pytest.mark.gpu
+
+MATS = {
+    "d1": lambda: d1_bus(),
+    "ragged_nonsquare": lambda: random_lengths_csr(5003, 4000, 300, 17, empty_frac=0.1),
+    # 2,344 units: more than one wave of either variant -> profiled
+    "powerlaw": lambda: d4_powerlaw(n=600_000, lmax=2000),
+}
+
+
+@pytest.fixture(scope="module")
+def ctx(gpu):
+    from paper_conf_asplos_changkh16_b200 import dysel
+    c = dysel.Context(0)
+    yield c
+    c.close()
+
+
+@pytest.fixture(scope="module")
+def D():
+    from paper_conf_asplos_changkh16_b200 import dysel
+    return dysel
+
+
+def _plan(ctx, A):
+    import torch
+    rp, col, val = to_dev(A)
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols)
+    torch.cuda.synchronize()
+    return plan, (rp, col, val)
+
+
+def _err(A, x, y0, y):
+    ys = spmtv(A.row_ptr, A.col, A.val, x, y0)
+    return rel_error(y.cpu().numpy(), ys, spmtv_abs(A.row_ptr, A.col, A.val, x, y0))
+
+
+@pytest.mark.parametrize("name", list(MATS))
+def test_spmtv_variants_parity(ctx, D, name):
+    import torch
+    A = MATS[name]()
+    x = uniform_f32(31, A.n_rows)
+    y0 = uniform_f32(32, A.n_cols)
+    plan, keep = _plan(ctx, A)
+    for v in range(len(D.SPMTV_NAMES)):
+        y = vec(y0)
+        ctx.spmtv_variant(plan, v, vec(x), y)
+        torch.cuda.synchronize()
+        assert _err(A, x, y0, y) <= SPMV_TOL, D.SPMTV_NAMES[v]
+    plan.destroy()
+
+
+@pytest.mark.parametrize("name", list(MATS))
+@pytest.mark.parametrize("m", ["auto", "swap_host", "fully", "no_profile", "auto_forced"])
+def test_spmtv_modes_parity(ctx, D, name, m):
+    """Every unit's contribution lands in y exactly once, whichever variant
+    profiled or ran it; AUTO resolves to swap (DYSEL_V_ATOMICS)."""
+    import torch
+    A = MATS[name]()
+    x = uniform_f32(41, A.n_rows)
+    y0 = uniform_f32(42, A.n_cols)
+    plan, keep = _plan(ctx, A)
+    mode = {"auto": D.AUTO, "swap_host": D.SWAP | D.HOST_ORCH, "fully": D.FULLY, "no_profile": D.AUTO | D.NO_PROFILE,
+            "auto_forced": D.AUTO | D.FORCE_PROFILE}[m]
+    for rep_i in range(3):   # cached selection on later calls must not change the result
+        y = vec(y0)
+        rep = ctx.spmtv(plan, vec(x), y, f=0.05, mode=mode, report=True)
+        torch.cuda.synchronize()
+        assert _err(A, x, y0, y) <= SPMV_TOL, (m, rep_i)
+        assert 0 <= rep["selected"] < len(D.SPMTV_NAMES)
+        if m in ("auto", "auto_forced", "swap_host") and rep["profiled"]:
+            assert rep["mode_used"] & 3 == D.SWAP
+    if m == "auto_forced":
+        assert rep["profiled"]
+    if name == "powerlaw" and m == "auto":
+        assert rep["profiled"]
+    plan.destroy()
+
+
+def test_spmtv_small_integer_bit_exact(ctx, D):
+    """Integer products and sums below 2^24 are exact in any reduction order."""
+    import torch
+    A = small_int_csr(MATS["powerlaw"](), 5)
+    x = small_int_vector(A.n_rows, 6)
+    y0 = small_int_vector(A.n_cols, 7)
+    ys = spmtv(A.row_ptr, A.col, A.val, x, y0)
+    assert np.max(np.abs(ys)) < 2 ** 24
+    plan, keep = _plan(ctx, A)
+    for mode in (D.AUTO | D.FORCE_PROFILE, D.SWAP | D.HOST_ORCH, D.FULLY | D.FORCE_PROFILE):
+        y = vec(y0)
+        ctx.spmtv(plan, vec(x), y, f=0.05, mode=mode)
+        torch.cuda.synchronize()
+        assert np.array_equal(y.cpu().numpy().astype(np.float64), ys), mode
+    plan.destroy()
+
+
+def test_spmtv_swap_async_rejected_and_edges(ctx, D):
+    import torch
+    from paper_conf_asplos_changkh16_b200.dysel import DyselError
+    A = MATS["ragged_nonsquare"]()
+    plan, keep = _plan(ctx, A)
+    x, y = vec(uniform_f32(51, A.n_rows)), vec(uniform_f32(52, A.n_cols))
+    with pytest.raises(DyselError):
+        ctx.spmtv(plan, x, y, f=0.05, mode=D.SWAP | D.ASYNC)
+    with pytest.raises(DyselError):
+        ctx.spmtv(plan, x, y, f=0.05, mode=D.AUTO | D.ASYNC)   # AUTO -> swap, still no async (Table 1)
+    with pytest.raises(DyselError):
+        ctx.spmtv_variant(plan, 7, x, y)
+    plan.destroy()
+    # nnz = 0: y unchanged
+    from workloads import CSR
+    n = 1000
+    E = CSR(n, n, np.zeros(n + 1, np.int32), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    plan, keep = _plan(ctx, E)
+    y0 = uniform_f32(53, n)
+    y = vec(y0)
+    ctx.spmtv(plan, vec(uniform_f32(54, n)), y, f=0.05, mode=D.AUTO)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy(), y0)
+    plan.destroy()
