@@ -524,6 +524,35 @@ def secondary_workloads(ctx, D, args, stream):
                                  "note": "in + out 134 MB > L2; fully|async, f = 0.02 (profiled unless the default's grid fits one "
                                          "wave, A-3b); forced: profile once; amortised: forced once + 19 activation-flag "
                                          "calls"}
+    # SpMTV (f-1): y += A^T x by atomic scatter -> swap-mode profiling
+    from workloads import d4_powerlaw
+    At = d4_powerlaw(n=2_000_000, lmax=4096)
+    rpt, colt, valt = (torch.from_numpy(a).cuda() for a in (At.row_ptr, At.col, At.val))
+    plant = ctx.spmv_prepare(rpt, colt, valt, At.n_cols)
+    xt = torch.from_numpy(uniform_f32(61, At.n_rows)).cuda()
+    yt = torch.zeros(At.n_cols, device="cuda")
+    tt = {D.SPMTV_NAMES[v]: time_b2b(lambda: ctx.spmtv_variant(plant, v, xt, yt), 20, stream) for v in range(2)}
+    bt = min(tt, key=tt.get)
+    tdt = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO), 20, stream)
+    rept = ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO, report=True)
+    tht = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.SWAP | D.HOST_ORCH), 10, stream)
+    def amortt():
+        ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO)
+        for _ in range(19):
+            ctx.spmtv(plant, xt, yt, mode=D.AUTO | D.NO_PROFILE)
+    tat = time_b2b(amortt, 3, stream) / 20
+    nbt = spmv_bytes(At.n_rows, At.n_cols, At.nnz)
+    out["spmtv_powerlaw_2M"] = {"nnz": int(At.nnz), "best_variant": bt, "best_us": round(tt[bt] * 1e6, 2),
+                                "best_gbs": round(nbt / tt[bt] / 1e9, 1), "dysel_us": round(tdt * 1e6, 2),
+                                "selected": rept["selected_name"], "profiled": rept["profiled"],
+                                "mode_used": rept["mode_used"],
+                                "overhead_pct": round((tdt / tt[bt] - 1) * 100, 2),
+                                "host_orch_overhead_pct": round((tht / tt[bt] - 1) * 100, 2),
+                                "amortized_overhead_pct": round((tat / tt[bt] - 1) * 100, 2),
+                                "all_us": {k: round(v * 1e6, 2) for k, v in tt.items()},
+                                "note": "y += A^T x (red.global.add per nonzero): AUTO -> swap (private copies of y, "
+                                        "winner's swapped in), f = 0.01, sync only (Table 1)"}
+    del plant
     # D2m: Parboil-medium SGEMM 1024 x 992 x 1056
     M, K, N = 1024, 992, 1056
     Ah, Bh, _ = sgemm_inputs(M, K, N)

@@ -728,7 +728,10 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
   }
   if (!host_orch) {
     // ---- device path: gated remainder, selection never leaves the device
-    const bool dominance = !(mode & DYSEL_NO_ABORT) && P.mode != DYSEL_SWAP;
+    // swap too (reading A-44): the winner's private copy is complete when its
+    // last CTA decides it, so the copy-in and the remainder wait for the
+    // selection only, not for a dominated variant's discarded private copy
+    const bool dominance = !(mode & DYSEL_NO_ABORT);
     // the remainder is ordered behind the selection only — not behind the
     // eager wave (its CTAs take the slots the eager ones free) nor, with
     // dominance, behind dominated variants finishing productive tiles

@@ -39,37 +39,61 @@ __device__ __forceinline__ void red_add(float *p, float v) {
   asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
 }
 
+// Dominance (reading A-32) applies to swap too: a dominated variant's
+// PRIVATE copy is discarded, so its CTAs stop at the next poll; the polls are
+// CTA-uniform (dysel_prof_poll holds a barrier).
 template <int VID>
 __global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restrict__ y, dysel_slice s) {
   __shared__ dysel_prof_smem psm;
   if (!dysel_gate_open(s)) return;
   const uint32_t wa[3] = {1, 1, 1};
   const bool persistent = s.timer == nullptr && s.gate != nullptr;   // gated remainder: one wave walks the units
+  const bool timed = s.timer != nullptr;
   const uint64_t n_cta = persistent ? dysel_slice_ctas(s, wa) : (uint64_t)blockIdx.x + 1;
   dysel_prof_begin(s, psm);
   uint32_t units = 0;
-  for (uint64_t cta = blockIdx.x; cta < n_cta; cta += gridDim.x) {
+  bool stop = false;
+  for (uint64_t cta = blockIdx.x; cta < n_cta && !stop; cta += gridDim.x) {
     uint64_t u[3];
     if (!dysel_cta_origin(s, wa, cta, u)) continue;
     ++units;
     const int64_t r0 = (int64_t)u[0] * kSpmtvRows;
-    if constexpr (VID == 0) {
+    if constexpr (VID == 0) {   // thread per row, entries in CSR order
       const int64_t r = r0 + threadIdx.x;
+      int k = 0, e = 0;
+      float xr = 0.0f;
       if (r < a.n_rows) {
-        const float xr = __ldg(a.x + r);
-        const int e = __ldg(a.row_ptr + r + 1);
-        for (int k = __ldg(a.row_ptr + r); k < e; ++k)
-          red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+        xr = __ldg(a.x + r);
+        k = __ldg(a.row_ptr + r);
+        e = __ldg(a.row_ptr + r + 1);
       }
-    } else {
+      if (!timed) {   // batch / remainder copies: no barrier in the row loop
+        for (; k < e; ++k) red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+        continue;
+      }
+      for (int it = 0;; ++it) {   // profiling copy: CTA-uniform chunks so it can poll
+        const int stop_k = min(e, k + 32);
+        for (; k < stop_k; ++k) red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+        if (!__syncthreads_or(k < e)) break;
+        if ((it & 3) == 3 && dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_PRIVATE) {
+          stop = true;
+          break;
+        }
+      }
+    } else {   // warp per row (32 rows per warp, in order), entries strided over the lanes
       const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
       for (int i = 0; i < 32; ++i) {
         const int64_t r = r0 + w * 32 + i;
-        if (r >= a.n_rows) break;
-        const float xr = __ldg(a.x + r);
-        const int e = __ldg(a.row_ptr + r + 1);
-        for (int k = __ldg(a.row_ptr + r) + lane; k < e; k += 32)
-          red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+        if (r < a.n_rows) {
+          const float xr = __ldg(a.x + r);
+          const int e = __ldg(a.row_ptr + r + 1);
+          for (int k = __ldg(a.row_ptr + r) + lane; k < e; k += 32)
+            red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+        }
+        if (timed && (i & 7) == 7 && dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_PRIVATE) {
+          stop = true;
+          break;
+        }
       }
     }
   }
