@@ -531,7 +531,7 @@ def secondary_workloads(ctx, D, args, stream):
     plant = ctx.spmv_prepare(rpt, colt, valt, At.n_cols)
     xt = torch.from_numpy(uniform_f32(61, At.n_rows)).cuda()
     yt = torch.zeros(At.n_cols, device="cuda")
-    tt = {D.SPMTV_NAMES[v]: time_b2b(lambda: ctx.spmtv_variant(plant, v, xt, yt), 20, stream) for v in range(2)}
+    tt = {D.SPMTV_NAMES[v]: time_b2b(lambda: ctx.spmtv_variant(plant, v, xt, yt), 20, stream) for v in range(len(D.SPMTV_NAMES))}
     bt = min(tt, key=tt.get)
     tdt = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO), 20, stream)
     rept = ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO, report=True)

@@ -418,11 +418,13 @@ dysel_status dysel_stencil_variant(dysel_ctx *ctx, int variant_id, int nx, int n
  * initialised from y; the winner's copy is swapped in; the winner runs the
  * rest); SWAP|ASYNC returns DYSEL_ERR_UNSUPPORTED.  Unit = 256 rows of A.
  * Variants: 0 scatter-thread (thread per row), 1 scatter-warp (warp per row,
- * entries strided over lanes).  One fp32 red.global.add per nonzero, in no
+ * entries strided over lanes), 2 scatter-segment (warp per 32-row segment,
+ * its nonzeros as one flat stream).  One fp32 red.global.add per nonzero, in no
  * fixed order: the result matches the fp64 oracle within fp32 rounding, not
  * bitwise.  n_rows = 0 or nnz = 0: no-op.  DYSEL_ERR_INVALID for a NULL plan
  * or buffer. */
-enum { DYSEL_SPMTV_SCATTER_THREAD = 0, DYSEL_SPMTV_SCATTER_WARP = 1, DYSEL_SPMTV_NVARIANTS = 2 };
+enum { DYSEL_SPMTV_SCATTER_THREAD = 0, DYSEL_SPMTV_SCATTER_WARP = 1, DYSEL_SPMTV_SCATTER_SEGMENT = 2,
+       DYSEL_SPMTV_NVARIANTS = 3 };
 dysel_status dysel_spmtv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,
                          float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
 /* Full-grid run of one SpMTV variant (exhaustive oracle timing): y += A^T x. */

@@ -12,10 +12,15 @@
 //   V0 scatter-thread  thread per row, the row's entries in CSR order
 //   V1 scatter-warp    warp per row (32 rows per warp, in order), the row's
 //                      entries strided over the lanes: coalesced col/val loads
+//   V2 scatter-segment warp per 32-row segment: the segment's nonzeros as one
+//                      flat coalesced stream, 4 x 32 entries in flight per
+//                      round, each entry's row found by a 5-step shuffle search
+//                      over the lanes' row ends (no per-row serial chain)
 // Both issue one fire-and-forget `red.global.add.f32` per nonzero
 // (y[col] += val * x[row]); the order of the reductions is not fixed, so the
 // result equals the fp64 oracle within fp32 rounding, not bit for bit.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -37,6 +42,12 @@ struct SpmtvArgs {
 
 __device__ __forceinline__ void red_add(float *p, float v) {
   asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+
+// No memory clobber: lets the compiler batch the next entries' loads ahead of
+// earlier reductions (the kernel never reads y).
+__device__ __forceinline__ void red_add_nc(float *p, float v) {
+  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v));
 }
 
 // Dominance (reading A-32) applies to swap too: a dominated variant's
@@ -80,6 +91,47 @@ __global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restri
           break;
         }
       }
+    } else if constexpr (VID == 2) {   // warp per 32-row segment, its nonzeros as one flat stream
+      const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      const int64_t rw = r0 + w * 32;   // first row of this warp's segment
+      int seg_b = 0, end_l = 0;
+      float xl = 0.0f;
+      if (rw < a.n_rows) {
+        const int64_t rl = min(rw + lane, a.n_rows - 1);
+        seg_b = __ldg(a.row_ptr + rw);
+        end_l = __ldg(a.row_ptr + rl + 1);   // lanes past n_rows repeat the last row's end
+        xl = rw + lane < a.n_rows ? __ldg(a.x + rw + lane) : 0.0f;
+      }
+      const int seg_e = __shfl_sync(0xffffffffu, end_l, 31);
+      int k = seg_b + lane;
+      auto step = [&](int kk) {   // entry kk of the segment: its row by a 5-step shuffle search
+        int pos = 0;
+#pragma unroll
+        for (int st = 16; st > 0; st >>= 1) {
+          const int v = __shfl_sync(0xffffffffu, end_l, pos + st - 1);
+          if (v <= kk) pos += st;
+        }
+        const float xr = __shfl_sync(0xffffffffu, xl, pos);
+        if (kk < seg_e) red_add_nc(y + __ldg(a.col + kk), __fmul_rn(__ldg(a.val + kk), xr));
+      };
+      if (!timed) {
+        for (; __any_sync(0xffffffffu, k < seg_e); k += 128) {
+#pragma unroll
+          for (int u = 0; u < 4; ++u) step(k + 32 * u);
+        }
+        continue;
+      }
+      for (int it = 0;; ++it, k += 128) {   // profiling copy: CTA-uniform rounds so it can poll
+        if (__any_sync(0xffffffffu, k < seg_e)) {
+#pragma unroll
+          for (int u = 0; u < 4; ++u) step(k + 32 * u);
+        }
+        if (!__syncthreads_or(k + 128 < seg_e)) break;
+        if ((it & 3) == 3 && dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_PRIVATE) {
+          stop = true;
+          break;
+        }
+      }
     } else {   // warp per row (32 rows per warp, in order), entries strided over the lanes
       const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
       for (int i = 0; i < 32; ++i) {
@@ -100,7 +152,8 @@ __global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restri
   dysel_prof_end(s, psm, persistent ? 0u : units);
 }
 
-static uint64_t g_spmtv_wave[DYSEL_SPMTV_NVARIANTS] = {0, 0};   // occupancy x #SM
+static uint64_t g_spmtv_wave[DYSEL_SPMTV_NVARIANTS] = {0, 0, 0};   // occupancy x #SM
+static const bool g_spmtv_persistent = getenv("DYSEL_SPMTV_PERSISTENT") != nullptr;   // ablation knob
 
 template <int VID>
 static dysel_status spmtv_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
@@ -109,24 +162,31 @@ static dysel_status spmtv_variant_fn(const dysel_slice *s, void *const *args, vo
   static const uint32_t WA[3] = {1, 1, 1};
   uint64_t ctas = dysel_slice_ctas(*s, WA);
   if (ctas == 0) return DYSEL_OK;
-  if (s->gate && !s->timer && g_spmtv_wave[VID] > 0) ctas = std::min<uint64_t>(ctas, g_spmtv_wave[VID]);
+  // gated remainder: a persistent wave only when asked (DYSEL_SPMTV_PERSISTENT);
+  // by default the full grid, whose CTAs the block scheduler hands out
+  // dynamically — skewed rows make a static round-robin walk imbalanced
+  if (g_spmtv_persistent && s->gate && !s->timer && g_spmtv_wave[VID] > 0)
+    ctas = std::min<uint64_t>(ctas, g_spmtv_wave[VID]);
   spmtv_kernel<VID><<<(unsigned)ctas, 256, 0, (cudaStream_t)stream>>>(a, y, *s);
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
 
-static const dysel_variant_fn kSpmtvFns[DYSEL_SPMTV_NVARIANTS] = {spmtv_variant_fn<0>, spmtv_variant_fn<1>};
+static const dysel_variant_fn kSpmtvFns[DYSEL_SPMTV_NVARIANTS] = {spmtv_variant_fn<0>, spmtv_variant_fn<1>,
+                                                                   spmtv_variant_fn<2>};
 
 dysel_status spmtv_register(dysel_ctx *ctx) {
   static const int sb[1] = {0};
-  int o[2] = {0, 0};
+  int o[3] = {0, 0, 0};
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[0], spmtv_kernel<0>, 256, 0);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[1], spmtv_kernel<1>, 256, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], spmtv_kernel<2>, 256, 0);
   cudaGetLastError();
   const uint64_t n = (uint64_t)ctx->n_sm;
   for (int i = 0; i < DYSEL_SPMTV_NVARIANTS; ++i) g_spmtv_wave[i] = (uint64_t)o[i] * n;
   dysel_variant v[DYSEL_SPMTV_NVARIANTS] = {
       {"scatter_thread", kSpmtvFns[0], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[0] * n},
       {"scatter_warp", kSpmtvFns[1], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[1] * n},
+      {"scatter_segment", kSpmtvFns[2], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[2] * n},
   };
   // initial version: thread per row, the textbook scatter
   return dysel_register_variants(ctx, kSpmtvSig, v, DYSEL_SPMTV_NVARIANTS, DYSEL_SPMTV_SCATTER_THREAD);

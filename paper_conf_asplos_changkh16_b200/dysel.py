@@ -43,7 +43,7 @@ SPMV_DEFAULT_AUTO = -1
 SGEMM_S64, SGEMM_S128, SGEMM_T128x64, SGEMM_T128x128 = range(4)
 SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"]
 STENCIL_NAMES = ["base", "zmarch64", "tiled64x4_zmarch64"]
-SPMTV_NAMES = ["scatter_thread", "scatter_warp"]
+SPMTV_NAMES = ["scatter_thread", "scatter_warp", "scatter_segment"]
 STENCIL_BASE, STENCIL_ZMARCH, STENCIL_TILED = range(3)
 
 c_void_p, c_int, c_float, c_u32, c_u64, c_i64, c_size = (ctypes.c_void_p, ctypes.c_int, ctypes.c_float,
