@@ -40,9 +40,6 @@ struct SpmtvArgs {
   const float *x;
 };
 
-__device__ __forceinline__ void red_add(float *p, float v) {
-  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
-}
 
 // No memory clobber: lets the compiler batch the next entries' loads ahead of
 // earlier reductions (the kernel never reads y).
@@ -79,12 +76,13 @@ __global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restri
         e = __ldg(a.row_ptr + r + 1);
       }
       if (!timed) {   // batch / remainder copies: no barrier in the row loop
-        for (; k < e; ++k) red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+#pragma unroll 4
+        for (; k < e; ++k) red_add_nc(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
         continue;
       }
       for (int it = 0;; ++it) {   // profiling copy: CTA-uniform chunks so it can poll
         const int stop_k = min(e, k + 32);
-        for (; k < stop_k; ++k) red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+        for (; k < stop_k; ++k) red_add_nc(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
         if (!__syncthreads_or(k < e)) break;
         if ((it & 3) == 3 && dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_PRIVATE) {
           stop = true;
@@ -139,8 +137,9 @@ __global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restri
         if (r < a.n_rows) {
           const float xr = __ldg(a.x + r);
           const int e = __ldg(a.row_ptr + r + 1);
+#pragma unroll 4
           for (int k = __ldg(a.row_ptr + r) + lane; k < e; k += 32)
-            red_add(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
+            red_add_nc(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
         }
         if (timed && (i & 7) == 7 && dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_PRIVATE) {
           stop = true;
