@@ -130,3 +130,20 @@ def test_spmtv_swap_async_rejected_and_edges(ctx, D):
     torch.cuda.synchronize()
     assert np.array_equal(y.cpu().numpy(), y0)
     plan.destroy()
+
+
+def test_spmtv_bench_size_parity(ctx, D):
+    """The bench's 2M-row power-law SpMTV (40M nnz) in its launch configuration
+    (AUTO -> swap, f = 0.01, profiled) against the fp64 oracle, every entry."""
+    import torch
+    A = d4_powerlaw(n=2_000_000, lmax=4096)
+    x = uniform_f32(61, A.n_rows)
+    y0 = uniform_f32(62, A.n_cols)
+    plan, keep = _plan(ctx, A)
+    for mode in (D.AUTO, D.AUTO | D.NO_PROFILE):
+        y = vec(y0)
+        rep = ctx.spmtv(plan, vec(x), y, f=0.01, mode=mode, report=True)
+        torch.cuda.synchronize()
+        assert rep["profiled"] == (mode == D.AUTO)
+        assert _err(A, x, y0, y) <= SPMV_TOL, mode
+    plan.destroy()
