@@ -16,7 +16,7 @@
 //                      flat coalesced stream, 4 x 32 entries in flight per
 //                      round, each entry's row found by a 5-step shuffle search
 //                      over the lanes' row ends (no per-row serial chain)
-// Both issue one fire-and-forget `red.global.add.f32` per nonzero
+// All issue one fire-and-forget `red.global.add.f32` per nonzero
 // (y[col] += val * x[row]); the order of the reductions is not fixed, so the
 // result equals the fp64 oracle within fp32 rounding, not bit for bit.
 #include <algorithm>
@@ -132,13 +132,20 @@ __global__ void __launch_bounds__(256) spmtv_kernel(SpmtvArgs a, float *__restri
       }
     } else {   // warp per row (32 rows per warp, in order), entries strided over the lanes
       const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+      const int64_t rl = r0 + w * 32 + lane;   // lane l holds row l's bounds and x: one load level for all 32
+      int beg_l = 0, end_l = 0;
+      float x_l = 0.0f;
+      if (rl < a.n_rows) {
+        beg_l = __ldg(a.row_ptr + rl);
+        end_l = __ldg(a.row_ptr + rl + 1);
+        x_l = __ldg(a.x + rl);
+      }
       for (int i = 0; i < 32; ++i) {
-        const int64_t r = r0 + w * 32 + i;
-        if (r < a.n_rows) {
-          const float xr = __ldg(a.x + r);
-          const int e = __ldg(a.row_ptr + r + 1);
+        {
+          const int b = __shfl_sync(0xffffffffu, beg_l, i), e = __shfl_sync(0xffffffffu, end_l, i);
+          const float xr = __shfl_sync(0xffffffffu, x_l, i);
 #pragma unroll 4
-          for (int k = __ldg(a.row_ptr + r) + lane; k < e; k += 32)
+          for (int k = b + lane; k < e; k += 32)
             red_add_nc(y + __ldg(a.col + k), __fmul_rn(__ldg(a.val + k), xr));
         }
         if (timed && (i & 7) == 7 && dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_PRIVATE) {
@@ -187,8 +194,11 @@ dysel_status spmtv_register(dysel_ctx *ctx) {
       {"scatter_warp", kSpmtvFns[1], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[1] * n},
       {"scatter_segment", kSpmtvFns[2], {1, 1, 1}, sb, 1, DYSEL_V_ATOMICS, nullptr, (uint64_t)o[2] * n},
   };
-  // initial version: thread per row, the textbook scatter
-  return dysel_register_variants(ctx, kSpmtvSig, v, DYSEL_SPMTV_NVARIANTS, DYSEL_SPMTV_SCATTER_THREAD);
+  // initial version: the default's gated remainder is launched
+  // first at high priority, so the initial version should be the variant
+  // that usually wins; warp per row (coalesced entry loads)
+  const int def = getenv("DYSEL_SPMTV_DEFAULT_THREAD") ? DYSEL_SPMTV_SCATTER_THREAD : DYSEL_SPMTV_SCATTER_WARP;
+  return dysel_register_variants(ctx, kSpmtvSig, v, DYSEL_SPMTV_NVARIANTS, def);
 }
 
 static dysel_status spmtv_check(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *x, float *y) {
