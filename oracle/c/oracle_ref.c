@@ -2,7 +2,8 @@
  *
  * The same definitions as oracle/spmv.py (SURVEY c-1) and oracle/sgemm.py
  * (c-2), as straight loops: used for the CPU baseline timing in bench.py and
- * pinned against the numpy oracle and scipy in tests/test_oracle_c.py.
+ * pinned against the numpy oracle and a triple loop in tests/test_oracle_sgemm.py
+ * (test_c_oracle_spmv, test_c_oracle_gemm).
  *   y_i = sum_{k in row i} (double)val_k * (double)x[col_k]   (CSR order;
  *         SHOC spmv-csr scalar, §4.2)
  *   C   = alpha * A B + beta * C0, row-major, fp64 accumulation

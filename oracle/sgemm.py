@@ -6,7 +6,9 @@ Parboil sgemm the paper profiles (§4.3; work-assignment factor
 (reading A-17 in DESIGN.md).  The matmul is a library primitive (numpy fp64).
 
 Pinned by tests/test_oracle_sgemm.py: triple loop on small shapes, B = I closed
-form, small-integer exactness.
+form, small-integer exactness; sgemm_abs by tests/test_oracle_denominators.py
+(explicit triple loop of |A||B| + |beta||C0|, non-square, negative scalars,
+hand example).
 """
 from __future__ import annotations
 

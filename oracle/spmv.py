@@ -11,7 +11,9 @@ and every profiling mode.
 Pinned by tests/test_oracle_spmv.py: small-integer exactness, identity /
 diagonal closed forms, dense brute force, scipy.sparse; spmtv by dense
 brute force (explicit loops), scipy's A.T @ x and the duality u.(A^T x) =
-(A u).x against spmv.
+(A u).x against spmv; the denominators spmv_abs / spmtv_abs by
+tests/test_oracle_denominators.py (explicit loops, sign cancellation, a
+y0-dominated empty column).
 """
 from __future__ import annotations
 

@@ -16,7 +16,9 @@ DySel only changes which variant computes each 32x4x1 block of points
 
 Pinned by tests/test_oracle_stencil.py: constant and linear fields (the
 6-neighbour sum of a linear field is 6 * its centre value), a pure-Python
-triple loop on tiny grids, boundary copy.
+triple loop on tiny grids, boundary copy; the denominator stencil_abs and
+rel_error by tests/test_oracle_denominators.py (pure-Python loop of
+|c1| sum |nb| + |c0| |c|, constant-field closed form, hand-computed errors).
 """
 from __future__ import annotations
 
@@ -43,6 +45,10 @@ STENCIL_TOL = 1e-6   # fp32: 5 adds + 2 products + 1 subtraction, |rel| <= 8 * 2
 
 
 def rel_error(out, ref, den) -> float:
+    """max |out - ref| / den, den = 0 counted as 1 (the absolute difference);
+    a non-finite out where ref is finite counts as +inf (as spmv.rel_error)."""
     out = np.asarray(out, np.float64)
-    den = np.where(den == 0, 1.0, den)
-    return float(np.max(np.abs(out - ref) / den)) if out.size else 0.0
+    den = np.where(np.asarray(den) == 0, 1.0, den)
+    e = np.abs(out - ref) / den
+    e = np.where(np.isnan(e), np.inf, e)
+    return float(np.max(e)) if out.size else 0.0
