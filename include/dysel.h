@@ -83,24 +83,10 @@ const char *dysel_status_str(dysel_status s);
 #define DYSEL_CONTIGUOUS 64u    /* fully mode: contiguous per-variant slices instead of interleaved granules (A-24) */
 #define DYSEL_SCORE_CYCLES 128u /* score = sum of per-CTA clock64 cycles / units (A-6) */
 #define DYSEL_SCORE_MAKESPAN 256u /* score = latest CTA end - earliest CTA start (%globaltimer), Fig. 7b */
-#define DYSEL_NO_TAIL 512u      /* SpMV device path: the remainder kernel waits for the profiling kernel to
-                                   complete (stream order) instead of starting beside it (PDL) / no CDP2 tail */
 #define DYSEL_NO_ABORT 1024u    /* no dominance: never stop dominated sandbox units early (SpMV, A-26) nor decide
                                    a variant before its profiling CTAs finish (generic launcher, A-32) */
 #define DYSEL_SEQUENTIAL 2048u  /* SpMV device path: profile the variants one after another, each alone on the
                                    GPU (default variant first), scored by makespan (reading A-23) */
-#define DYSEL_DEVICE_LAUNCH 4096u /* SpMV device path, round-1 scheme (ablation): eager kernel and remainder
-                                     launched from the device (CDP2 fire-and-forget) instead of the
-                                     host-launched PDL work kernel */
-#define DYSEL_SOLO 8192u        /* SpMV device path (reading A-38): launch only the default's claim kernel, which
-                                   also runs the winner's remainder slots (through a dispatch over the pool's
-                                   variants at the default's occupancy) — saves the non-winning claim grids
-                                   (~1.6% on D4 when the default wins), costs far more when it does not
-                                   (+44% with a CSR-V default on D4); ignored when the pool holds CSR-T */
-#define DYSEL_ALL_CLAIMS 16384u /* SpMV device path (ablation of reading A-42): host-launch every pool variant's
-                                   claim kernel (PDL-chained, default first) instead of the default's claim kernel
-                                   plus a one-warp switch kernel that device-launches the winner's claim kernel
-                                   only when the default lost */
 /* Default score: generic launcher = makespan (variants are separate concurrent
  * grids, Fig. 7b); SpMV dispatcher = mean per-unit busy time (%globaltimer end -
  * start of each profiled unit; all variants share one launch and occupancy). */
@@ -256,6 +242,15 @@ typedef struct {
    * [4] last eager CTA ended, [5] first remainder CTA started, [6] last
    * remainder CTA ended, [7] longest profiling unit (ns); ~0 = did not happen. */
   uint64_t timeline_ns[8];
+  /* Table 1 allocation record of this launch: extra output
+   * buffers the profiling slices wrote instead of the real output, and their
+   * bytes.  FULLY: 0.  HYBRID: generic launcher K-1 (the default's slice is
+   * productive, A-4), SpMV device path K slice-sized sandboxes (every
+   * variant's profiled units are discardable, the winner's are copied in:
+   * reading A-4').  SWAP: K full private outputs. */
+  uint32_t sandbox_buffers;
+  uint32_t pad_;
+  uint64_t sandbox_bytes;
 } dysel_report;
 
 /* Launch kernel_sig over an NDRange of ndrange_units[3] units
@@ -310,8 +305,10 @@ typedef struct {
   uint64_t prep_ns;              /* device time of format preparation (a-1) */
   uint64_t ell_bytes, jds_bytes; /* extra device memory held by the plan */
   int32_t default_variant;       /* DYSEL_SPMV_* id of the initial version (resolved when AUTO) */
-  int32_t n_heavy;               /* units the claim kernels run first: >= max(8192, 4 x mean) nonzeros,
-                                    by nonzeros descending (longest-processing-time order, A-40) */
+  int32_t n_heavy;               /* units the winner runs first, nonzeros descending (longest-processing-time
+                                    order, A-40): >= max(8192, 4 x mean) nonzeros or a row longer
+                                    than max(1024, 8 x mean row) (A-45); 0 when the plan keeps index order */
+  int32_t n_light;               /* the other units: the profiling sample and the eager default's range (A-45) */
 } dysel_spmv_plan_info;
 
 /* Build the variant pool for one CSR matrix: CSR -> ELL and CSR -> block JDS
@@ -329,22 +326,29 @@ dysel_status dysel_spmv_plan_get_info(const dysel_spmv_plan *plan, dysel_spmv_pl
 /* Test / debug: copy one of the plan's format arrays (layouts in DESIGN.md
  * §Data layout) to HOST memory, synchronously.  which: 0 ell_col (int32),
  * 1 ell_val (f32), 2 perm (int32), 3 jds_len (int32), 4 blk_off (int64),
- * 5 jd_off (int64), 6 jd_ptr (int32), 7 jds_col (int32), 8 jds_val (f32).
+ * 5 jd_off (int64), 6 jd_ptr (int32), 7 jds_col (int32), 8 jds_val (f32),
+ * 9 unit order seq (int32 [n_units]: light units in index order, then the
+ * heavy / long-row units by nonzeros descending; DYSEL_ERR_NOT_FOUND when the
+ * plan keeps index order).
  * *bytes: in = capacity of dst, out = size of the array; dst NULL = query.
  * DYSEL_ERR_NOT_FOUND if the plan has no such format. */
 dysel_status dysel_spmv_plan_copy_array(const dysel_spmv_plan *plan, int which, void *dst, size_t *bytes);
 void dysel_spmv_plan_destroy(dysel_spmv_plan *plan);
 
-/* One DySel SpMV launch: y = A x.  d_x fp32 [n_cols], d_y fp32 [n_rows].
- * Device path (default): ONE persistent launch; tickets claim granules, the
- * profiling tickets first; the last profiling CTA publishes the selection on
- * the device; sync mode spins on it, async mode reads the best so far
- * (SURVEY §8a device protocol); hybrid sandbox units of a provably losing
- * variant stop early (dominance, unless DYSEL_NO_ABORT), and once the
- * selection is published the last profiling CTA hands every unclaimed unit to
- * the winner's plain kernel with a CDP2 tail launch (unless DYSEL_NO_TAIL).
- * With DYSEL_HOST_ORCH: one kernel per variant
- * on forked streams, host reads the selection, then the remainder kernel
+/* One DySel SpMV launch: y = A x.  d_x fp32 [n_cols], d_y fp32 [n_rows] (any
+ * 4-byte alignment).  Device path (default; SURVEY §8a device protocol):
+ * an init kernel, ONE profiling kernel running all K variants' slices (the
+ * units seq[0, p_end) of the plan's unit order: light units, A-45), the
+ * default variant's claim kernel and a one-warp switch kernel, chained by
+ * programmatic dependent launch, no host round trip.  The last profiling CTA
+ * publishes the selection on the device.  SYNC: the claim kernel's warps wait
+ * for it; ASYNC: they first claim light remainder slots with the default
+ * variant (eager execution), then the winner's warps take the
+ * heavy / long-row units first and the rest; when a non-default variant won,
+ * the switch kernel launches its claim kernel from the device (reading A-42).
+ * Hybrid sandbox units of a provably losing variant stop early (dominance,
+ * unless DYSEL_NO_ABORT).  With DYSEL_HOST_ORCH: one kernel per variant on
+ * forked streams, the host reads the selection, then the remainder kernel
  * (paper-faithful).  Mode AUTO uses the plan's uniformity flag. */
 dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,
                         float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
@@ -413,7 +417,7 @@ dysel_status dysel_stencil_variant(dysel_ctx *ctx, int variant_id, int nx, int n
  * scatter-add kernel whose work-groups write overlapping outputs through
  * global atomics, i.e. the paper's case for swap-based partial-productive
  * profiling (§2.2, §3.3, Table 1
- * P:L735-739).  Both built-in variants carry DYSEL_V_ATOMICS: AUTO resolves
+ * P:L735-739).  All three built-in variants carry DYSEL_V_ATOMICS: AUTO resolves
  * to SWAP (each variant profiles the same slice into a private copy of y
  * initialised from y; the winner's copy is swapped in; the winner runs the
  * rest); SWAP|ASYNC returns DYSEL_ERR_UNSUPPORTED.  Unit = 256 rows of A.
@@ -494,14 +498,6 @@ dysel_status dysel_timer_calibrate(dysel_ctx *ctx, uint64_t samples, uint64_t sp
 /* Known-cost test variants (c-8): registers sig with n variants whose CTAs
  * spin cost_ns[v] per unit (wa = 1) and write out[u] = v+1 for each unit u
  * (args[0] = uint32_t* out).  Used to check selection end to end. */
-/* Launch-path experiment: the full grid of one SpMV pool variant launched
- * from the host (how = 0), from the device fire-and-forget (1) or as a device
- * tail launch (2) by a one-thread parent kernel, stream-ordered on `stream`.
- * h_resident_max (nullable, n_sm entries, HOST): the maximum number of CTAs
- * resident at once on each SM (measured with %smid counters; blocks). */
-dysel_status dysel_debug_spmv_device_launch(dysel_ctx *ctx, dysel_spmv_plan *plan, int variant_id,
-                                            const float *d_x, float *d_y, int how, void *stream,
-                                            uint32_t *h_resident_max, int n_sm);
 dysel_status dysel_register_spin_variants(dysel_ctx *ctx, const char *sig, const uint32_t *cost_ns, int n,
                                           int default_variant);
 

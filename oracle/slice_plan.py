@@ -225,3 +225,47 @@ def granule_units(p: Plan, j: int, U):
             for x in range(gx * p.g[0], min(U[0], (gx + 1) * p.g[0])):
                 out.append((x, y, z))
     return out
+
+
+# ----------------------------------------------------- SpMV unit order (A-40, A-45)
+UNIT_ROWS = 256
+HEAVY_UNIT_NNZ = 8192
+LONG_ROW = 1024
+
+
+def unit_order(row_ptr, n_sm):
+    """The SpMV plan's unit order (readings A-40 and A-45): returns
+    (seq, n_light) or (None, n_units) for index order.
+
+    The paper's NDRange runs work-groups in index order and profiles a prefix
+    (P:L865-869); on a heavy-tailed matrix the device path instead (A-45)
+    profiles, and lets the not-yet-proven initial version run eagerly, only
+    LIGHT units, and the winner runs the others first, longest first (A-40).
+      unit u = rows [256 u, 256 u + 256); nnz_u, max_u = its nonzeros / longest row
+      thr  = max(8192, 4 * floor(nnz / n_units))       (heavy: nnz_u >= thr)
+      lcap = max(1024, 8 * ceil(nnz / n_rows))          (long:  max_u > lcap)
+      applied when n_units >= 4 * n_sm and some unit is heavy or long;
+      seq = light units in index order ++ the others by nnz_u descending (stable).
+    Integer work: the library must agree bit-exactly."""
+    rp = [int(v) for v in row_ptr]
+    n = len(rp) - 1
+    nnz = rp[-1] if n >= 0 else 0
+    nu = (n + UNIT_ROWS - 1) // UNIT_ROWS
+    if nu == 0:
+        return None, 0
+    mean = nnz // nu
+    thr = max(HEAVY_UNIT_NNZ, 4 * mean)
+    lcap = max(LONG_ROW, 8 * ((nnz + n - 1) // n)) if n > 0 else LONG_ROW
+    if nu < 4 * n_sm:
+        return None, nu
+    light, rest, nz = [], [], []
+    for u in range(nu):
+        r0, r1 = u * UNIT_ROWS, min((u + 1) * UNIT_ROWS, n)
+        cnt = rp[r1] - rp[r0]
+        mx = max(rp[r + 1] - rp[r] for r in range(r0, r1))
+        nz.append(cnt)
+        (light if (cnt < thr and mx <= lcap) else rest).append(u)
+    if not rest:
+        return None, nu
+    rest = sorted(rest, key=lambda u: -nz[u])      # Python's sort is stable
+    return light + rest, len(light)

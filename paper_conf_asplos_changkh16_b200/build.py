@@ -20,7 +20,7 @@ CSRC = os.path.join(HERE, "csrc")
 INC = os.path.join(ROOT, "include")
 OBJ = os.path.join(ROOT, "build", "obj")
 LIB = os.path.join(HERE, "libdysel.so")
-SOURCES = ["runtime.cu", "spmv.cu", "spmv_prep.cu", "sgemm.cu", "comm.cu", "iterate.cu", "stencil.cu", "spmtv.cu"]
+SOURCES = ["runtime.cu", "spmv.cu", "spmv_probe.cu", "spmv_prep.cu", "sgemm.cu", "comm.cu", "iterate.cu", "stencil.cu", "spmtv.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
@@ -33,7 +33,7 @@ def _deps():
     return max(os.path.getmtime(h) for h in hdrs)
 
 
-RDC = {"spmv.cu"}   # device-side (CDP2 tail) launches need relocatable device code
+RDC = {"spmv.cu"}   # the switch kernel's device-side launch (A-42) needs relocatable device code
 
 
 def _compile(src, verbose):

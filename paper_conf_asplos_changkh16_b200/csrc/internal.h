@@ -110,6 +110,10 @@ struct dysel_ctx {
   uint64_t *h_pending_sel = nullptr;   // pinned + mapped, kPendingRing words
   uint64_t *d_pending_sel = nullptr;   // device alias of h_pending_sel
   int pending_head = 0;
+  // set (mapped pinned word) by a device-path wait for the selection that
+  // timed out; reported as DYSEL_ERR_CUDA by the next call / the report
+  uint32_t *h_sel_timeout = nullptr;
+  uint32_t *d_sel_timeout = nullptr;
   uint64_t launches = 0;
   uint64_t plan_serial = 0;
   // multi-GPU
@@ -128,6 +132,8 @@ dysel_status push_pending_sel(dysel_ctx *ctx, const std::string &sig, const uint
 // handed to the kernel that publishes the selection), then commit after launch
 int reserve_pending_sel(dysel_ctx *ctx, uint64_t **d_slot);
 dysel_status commit_pending_sel(dysel_ctx *ctx, int slot, const std::string &sig, cudaStream_t st);
+// DYSEL_ERR_CUDA (and clears the flag) if a device-path selection wait timed out
+dysel_status check_sel_timeout(dysel_ctx *ctx);
 // move landed selections into the cache; block_sig != NULL waits for that sig
 void resolve_pending(dysel_ctx *ctx, const char *block_sig);
 // dysel_launch with a selection-cache key distinct from the registry sig

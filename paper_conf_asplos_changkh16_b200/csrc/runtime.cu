@@ -96,6 +96,17 @@ void resolve_pending(dysel_ctx *ctx, const char *block_sig) {
   cudaGetLastError();
 }
 
+dysel_status check_sel_timeout(dysel_ctx *ctx) {
+  if (ctx && ctx->h_sel_timeout && *(volatile uint32_t *)ctx->h_sel_timeout) {
+    *(volatile uint32_t *)ctx->h_sel_timeout = 0u;
+    set_error(ctx, "a device-path launch timed out (5 s) waiting for its profiling slices to publish the "
+                   "selection; fully/hybrid ran the remainder with the default variant, swap left the output "
+                   "without the remainder");
+    return DYSEL_ERR_CUDA;
+  }
+  return DYSEL_OK;
+}
+
 static uint64_t lcm64(uint64_t a, uint64_t b) { return a / std::gcd(a, b) * b; }
 
 // Slice planning — a-2 / readings A-1, A-2, A-3.  Mirrors oracle/slice_plan.py
@@ -193,24 +204,50 @@ __global__ void init_prof_kernel(DevProf *p, int K, int def) {
   }
 }
 
+// Swap-mode copy-in of the winner's private output (Table 1): EVERY byte is
+// gated on the selection (a losing variant's private copy may be partial —
+// dominance stops it — so nothing of it may reach the output).  16-byte
+// vector body when both pointers are 16-byte aligned, bytes otherwise.
+__global__ void gated_copy_kernel(char *dst, const char *src, size_t bytes, const uint64_t *gate, int v) {
+  if ((int)(dysel_ld_acquire_u64(gate) & 0xffu) != v) return;
+  const size_t tid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, nt = (size_t)gridDim.x * blockDim.x;
+  size_t head = 0;
+  if ((((uintptr_t)dst | (uintptr_t)src) & 15) == 0) {
+    const size_t n16 = bytes / 16;
+    for (size_t i = tid; i < n16; i += nt) reinterpret_cast<uint4 *>(dst)[i] = reinterpret_cast<const uint4 *>(src)[i];
+    head = n16 * 16;
+  }
+  for (size_t i = head + tid; i < bytes; i += nt) dst[i] = src[i];
+}
+
+// Bounded wait for the selection (reading A-32's wait kernel) failed: flag it
+// for the host (mapped pinned word, checked by the next call and by the
+// report) and, where the default variant's output is usable — fully and
+// hybrid, whose profiling slices are productive in place — publish the
+// default so the remainder still runs; swap (private outputs) keeps the gate
+// closed and the host returns an error.
+__device__ __forceinline__ void selection_timeout(uint64_t *sel, uint32_t *flag, int def, int swap) {
+  if (flag) *(volatile uint32_t *)flag = 1u;
+  if (!swap) atomicCAS((unsigned long long *)sel, ~0ull, ((((1ull << 56) - 1)) << 8) | (uint64_t)def);
+  __threadfence_system();
+}
+
 // Device path: stream-order the gated remainder behind the SELECTION rather
 // than behind the profiling kernels' completion — a variant decided by
 // dominance (A-32) may still be finishing productive tiles.  One thread; the
 // selection is always published (every variant is decided by completion or
 // dominance), so the wait ends.
-__global__ void wait_selection_kernel(const uint64_t *sel) {
+__global__ void wait_selection_kernel(uint64_t *sel, uint32_t *timeout_flag, int def, int swap) {
   // bounded (5 s): a variant that never calls dysel_prof_end would otherwise
-  // hang the stream; its gated copies then all exit (no variant selected)
+  // hang the stream; the timeout is reported, never silent (selection_timeout)
   const uint64_t t0 = dysel_globaltimer();
-  for (uint32_t ns = 64; dysel_ld_acquire_u64(sel) == ~0ull && dysel_globaltimer() - t0 < 5000000000ull;
-       ns = ns < 2048 ? 2 * ns : ns)
+  for (uint32_t ns = 64; dysel_ld_acquire_u64(sel) == ~0ull; ns = ns < 2048 ? 2 * ns : ns) {
+    if (dysel_globaltimer() - t0 >= 5000000000ull) {
+      selection_timeout(sel, timeout_flag, def, swap);
+      return;
+    }
     __nanosleep(ns);
-}
-
-__global__ void gated_copy_kernel(uint4 *dst, const uint4 *src, size_t n16, const uint64_t *gate, int v) {
-  if ((int)(dysel_ld_acquire_u64(gate) & 0xffu) != v) return;
-  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n16; i += (size_t)gridDim.x * blockDim.x)
-    dst[i] = src[i];
+  }
 }
 
 __global__ void timer_calib_kernel(uint64_t samples, uint64_t spin_ns, uint64_t *out) {
@@ -318,6 +355,8 @@ static void fill_report_common(dysel_report *rep, const Plan &p, int mode_used, 
   rep->eager_units = 0;
   rep->tail_units = 0;
   rep->n_slices = 0;
+  rep->sandbox_buffers = 0;
+  rep->sandbox_bytes = 0;
   for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v) {
     rep->score[v] = rep->makespan_ns[v] = rep->units[v] = rep->cycles[v] = 0;
     rep->busy_ns[v] = rep->aborted[v] = 0;
@@ -410,6 +449,10 @@ dysel_status dysel_create(int cuda_device, dysel_ctx **out) {
     return fail(DYSEL_ERR_NOMEM);
   for (int i = 0; i < kPendingRing; ++i)
     if (cudaEventCreateWithFlags(&ctx->pending[i].ev, cudaEventDisableTiming) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+  if (cudaHostAlloc((void **)&ctx->h_sel_timeout, sizeof(uint32_t), cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostGetDevicePointer((void **)&ctx->d_sel_timeout, ctx->h_sel_timeout, 0) != cudaSuccess)
+    return fail(DYSEL_ERR_NOMEM);
+  *ctx->h_sel_timeout = 0u;
   if (spmv_ctx_init(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   if (sgemm_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
   if (stencil_register(ctx) != DYSEL_OK) return fail(DYSEL_ERR_CUDA);
@@ -441,6 +484,7 @@ void dysel_destroy(dysel_ctx *ctx) {
   if (ctx->d_prof) cudaFree(ctx->d_prof);
   if (ctx->h_prof) cudaFreeHost(ctx->h_prof);
   if (ctx->h_pending_sel) cudaFreeHost(ctx->h_pending_sel);
+  if (ctx->h_sel_timeout) cudaFreeHost(ctx->h_sel_timeout);
   for (int i = 0; i < kPendingRing; ++i)
     if (ctx->pending[i].ev) cudaEventDestroy(ctx->pending[i].ev);
   for (auto &b : ctx->sandbox)
@@ -518,6 +562,7 @@ dysel_status dysel_register_spin_variants(dysel_ctx *ctx, const char *sig, const
 dysel_status dysel_get_selection(dysel_ctx *ctx, const char *key, int *variant) {
   if (!ctx || !key || !variant) return DYSEL_ERR_INVALID;
   resolve_pending(ctx, key);
+  DYSEL_TRY(check_sel_timeout(ctx));
   auto it = ctx->sel_cache.find(key);
   if (it == ctx->sel_cache.end()) return DYSEL_ERR_NOT_FOUND;
   *variant = it->second;
@@ -570,6 +615,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     set_error(ctx, std::string("dysel_launch: unknown kernel_sig ") + sig);
     return DYSEL_ERR_INVALID;
   }
+  DYSEL_TRY(check_sel_timeout(ctx));   // a previous launch's selection wait timed out
   const Registered &R = it->second;
   const int K = (int)R.v.size();
   // initial ("default") version: the registered one, or a per-call choice of
@@ -637,6 +683,8 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     set_error(ctx, "dysel_launch: sandbox_arg_bytes required for hybrid / swap");
     return DYSEL_ERR_INVALID;
   }
+  uint32_t n_sandbox = 0;   // Table 1 allocation record (dysel_report.sandbox_buffers / _bytes)
+  uint64_t sandbox_total = 0;
   if (P.mode == DYSEL_HYBRID || P.mode == DYSEL_SWAP) {
     int slot = 0;
     for (int v = 0; v < K; ++v) {
@@ -654,6 +702,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
                                               cudaMemcpyDeviceToDevice, st));
         vargs[v][a] = ctx->sandbox[slot].ptr;
         slot++;
+        sandbox_total += bytes;
       }
     }
   }
@@ -662,6 +711,12 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
   DYSEL_TRY(check_launch(ctx, "init_prof_kernel"));
   DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_start, st));
   fill_report_common(rep, P, P.mode | (async ? DYSEL_ASYNC : 0), 1, -1);
+  if (rep) {   // buffers per variant redirected: one per sandbox arg (Table 1)
+    for (int v = 0; v < K; ++v)
+      if (!(P.mode == DYSEL_HYBRID && v == def) && P.mode != DYSEL_FULLY && !R.sandbox_args[v].empty()) n_sandbox++;
+    rep->sandbox_buffers = n_sandbox;
+    rep->sandbox_bytes = sandbox_total;
+  }
   for (int v = 0; v < K; ++v) {
     dysel_slice s = base_slice(P);
     s.variant = v;
@@ -738,7 +793,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     cudaStream_t gate_st = ctx->wsel;
     DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_start, 0));
     if (dominance) {
-      wait_selection_kernel<<<1, 1, 0, gate_st>>>(&ctx->d_prof->sel);
+      wait_selection_kernel<<<1, 1, 0, gate_st>>>(&ctx->d_prof->sel, ctx->d_sel_timeout, def, P.mode == DYSEL_SWAP);
       DYSEL_TRY(check_launch(ctx, "wait_selection_kernel"));
     } else {
       for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_join[v], 0));
@@ -749,13 +804,9 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
       for (int v = 0; v < K; ++v)
         for (size_t k = 0; k < R.sandbox_args[v].size(); ++k) {
           int a = R.sandbox_args[v][k];
-          size_t n16 = sandbox_bytes[k] / 16;
-          gated_copy_kernel<<<2 * ctx->n_sm, 256, 0, st>>>((uint4 *)base_args[a], (const uint4 *)vargs[v][a], n16,
-                                                          &ctx->d_prof->sel, v);
+          gated_copy_kernel<<<2 * ctx->n_sm, 256, 0, st>>>((char *)base_args[a], (const char *)vargs[v][a],
+                                                          sandbox_bytes[k], &ctx->d_prof->sel, v);
           DYSEL_TRY(check_launch(ctx, "gated_copy_kernel"));
-          if (sandbox_bytes[k] % 16)
-            DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync((char *)base_args[a] + n16 * 16, (char *)vargs[v][a] + n16 * 16,
-                                                sandbox_bytes[k] % 16, cudaMemcpyDeviceToDevice, st));
         }
       DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, st));
     }
@@ -786,6 +837,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     if (rep) {   // a report costs a D2H copy + sync
       DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(ctx->h_prof, ctx->d_prof, sizeof(DevProf), cudaMemcpyDeviceToHost, st));
       DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
+      DYSEL_TRY(check_sel_timeout(ctx));
       selected = (int)(ctx->h_prof->sel & 0xff);
       ctx->sel_cache[key] = selected;
     }

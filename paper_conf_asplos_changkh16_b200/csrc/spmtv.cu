@@ -202,7 +202,7 @@ dysel_status spmtv_register(dysel_ctx *ctx) {
 }
 
 static dysel_status spmtv_check(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *x, float *y) {
-  if (!pl || (pl->dev.n_rows > 0 && !x) || (pl->dev.n_cols > 0 && !y)) {
+  if (!pl || pl->ctx != ctx || (pl->dev.n_rows > 0 && !x) || (pl->dev.n_cols > 0 && !y)) {
     set_error(ctx, "dysel_spmtv: invalid arguments");
     return DYSEL_ERR_INVALID;
   }

@@ -20,16 +20,19 @@ struct dysel_spmv_plan {
   int vids[DYSEL_SPMV_NVARIANTS] = {};  // pool index -> DYSEL_SPMV_* id
   int def = 0;                        // pool index of the default (initial) variant
   uint32_t n_units = 0;               // 256-row units
-  // heavy-first claim order (reading A-40): units with >= 4x the mean and
-  // >= kHeavyUnitNnz nonzeros, by nonzeros descending; bitmap over units
-  int32_t *heavy = nullptr;
-  uint32_t *heavy_bits = nullptr;
-  uint32_t n_heavy = 0;
+  // unit order (readings A-40, A-45): seq[0, n_light) = light units (no row
+  // longer than the long-row cap, fewer nonzeros than the heavy threshold)
+  // in index order, seq[n_light, n_units) = the rest, nonzeros descending
+  // (longest-processing-time first).  seq = nullptr: identity, every unit
+  // light (uniform matrices, single-wave grids).
+  int32_t *seq = nullptr;
+  uint32_t n_light = 0;
   std::string sig;                    // generic-registry signature (host path)
 };
 
 namespace dysel {
-constexpr int64_t kHeavyUnitNnz = 8192;   // heavy-first order: minimum nonzeros of a heavy unit (A-40)
+constexpr int64_t kHeavyUnitNnz = 8192;   // a unit with >= max(this, 4 x mean) nonzeros is heavy (A-40)
+constexpr int64_t kLongRow = 1024;        // a unit with a row longer than max(this, 8 x mean row) is long (A-45)
 int spmv_pool_index(const dysel_spmv_plan *pl, int vid);
 // register the plan's pool with the generic launcher (host-orchestrated path)
 dysel_status spmv_register_pool(dysel_ctx *ctx, dysel_spmv_plan *pl);

@@ -38,12 +38,25 @@ __global__ void ell_fill_kernel(const int32_t *__restrict__ rp, const int32_t *_
   }
 }
 
-// phase 1: per block, stable sort by length (rank counting), W_b + 1
-// row_ptr at the 256-row unit boundaries (heavy-first order, reading A-40)
-__global__ void unit_bounds_kernel(const int32_t *__restrict__ rp, int64_t n, int64_t nu, int32_t *__restrict__ ub) {
-  const int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (u <= nu) ub[u] = rp[min(u * kUnitRows, n)];
+// per 256-row unit: nonzeros and longest row (unit order, readings A-40 / A-45);
+// one warp per unit
+__global__ void unit_stats_kernel(const int32_t *__restrict__ rp, int64_t n, int64_t nu, int32_t *__restrict__ nnz_u,
+                                  int32_t *__restrict__ max_u) {
+  const int64_t u = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (u >= nu) return;
+  const int64_t r0 = u * kUnitRows, r1 = min(r0 + kUnitRows, n);
+  int m = 0;
+  for (int64_t r = r0 + lane; r < r1; r += 32) m = max(m, rp[r + 1] - rp[r]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = max(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if (lane == 0) {
+    nnz_u[u] = rp[r1] - rp[r0];
+    max_u[u] = m;
+  }
 }
+
+// phase 1: per block, stable sort by length (rank counting), W_b + 1
 
 __global__ void __launch_bounds__(kUnitRows) jds_sort_kernel(const int32_t *__restrict__ rp, int64_t n,
                                                              int32_t *__restrict__ perm,
@@ -239,44 +252,44 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
   if (formats_mask & DYSEL_FMT_STREAM) pl->vids[pl->K++] = DYSEL_SPMV_CSR_STREAM;
   if (formats_mask & DYSEL_FMT_TMA) pl->vids[pl->K++] = DYSEL_SPMV_CSR_TMA;
   if (cudaStreamSynchronize(st) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
-  {   // heavy-first claim order (reading A-40): the claim kernels run the
-      // heaviest units first (longest-processing-time order), so no warp
-      // starts a 10^4-entry row in the last microseconds of a launch
+  {   // unit order (readings A-40, A-45).  Heavy units (>= max(8192, 4 x
+      // mean) nonzeros) and long-row units (a row longer than max(1024, 8 x
+      // mean row)) are run FIRST by the winner, nonzeros descending
+      // (longest-processing-time order: no warp starts a 10^4-entry row in the
+      // last microseconds of a launch); the rest ("light" units) are sampled
+      // by the profiling slices and run eagerly by the not-yet-proven default
+      // variant, which therefore never starts a long row it may be slow on
+      // (a thread-per-row default on a 16,384-entry row, Fig. 5(b)).
     const int64_t nu = pl->n_units;
     const int64_t mean = nu > 0 ? nnz / nu : 0;
     const int64_t thr = std::max<int64_t>(kHeavyUnitNnz, 4 * mean);
-#ifndef DYSEL_EXP_NO_HEAVY
-#define DYSEL_EXP_NO_HEAVY 0   // experiment knob (scripts/build_exp.py): rows-in-order claims
-#endif
+    const int64_t lcap = std::max<int64_t>(kLongRow, n_rows > 0 ? 8 * ((nnz + n_rows - 1) / n_rows) : 0);
     // (single-wave grids -- fewer than 4 units per SM -- keep the plain order:
     // every slot starts at once; measured 39 vs 41 us at 235 units)
-    if (!DYSEL_EXP_NO_HEAVY && nu >= 4 * (int64_t)ctx->n_sm && nnz >= 2 * thr) {
-      std::vector<int32_t> ub(nu + 1);
-      int32_t *d_ub = nullptr;
-      if (cudaMalloc(&d_ub, (nu + 1) * 4) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
-      unit_bounds_kernel<<<(unsigned)((nu + 256) / 256), 256, 0, st>>>(d_row_ptr, n_rows, nu, d_ub);
-      const bool ok = cudaMemcpyAsync(ub.data(), d_ub, (nu + 1) * 4, cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+    if (nu >= 4 * (int64_t)ctx->n_sm && (nnz >= 2 * thr || W > lcap)) {
+      std::vector<int32_t> un(nu), um(nu);
+      int32_t *d_st = nullptr;
+      if (cudaMalloc(&d_st, 2 * nu * 4) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+      unit_stats_kernel<<<(unsigned)((nu * 32 + 255) / 256), 256, 0, st>>>(d_row_ptr, n_rows, nu, d_st, d_st + nu);
+      const bool ok = cudaMemcpyAsync(un.data(), d_st, nu * 4, cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+                      cudaMemcpyAsync(um.data(), d_st + nu, nu * 4, cudaMemcpyDeviceToHost, st) == cudaSuccess &&
                       cudaStreamSynchronize(st) == cudaSuccess;
-      cudaFree(d_ub);
+      cudaFree(d_st);
       if (!ok) return fail(DYSEL_ERR_CUDA);
-      std::vector<int32_t> hv;
+      std::vector<int32_t> light, rest;
       for (int64_t u = 0; u < nu; ++u)
-        if ((int64_t)ub[u + 1] - ub[u] >= thr) hv.push_back((int32_t)u);
-      std::stable_sort(hv.begin(), hv.end(),
-                       [&](int32_t a, int32_t b) { return ub[a + 1] - ub[a] > ub[b + 1] - ub[b]; });
-      if (!hv.empty()) {
-        std::vector<uint32_t> bits((nu + 31) / 32, 0u);
-        for (int32_t u : hv) bits[u >> 5] |= 1u << (u & 31);
-        if (cudaMalloc(&pl->heavy, hv.size() * 4) != cudaSuccess ||
-            cudaMalloc(&pl->heavy_bits, bits.size() * 4) != cudaSuccess)
-          return fail(DYSEL_ERR_NOMEM);
-        if (cudaMemcpy(pl->heavy, hv.data(), hv.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-            cudaMemcpy(pl->heavy_bits, bits.data(), bits.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
-          return fail(DYSEL_ERR_CUDA);
-        pl->n_heavy = (uint32_t)hv.size();
-        I.n_heavy = (int32_t)hv.size();
+        ((int64_t)un[u] < thr && (int64_t)um[u] <= lcap ? light : rest).push_back((int32_t)u);
+      std::stable_sort(rest.begin(), rest.end(), [&](int32_t a, int32_t b) { return un[a] > un[b]; });
+      if (!rest.empty()) {
+        std::vector<int32_t> seq(light);
+        seq.insert(seq.end(), rest.begin(), rest.end());
+        if (cudaMalloc(&pl->seq, nu * 4) != cudaSuccess) return fail(DYSEL_ERR_NOMEM);
+        if (cudaMemcpy(pl->seq, seq.data(), nu * 4, cudaMemcpyHostToDevice) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
+        pl->n_light = (uint32_t)light.size();
+        I.n_heavy = (int32_t)rest.size();
       }
     }
+    I.n_light = pl->seq ? (int32_t)pl->n_light : (int32_t)nu;
   }
   if (default_variant == DYSEL_SPMV_DEFAULT_AUTO) {   // reading A-30: initial version from row statistics
     if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
@@ -321,9 +334,17 @@ dysel_status dysel_spmv_plan_copy_array(const dysel_spmv_plan *pl, int which, vo
     case 6: src = pl->jd_ptr; sz = (size_t)jd_total * 4; break;
     case 7: src = pl->jds_col; sz = (size_t)nnz * 4; break;
     case 8: src = pl->jds_val; sz = (size_t)nnz * 4; break;
+    case 9: break;
     default: return DYSEL_ERR_INVALID;
   }
-  const bool has = (which <= 1) ? spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0 : spmv_pool_index(pl, DYSEL_SPMV_JDS) >= 0;
+  if (which == 9) {   // unit order (A-45): identity when the plan keeps none
+    src = pl->seq;
+    sz = pl->seq ? (size_t)nb * 4 : 0;
+    if (!pl->seq) return DYSEL_ERR_NOT_FOUND;
+  }
+  const bool has = which == 9 ? true
+                   : (which <= 1) ? spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0
+                                  : spmv_pool_index(pl, DYSEL_SPMV_JDS) >= 0;
   if (!has) return DYSEL_ERR_NOT_FOUND;
   if (!dst) {
     *bytes = sz;
@@ -354,8 +375,7 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *pl) {
   cudaFree(pl->jds_val);
   cudaFree(pl->blk_off);
   cudaFree(pl->jd_off);
-  cudaFree(pl->heavy);
-  cudaFree(pl->heavy_bits);
+  cudaFree(pl->seq);
   cudaGetLastError();
   delete pl;
 }

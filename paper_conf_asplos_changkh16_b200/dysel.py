@@ -26,8 +26,7 @@ OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_NOMEM, ERR_CUDA, ERR_NOT_FOUND, ERR_NCCL =
 FULLY, HYBRID, SWAP, AUTO = 0, 1, 2, 3
 SYNC, ASYNC = 0, 4
 NO_PROFILE, HOST_ORCH, FORCE_PROFILE, CONTIGUOUS, SCORE_CYCLES = 8, 16, 32, 64, 128
-SCORE_MAKESPAN, NO_TAIL, NO_ABORT, SEQUENTIAL, DEVICE_LAUNCH, SOLO = 256, 512, 1024, 2048, 4096, 8192
-ALL_CLAIMS = 16384
+SCORE_MAKESPAN, NO_ABORT, SEQUENTIAL = 256, 1024, 2048
 DEFAULT_MODE = FULLY | ASYNC
 V_ATOMICS, V_NONUNIFORM = 1, 2
 ROLE_PRODUCTIVE, ROLE_SANDBOX, ROLE_BATCH, ROLE_PRIVATE, ROLE_EAGER = range(5)
@@ -65,14 +64,14 @@ class Report(ctypes.Structure):
                 ("eager_units", c_u64), ("host_ns", c_u64), ("slices", ctypes.POINTER(SliceRec)),
                 ("slices_cap", ctypes.c_int32), ("n_slices", ctypes.c_int32),
                 ("unit_variant", ctypes.POINTER(ctypes.c_uint8)), ("unit_variant_cap", c_u64),
-                ("timeline_ns", c_u64 * 8)]
+                ("timeline_ns", c_u64 * 8), ("sandbox_buffers", c_u32), ("pad_", c_u32), ("sandbox_bytes", c_u64)]
 
 
 class PlanInfo(ctypes.Structure):
     _fields_ = [("n_rows", c_i64), ("n_cols", c_i64), ("nnz", c_i64), ("n_variants", ctypes.c_int32),
                 ("variant_ids", ctypes.c_int32 * SPMV_NVARIANTS), ("ell_width", ctypes.c_int32), ("uniform", ctypes.c_int32),
                 ("max_row_len", ctypes.c_int32), ("prep_ns", c_u64), ("ell_bytes", c_u64), ("jds_bytes", c_u64),
-                ("default_variant", ctypes.c_int32), ("n_heavy", ctypes.c_int32)]
+                ("default_variant", ctypes.c_int32), ("n_heavy", ctypes.c_int32), ("n_light", ctypes.c_int32)]
 
 
 def _sig(name, res, *args):
@@ -124,7 +123,6 @@ dysel_comm_broadcast = _sig("dysel_comm_broadcast", c_int, P, P, c_size, c_int, 
 dysel_sgemm_sharded = _sig("dysel_sgemm_sharded", c_int, P, c_int, c_int, c_int, c_float, P, c_int, P, c_int, c_float,
                            P, c_int, c_float, c_u32, P, ctypes.POINTER(Report))
 dysel_kernel_launches = _sig("dysel_kernel_launches", c_u64, P)
-dysel_debug_spmv_device_launch = _sig("dysel_debug_spmv_device_launch", c_int, P, P, c_int, P, P, c_int, P, P, c_int)
 dysel_timer_calibrate = _sig("dysel_timer_calibrate", c_int, P, c_u64, c_u64, ctypes.POINTER(c_u64),
                              ctypes.POINTER(ctypes.c_double))
 dysel_register_spin_variants = _sig("dysel_register_spin_variants", c_int, P, ctypes.c_char_p,
@@ -161,7 +159,8 @@ def report_dict(rep: Report, names=None, uv=None):
              score=list(rep.score[:MAX_VARIANTS]), makespan_ns=list(rep.makespan_ns[:MAX_VARIANTS]),
              units=list(rep.units[:MAX_VARIANTS]), cycles=list(rep.cycles[:MAX_VARIANTS]),
              busy_ns=list(rep.busy_ns[:MAX_VARIANTS]), aborted=list(rep.aborted[:MAX_VARIANTS]),
-             tail_units=rep.tail_units, n_slices=rep.n_slices,
+             tail_units=rep.tail_units, n_slices=rep.n_slices, sandbox_buffers=rep.sandbox_buffers,
+             sandbox_bytes=rep.sandbox_bytes,
              timeline_ns=[None if t == 2 ** 64 - 1 else int(t) for t in rep.timeline_ns])
     if rep.slices and rep.slices_cap:
         d["slices"] = [dict(begin=rep.slices[i].granule_begin, count=rep.slices[i].granule_count,
@@ -200,7 +199,7 @@ class SpmvPlan:
 
     _ARRAYS = {"ell_col": (0, "int32"), "ell_val": (1, "float32"), "perm": (2, "int32"), "jds_len": (3, "int32"),
                "blk_off": (4, "int64"), "jd_off": (5, "int64"), "jd_ptr": (6, "int32"), "jds_col": (7, "int32"),
-               "jds_val": (8, "float32")}
+               "jds_val": (8, "float32"), "seq": (9, "int32")}
 
     def array(self, name):
         """Copy a format array of the plan to a host numpy array (tests)."""
@@ -295,15 +294,6 @@ class Context:
                                      int(mode), _stream(stream), _ptr(norms) if norms is not None else None,
                                      ctypes.byref(rep) if rep is not None else None))
         return report_dict(rep, SPMV_NAMES) if rep is not None else None
-
-    def debug_spmv_device_launch(self, plan, variant_id, x, y, how, stream=None, resident=False):
-        """Full grid of one variant launched from the host (0) / device fire-and-forget (1) / tail (2);
-        resident=True returns the max resident CTAs per SM."""
-        n_sm = 148 if resident else 0
-        buf = (ctypes.c_uint32 * 1024)() if resident else None
-        self._check(dysel_debug_spmv_device_launch(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), int(how),
-                                                   _stream(stream), buf, n_sm))
-        return list(buf[:n_sm]) if resident else None
 
     def spmv_variant(self, plan, variant_id, x, y, stream=None):
         self._check(dysel_spmv_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), _stream(stream)))

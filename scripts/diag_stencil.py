@@ -19,4 +19,4 @@ for shape in ((64, 512, 512), (256, 256, 256)):
     nb = 8 * a.numel()
     r = {D.STENCIL_NAMES[v]: b2b(lambda: ctx.stencil_variant(v, a, o, 0.8, 0.15)) for v in range(3)}
     t = b2b(lambda: ctx.stencil(a, o, 0.8, 0.15, f=0.02, mode=D.FULLY | D.ASYNC))
-    print(os.environ.get("DYSEL_LIB", "main"), shape, {k: f"{v:.1f}us {nb / v / 1e3:.0f}GB/s" for k, v in r.items()}, f"dysel {t:.1f}us", flush=True)
+    print(shape, {k: f"{v:.1f}us {nb / v / 1e3:.0f}GB/s" for k, v in r.items()}, f"dysel {t:.1f}us", flush=True)

@@ -173,3 +173,26 @@ def test_partition_balanced_and_cover():
         nz = np.diff(A.row_ptr.astype(np.int64)[b])
         # each shard within one unit's nnz of the ideal share
         assert np.abs(nz - A.nnz / G).max() <= A.row_ptr[-1] / A.n_rows * 256 * 4 + A.lengths().max()
+
+
+def test_unit_order_hand_example():
+    """Readings A-40 / A-45 restated on a hand-built matrix (n_sm = 1, so the
+    rule applies from 4 units): 6 units of 256 rows; unit 1 holds one
+    2,000-entry row (long: > max(1024, 8 x ceil(mean row))), unit 4 holds
+    256 rows of 40 entries (10,240 >= max(8192, 4 x floor(nnz / 6))): heavy.
+    seq = light units in index order, then heavy / long by nonzeros desc."""
+    import numpy as np
+    L = np.full(6 * 256, 2)
+    L[256 + 7] = 2000
+    L[4 * 256:5 * 256] = 40
+    rp = np.concatenate([[0], np.cumsum(L)])
+    nnz = int(rp[-1])   # thr = max(8192, 4 * (14798 // 6)) = 9864, lcap = max(1024, 8 * 10) = 1024
+    assert nnz == 4 * 512 + (255 * 2 + 2000) + 256 * 40
+    seq, n_light = P.unit_order(rp, 1)
+    # unit nnz: u1 = 2510, u4 = 10240 -> rest sorted desc: [4, 1]
+    assert seq == [0, 2, 3, 5, 4, 1] and n_light == 4
+    # fewer than 4 units per SM: index order
+    assert P.unit_order(rp, 2) == (None, 6)
+    # uniform rows: nothing heavy or long -> index order
+    rp2 = np.arange(0, 2 * 6 * 256 + 1, 2)
+    assert P.unit_order(rp2, 1) == (None, 6)

@@ -123,9 +123,8 @@ def test_identity_and_diagonal_exact(ctx):
 
 
 MODES = ["fully_sync", "fully_async", "hybrid_sync", "hybrid_async", "fully_sync_host", "fully_async_host",
-         "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles", "hybrid_async_cdp", "fully_sync_cdp",
-         "hybrid_async_notail", "fully_sync_seq", "hybrid_async_solo", "fully_sync_solo", "hybrid_async_allclaims",
-         "fully_async_allclaims"]
+         "hybrid_sync_host", "fully_contig_sync", "fully_sync_cycles", "fully_sync_seq", "hybrid_async_seq",
+         "hybrid_sync_noabort", "fully_async_makespan"]
 
 
 def mode_bits(D, m):
@@ -135,12 +134,16 @@ def mode_bits(D, m):
     b |= D.HOST_ORCH if m.endswith("host") else 0
     b |= D.CONTIGUOUS if "contig" in m else 0
     b |= D.SCORE_CYCLES if "cycles" in m else 0
-    b |= D.DEVICE_LAUNCH if "cdp" in m else 0
-    b |= D.NO_TAIL if "notail" in m else 0
     b |= D.SEQUENTIAL if "seq" in m else 0
-    b |= D.SOLO if "solo" in m else 0
-    b |= D.ALL_CLAIMS if "allclaims" in m else 0
+    b |= D.NO_ABORT if "noabort" in m else 0
+    b |= D.SCORE_MAKESPAN if "makespan" in m else 0
     return b
+
+
+def unit_order(plan):
+    """The plan's unit order (reading A-45): identity unless it keeps one."""
+    s = plan.array("seq")
+    return np.arange(plan.n_units) if s is None else s
 
 
 @pytest.mark.parametrize("m", MODES)
@@ -153,7 +156,7 @@ def test_dysel_composition(ctx, D, name, m):
     x = uniform_f32(7, A.n_cols)
     # solo (A-38) needs a pool without CSR-T; its remainder then runs the winner
     # through the default's (CSR-S's) claim kernel
-    plan = prepared(ctx, A, default=0, formats=D.FMT_DEFAULT if "solo" in m else None)
+    plan = prepared(ctx, A, default=0)
     xd = vec(x)
     full = {}
     for v in plan.variant_ids:
@@ -183,14 +186,21 @@ def test_dysel_composition(ctx, D, name, m):
     # Device-path hybrid (reading A-4'): the shared profiled units are the
     # winner's (its sandbox is copied in); the host path keeps the paper's
     # productive default (A-4).
+    # The device path profiles the first units of the plan's unit order
+    # (light units first, A-45); the host path the NDRange prefix (paper).
     pool = plan.variant_ids
     owner = slice_plan.productive_cover(p, pool.index(sel))
-    dev_hybrid = p.mode == slice_plan.HYBRID and not m.endswith("host")
+    host = m.endswith("host")
+    order = np.arange(plan.n_units) if host else unit_order(plan)
+    dev_hybrid = p.mode == slice_plan.HYBRID and not host
+    n_prof = p.c * (K if p.mode == slice_plan.FULLY else 1)
     for j in range(p.Gn):
-        if j < len(owner) and (j < p.c * (K if p.mode == slice_plan.FULLY else 1)):
-            assert uv[j] == (sel if dev_hybrid else pool[owner[j]]), j
+        u = order[j]
+        if j < len(owner) and j < n_prof:
+            assert uv[u] == (sel if dev_hybrid else pool[owner[j]]), j
         elif "async" not in m:
-            assert uv[j] == sel, j
+            assert uv[u] == sel, j
+    assert sorted(order) == list(range(plan.n_units))      # a permutation: every unit exactly once
     plan.destroy()
 
 
@@ -255,62 +265,66 @@ def test_edge_cases(ctx, D):
     assert e.value.status == D.ERR_UNSUPPORTED
 
 
+@pytest.mark.parametrize("name", ["powerlaw", "heavy"])
+@pytest.mark.parametrize("default", [1, 3])
 @pytest.mark.parametrize("asy", [False, True])
-def test_remainder_hand_off(ctx, D, asy):
-    """The remainder goes to the winner in every launch scheme: the default's
-    claim kernel + the switch kernel that device-launches a non-default
-    winner's claim kernel (A-42, default), every variant's claim kernel
-    host-launched beside profiling (PDL, ALL_CLAIMS), the same after
-    profiling completes (NO_TAIL), and the round-1 device-launched scheme
-    (DEVICE_LAUNCH: CDP2 eager + remainder, with and without NO_TAIL).
-    Sync: every remainder unit is the winner's (eager = 0); async: the
-    eager units are whole units of the default, the rest the winner's."""
+def test_remainder_hand_off(ctx, D, asy, default, name):
+    """The remainder goes to the winner: the default's claim kernel runs it
+    when the default wins, the switch kernel device-launches the winner's
+    claim kernel otherwise (A-42).  Sync: every remainder unit is the
+    winner's (eager = 0).  Async: the eager units are whole LIGHT units of
+    the default (A-45: an unproven default never starts a heavy or long-row
+    unit, here a thread-per-row JDS default on 16,384-entry rows), the rest
+    the winner's."""
     import torch
-    A = MATS["powerlaw"]()
+    A = MATS[name]()
     x = uniform_f32(11, A.n_cols)
-    plan = prepared(ctx, A, default=1)
+    plan = prepared(ctx, A, default=default)
     K = len(plan.variant_ids)
-    for extra in (0, D.ALL_CLAIMS, D.NO_TAIL, D.DEVICE_LAUNCH, D.DEVICE_LAUNCH | D.NO_TAIL):
-        mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0) | extra
-        y = torch.full((A.n_rows,), float("nan"), device="cuda")
-        r = ctx.spmv(plan, vec(x), y, f=0.05, mode=mode, report=True, unit_map=True)
-        assert spmv_err(A, x, y) <= SPMV_TOL, extra
-        rem = plan.n_units - K * r["c"]
-        uv = r["unit_variant"]
-        if not asy:
-            assert r["eager_units"] == 0 and r["tail_units"] == rem, (extra, r)
-            assert all(uv[u] == r["selected"] for u in range(K * r["c"], plan.n_units)), extra
-        elif not (extra & D.DEVICE_LAUNCH):
-            e = r["eager_units"]
-            assert e + r["tail_units"] == rem, (extra, r)
-            assert all(uv[u] == 1 for u in range(K * r["c"], K * r["c"] + e)), extra
-            assert all(uv[u] == r["selected"] for u in range(K * r["c"] + e, plan.n_units)), extra
+    order = unit_order(plan)
+    n_light = plan.info.n_light
+    if name == "heavy":
+        assert plan.info.n_heavy > 0 and n_light + plan.info.n_heavy == plan.n_units
+    mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0)
+    y = torch.full((A.n_rows,), float("nan"), device="cuda")
+    r = ctx.spmv(plan, vec(x), y, f=0.05, mode=mode, report=True, unit_map=True)
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    P = K * r["c"]
+    rem = plan.n_units - P
+    uv = r["unit_variant"]
+    if not asy:
+        assert r["eager_units"] == 0 and r["tail_units"] == rem, r
+        assert all(uv[order[j]] == r["selected"] for j in range(P, plan.n_units))
+    else:
+        e = r["eager_units"]
+        assert e + r["tail_units"] == rem, r
+        assert P + e <= max(P, n_light)                         # eager units are light
+        assert all(uv[order[j]] == default for j in range(P, P + e))
+        assert all(uv[order[j]] == r["selected"] for j in range(P + e, plan.n_units))
     plan.destroy()
 
 
-def test_tail_launch_is_stream_ordered(ctx, D):
-    """Work queued on the launching stream after dysel_spmv must see the
-    tail-launched remainder complete (the device-launched grid belongs to its
-    parent's completion), without any host synchronisation in between."""
+def test_remainder_is_stream_ordered(ctx, D):
+    """Work queued on the launching stream after dysel_spmv must see the whole
+    remainder complete -- also a winner's claim kernel device-launched by the
+    switch kernel (it belongs to its parent's completion) -- without any host
+    synchronisation in between."""
     import torch
     A = d4_powerlaw(n=400_000, lmax=8000)
     x = uniform_f32(12, A.n_cols)
-    plan = prepared(ctx, A)
     xd = vec(x)
-    ref = torch.empty(A.n_rows, device="cuda")
-    ctx.spmv_variant(plan, 1, xd, ref)
-    torch.cuda.synchronize()
-    for mode in (D.HYBRID | D.SYNC, D.HYBRID | D.ASYNC, D.FULLY | D.SYNC, D.HYBRID | D.ASYNC | D.DEVICE_LAUNCH,
-                 D.FULLY | D.SYNC | D.DEVICE_LAUNCH):
-        for _ in range(3):
-            y = torch.full((A.n_rows,), float("nan"), device="cuda")
-            ctx.spmv(plan, xd, y, f=0.01, mode=mode | D.FORCE_PROFILE)
-            nan_count = torch.isnan(y).sum()          # same stream, no sync
-            snap = y.clone()
-            torch.cuda.synchronize()
-            assert nan_count.item() == 0, mode
-            assert spmv_err(A, x, snap) <= SPMV_TOL
-    plan.destroy()
+    for default in (1, 3):      # 3 (JDS) loses on this matrix: its claim kernel hands over via the switch kernel
+        plan = prepared(ctx, A, default=default)
+        for mode in (D.HYBRID | D.SYNC, D.HYBRID | D.ASYNC, D.FULLY | D.SYNC, D.FULLY | D.ASYNC):
+            for _ in range(3):
+                y = torch.full((A.n_rows,), float("nan"), device="cuda")
+                ctx.spmv(plan, xd, y, f=0.01, mode=mode | D.FORCE_PROFILE)
+                nan_count = torch.isnan(y).sum()          # same stream, no sync
+                snap = y.clone()
+                torch.cuda.synchronize()
+                assert nan_count.item() == 0, mode
+                assert spmv_err(A, x, snap) <= SPMV_TOL
+        plan.destroy()
 
 
 def test_dominance_abort_is_exact(ctx, D):
@@ -403,21 +417,24 @@ def test_gather_probe_runs_and_validates(ctx, D):
 
 
 @pytest.mark.parametrize("name", ["heavy", "powerlaw", "d3small"])
-def test_heavy_first_units(ctx, D, name):
-    """Reading A-40: the plan's heavy units are exactly those with at least
-    max(8192, 4 x mean) nonzeros when the grid spans >= 4 units per SM (rule
-    restated here); every pure variant's heavy-first claim run is within
-    tolerance of the oracle, and CSR-S / ELL / JDS stay bit-identical."""
+def test_unit_order(ctx, D, name):
+    """Readings A-40 / A-45: the plan's unit order (light units in index
+    order, then heavy / long-row units by nonzeros descending) equals the
+    oracle's restatement of the rule bit for bit; every pure variant's
+    heavy-first claim run is within tolerance of the oracle, and CSR-S / ELL /
+    JDS stay bit-identical."""
     import torch
     A = MATS[name]()
     plan = prepared(ctx, A)
-    nu = (A.n_rows + 255) // 256
-    ub = A.row_ptr[np.minimum(np.arange(nu + 1) * 256, A.n_rows)].astype(np.int64)
-    thr = max(8192, 4 * (A.nnz // nu))
-    want = int((np.diff(ub) >= thr).sum()) if (A.nnz >= 2 * thr and nu >= 4 * ctx.n_sm) else 0
-    assert plan.info.n_heavy == want
+    seq, n_light = slice_plan.unit_order(A.row_ptr, ctx.n_sm)
+    got = plan.array("seq")
+    if seq is None:
+        assert got is None and plan.info.n_heavy == 0 and plan.info.n_light == plan.n_units
+    else:
+        assert np.array_equal(got, np.asarray(seq, np.int32))
+        assert plan.info.n_light == n_light and plan.info.n_heavy == plan.n_units - n_light
     if name == "heavy":
-        assert want > 0
+        assert seq is not None and n_light < plan.n_units
     x = uniform_f32(9, A.n_cols)
     xd = vec(x)
     ys = {}
