@@ -1,15 +1,24 @@
-"""DySel benchmark — one JSON line (driver contract).
+"""DySel benchmark — one JSON line (driver contract; DESIGN.md §7 Measurement).
 
 Step = one DySel SpMV launch over the D4 power-law matrix (10^7 rows, ~2*10^8
 nnz): profiling ON every step (single-shot, AUTO mode ->
 hybrid, async), i.e. format-prepared pool -> micro-profiling -> device-side
 selection -> remainder, all in libdysel.so.  `value` = algorithmic SpMV bytes
-(8 nnz + 4 (n+1) + 4 n_cols + 4 n) / step time, aggregated over ranks.
-Inputs (1.72 GB) are larger than L2, so no flush is needed between steps.
+(8 nnz + 4 (n+1) + 4 n_cols + 4 n) of the whole matrix / step time (max over
+ranks).  Inputs (1.72 GB) are larger than L2, so no flush between steps.
 
-Also reported in the same line: the exhaustive-oracle best pure variant T*
- and DySel's overhead vs it, amortised overhead with the
-activation flag, and secondary workloads (D3 SpMV, D2m SGEMM).
+N > 1 (`--gpus N`): rows are sharded nnz-balanced over N ranks (one process
+per GPU; spawned here when not launched by torchrun), each rank profiles and
+selects on its own shard (a "mixed version") and y is
+all-gathered over NCCL inside the step (dysel_spmv_sharded): strong scaling.
+
+Also in the same line: the exhaustive-oracle best pure variant T*
+ and DySel's overhead vs it, step-time percentiles, amortised
+overhead with the activation flag, ablations (SYNC, a non-best default, f),
+e2e through the public call with host buffers (dependent steps, and
+pipelined independent requests), the roofline of the dominant kernel, the CPU
+oracle baseline, and secondary workloads (D1, D2s, D2m, D3, a 2.25M-row FEM
+matrix, D6, D7 SGEMM 8192^3, the stencil and SpMTV pools).
 
     python bench.py [--gpus N --steps K --warmup W] [--impl dysel|reference]
 """
@@ -18,6 +27,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import socket
 import subprocess
 import sys
 import threading
@@ -30,13 +40,14 @@ sys.path.insert(0, ROOT)
 
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM = 6650.0
+METRIC = "DySel SpMV GB/s (power-law 1e7 rows, profiling on every call) + overhead % vs best-variant oracle"
 
 
 def peaks():
     try:
-        return json.load(open(PEAKS_PATH)), "measured"
+        return json.load(open(PEAKS_PATH)), "measured (MEASURED_PEAKS.json)"
     except Exception:
-        return {"hbm_gbs": FALLBACK_HBM, "bf16_tflops": 1590.0}, "fallback"
+        return {"hbm_gbs": FALLBACK_HBM, "bf16_tflops": 1590.0}, "fallback (B200_PROFILING.md)"
 
 
 def spmv_bytes(n_rows, n_cols, nnz):
@@ -99,10 +110,10 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------- CPU oracle
-def cpu_oracle_spmv(A, x, reps=3):
-    """The oracle as it stands (plain C fp64 loops, OpenMP over all cores)."""
+def cpu_oracle_spmv(A, x, reps=3, threads=None):
+    """The oracle as it stands (plain C fp64 loops, OpenMP over `threads` cores)."""
     from oracle import ref_c
-    cores = len(os.sched_getaffinity(0))
+    cores = threads or len(os.sched_getaffinity(0))
     ref_c.spmv_f64(A.row_ptr, A.col, A.val, x, cores)    # warm
     ts = []
     for _ in range(reps):
@@ -110,6 +121,21 @@ def cpu_oracle_spmv(A, x, reps=3):
         ref_c.spmv_f64(A.row_ptr, A.col, A.val, x, cores)
         ts.append(time.perf_counter() - t0)
     return float(np.median(ts)), cores
+
+
+def cpu_single_thread_sample(A, x, rows=1_000_000):
+    """Single-threaded plain-C fp64 oracle on the first `rows` rows of A
+    (SURVEY §8d CPU timing (i)); returns (GB/s on the sample's algorithmic
+    bytes, sample description)."""
+    from oracle import ref_c
+    r1 = min(rows, A.n_rows)
+    hi = int(A.row_ptr[r1])
+    rp, col, val = A.row_ptr[:r1 + 1], A.col[:hi], A.val[:hi]
+    ref_c.spmv_f64(rp, col, val, x, 1)
+    t0 = time.perf_counter()
+    ref_c.spmv_f64(rp, col, val, x, 1)
+    t = time.perf_counter() - t0
+    return spmv_bytes(r1, A.n_cols, hi) / t / 1e9, f"first {r1} rows of D4 ({hi} nnz), 1 thread, fp64"
 
 
 # ------------------------------------------------------------- workloads
@@ -120,8 +146,17 @@ def make_d4(n):
     return A, x
 
 
+def config(A, world, f):
+    return {"workload": "D4 power-law SpMV: 10^7 rows, p(L)~L^-1.761 on [1,16384], uniform cols, fp32 CSR",
+            "n_rows": int(A.n_rows), "nnz": int(A.nnz),
+            "parallelism": f"row-shard{world}" + (" (nnz-balanced, NCCL y allgatherv)" if world > 1 else ""),
+            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": f"AUTO|ASYNC (hybrid), f={f}",
+            "default_variant": "DYSEL_SPMV_DEFAULT_AUTO (A-30)"}
+
+
 def reference_arm(args, world, rank):
-    """--impl reference: the oracle timed on the host cores, same metric/unit."""
+    """--impl reference: the oracle timed on the host cores, same metric/unit.
+    Under torchrun rank 0 alone runs it; the other ranks exit without work."""
     if rank != 0:
         return
     A, x = make_d4(args.rows)
@@ -147,18 +182,9 @@ def reference_arm(args, world, rank):
     print(json.dumps(line), flush=True)
 
 
-METRIC = "DySel SpMV GB/s (power-law 1e7 rows, profiling on every call) + overhead % vs best-variant oracle"
-
-
-def config(A, world, f):
-    return {"workload": "D4 power-law SpMV: 10^7 rows, p(L)~L^-1.761 on [1,16384], uniform cols, fp32 CSR",
-            "n_rows": int(A.n_rows), "nnz": int(A.nnz), "parallelism": f"row-shard{world}",
-            "l2": "inputs (1.72 GB) larger than L2; no flush", "mode": f"AUTO|ASYNC (hybrid), f={f}",
-            "default_variant": "DYSEL_SPMV_DEFAULT_AUTO (A-30)"}
-
-
 # ------------------------------------------------------------------ timing
 def time_events(fn, reps, stream):
+    """Per-call times (s): one event pair around each call."""
     import torch
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
     torch.cuda.synchronize()
@@ -170,7 +196,27 @@ def time_events(fn, reps, stream):
     return [a.elapsed_time(b) * 1e-3 for a, b in evs]
 
 
-def dysel_arm(args, world, rank, local_rank):
+def time_b2b(fn, reps, stream):
+    """Mean time (s) of `reps` back-to-back calls between two events."""
+    import torch
+    for _ in range(2):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for _ in range(reps):
+        fn()
+    b.record(stream)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) * 1e-3 / reps
+
+
+def pct(ts, q):
+    return round(float(np.percentile(np.asarray(ts), q)) * 1e3, 4)
+
+
+# ----------------------------------------------------------------- the arm
+def dysel_arm(args, world, rank, local_rank, A=None, x=None):
     import torch
     import torch.distributed as dist
     from paper_conf_asplos_changkh16_b200 import dysel as D
@@ -182,7 +228,8 @@ def dysel_arm(args, world, rank, local_rank):
         uid = [D.comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         ctx.comm_init(rank, world, uid[0])
-    A, x = make_d4(args.rows)
+    if A is None:
+        A, x = make_d4(args.rows)
     nbytes_total = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
     bounds = D.partition_rows(A.row_ptr, world)
     r0, r1 = bounds[rank], bounds[rank + 1]
@@ -198,15 +245,15 @@ def dysel_arm(args, world, rank, local_rank):
     default_name = D.SPMV_NAMES[plan.info.default_variant]
     mode = D.AUTO | D.ASYNC
     f = args.f
+    yl = y[r0:r1]
 
     def step():
         if world > 1:
             ctx.spmv_sharded(plan, bounds, xd, y, f=f, mode=mode)
         else:
-            ctx.spmv(plan, xd, y[r0:r1], f=f, mode=mode)
+            ctx.spmv(plan, xd, yl, f=f, mode=mode)
 
-    # ---- exhaustive oracle: every pure variant, full grid
-    yl = y[r0:r1]
+    # ---- exhaustive oracle: every pure variant over this rank's rows
     T_v = {}
     for v in plan.variant_ids:
         for _ in range(2):
@@ -220,8 +267,6 @@ def dysel_arm(args, world, rank, local_rank):
     probe = {}
     try:
         for fl, nm in ((0, "gather"), (1, "stream")):
-            for _ in range(2):
-                ctx.spmv_gather_probe(plan, fl, xd, yl)
             probe[nm] = time_b2b(lambda: ctx.spmv_gather_probe(plan, fl, xd, yl), args.oracle_reps, stream)
     except Exception as e:   # unaligned col / val: no probe
         probe = {"error": str(e)}
@@ -252,14 +297,25 @@ def dysel_arm(args, world, rank, local_rank):
         T_total = float(t.item())
     T_step = T_total / args.steps
     value = nbytes_total / T_step / 1e9
+    # per-step percentiles (one event pair per step, after the timed region)
+    if world > 1:
+        dist.barrier()
+    per_step = time_events(step, args.steps, stream)
     # report of one extra (untimed) launch: selection, scores
     rep = ctx.spmv(plan, xd, yl, f=f, mode=mode, report=True)
+    sels = [None] * world
+    if world > 1:
+        dist.all_gather_object(sels, rep["selected_name"])
+    else:
+        sels = [rep["selected_name"]]
     # selection accuracy over repeated single-shot launches (95%)
     accuracy = {}
-    for ff in sorted({f, 0.001, 0.005}):
-        sels = [ctx.spmv(plan, xd, yl, f=ff, mode=mode, report=True)["selected_name"] for _ in range(20)]
-        accuracy[str(ff)] = {"exact": round(sum(n == best_name for n in sels) / len(sels), 3),
-                             "within_5pct": round(sum(T_v.get(n, 1e9) <= 1.05 * T_star for n in sels) / len(sels), 3)}
+    if world == 1:
+        for ff in sorted({f, 0.001, 0.005}):
+            ss = [ctx.spmv(plan, xd, yl, f=ff, mode=mode, report=True)["selected_name"] for _ in range(20)]
+            accuracy[str(ff)] = {"exact": round(sum(n == best_name for n in ss) / len(ss), 3),
+                                 "within_5pct": round(sum(T_v.get(n, 1e9) <= 1.05 * T_star for n in ss) / len(ss),
+                                                      3)}
     # ---- amortised: profile once, then the activation flag
     I = args.amortize
     def amort():
@@ -267,19 +323,14 @@ def dysel_arm(args, world, rank, local_rank):
         for _ in range(I - 1):
             ctx.spmv(plan, xd, yl, mode=D.NO_PROFILE)
     ta = float(np.median(time_events(amort, 3, stream))) / I
-    # ---- e2e through the public API with host buffers: x H2D, y D2H per step
-    # ---- ablations (rank 0, 1 GPU): sync mode, a non-best default, f
+    # ---- ablations (1 GPU): SYNC, a non-best default (async and sync), f
     ablation = {}
     if world == 1 and not args.no_secondary:
         ablation["sync_overhead_pct"] = round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=D.AUTO), 10, stream)
                                                / T_star - 1) * 100, 2)
-        ablation["solo_claim_kernel_overhead_pct"] = round(
-            (time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=mode | D.SOLO), 10, stream) / T_star - 1) * 100, 2)
-        ablation["all_claim_kernels_overhead_pct"] = round(
-            (time_b2b(lambda: ctx.spmv(plan, xd, yl, f=f, mode=mode | D.ALL_CLAIMS), 10, stream) / T_star - 1) * 100,
-            2)
-        ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10, stream)
-                                                      / T_star - 1) * 100, 2) for ff in (0.001, 0.005, 0.01, 0.02)}
+        ablation["f_overhead_pct"] = {str(ff): round((time_b2b(lambda: ctx.spmv(plan, xd, yl, f=ff, mode=mode), 10,
+                                                               stream) / T_star - 1) * 100, 2)
+                                      for ff in (0.001, 0.005, 0.01, 0.02)}
         # iterative driver (SURVEY §8f f-3, P:L796-804 / §5.2): 20 power
         # iterations; profiling on iteration 0 only vs every iteration vs never
         xi, yi = xd.clone(), torch.empty_like(yl)
@@ -299,12 +350,16 @@ def dysel_arm(args, world, rank, local_rank):
         for dname, dv in (("csr_vector", D.SPMV_CSR_VECTOR), ("jds", D.SPMV_JDS)):
             pd = ctx.spmv_prepare(rp, col, val, A.n_cols, default=dv)
             td = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode), 10, stream)
+            tds = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=D.AUTO), 10, stream)
             rd = ctx.spmv(pd, xd, yl, f=f, mode=mode, report=True)
-            tda = time_b2b(lambda: ctx.spmv(pd, xd, yl, f=f, mode=mode | D.ALL_CLAIMS), 10, stream)
             ablation[f"default_{dname}"] = {"overhead_pct": round((td / T_star - 1) * 100, 2),
-                                            "all_claims_overhead_pct": round((tda / T_star - 1) * 100, 2),
-                                            "selected": rd["selected_name"], "eager_units": rd["eager_units"]}
+                                            "sync_overhead_pct": round((tds / T_star - 1) * 100, 2),
+                                            "selected": rd["selected_name"], "eager_units": rd["eager_units"],
+                                            "publish_us": (round(rd["timeline_ns"][1] / 1e3, 1)
+                                                           if rd["timeline_ns"][1] is not None else None)}
             pd.destroy()
+    # ---- e2e through the public call with HOST buffers: every step copies its
+    # x in from pinned memory and its y out (this rank's rows)
     xh = torch.from_numpy(x).pin_memory()
     yh = torch.empty(r1 - r0, dtype=torch.float32).pin_memory()
     def e2e_step():
@@ -313,10 +368,14 @@ def dysel_arm(args, world, rank, local_rank):
         yh.copy_(yl, non_blocking=True)
     for _ in range(2):
         e2e_step()
-    te = time_events(e2e_step, args.steps, stream)
-    T_e2e_serial = float(np.mean(te))
-    T_e2e = T_e2e_serial
-    e2e_pipelined = False
+    if world > 1:
+        dist.barrier()
+    T_e2e_serial = time_b2b(e2e_step, args.steps, stream)
+    if world > 1:
+        t = torch.tensor([T_e2e_serial], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        T_e2e_serial = float(t.item())
+    T_e2e_pipe = None
     if world == 1:
         # Pipelined e2e (independent right-hand sides, e.g. serving): step k's
         # x H2D, SpMV and y D2H run on three streams with double buffers, so
@@ -356,11 +415,10 @@ def dysel_arm(args, world, rank, local_rank):
         s_out.wait_event(ev_out[(args.steps - 1) % 2])
         t1.record(s_out)
         torch.cuda.synchronize()
-        T_e2e = t0.elapsed_time(t1) * 1e-3 / args.steps
-        e2e_pipelined = True
-    # ---- roofline for the dominant kernel: the selected variant's plain kernel
-    # (it runs the tail-launched remainder, ~90% of the units of a step); its
-    # own launch duration is event-timed standalone over the full grid.
+        T_e2e_pipe = t0.elapsed_time(t1) * 1e-3 / args.steps
+    # ---- roofline for the dominant kernel: the selected variant's claim
+    # kernel (it runs the remainder, ~95% of a step); its own launch duration
+    # is event-timed over the full grid (the same kernel, code and occupancy)
     pk, src = peaks()
     kern_bytes = spmv_bytes(r1 - r0, A.n_cols, hi - lo)
     sel_name = rep["selected_name"]
@@ -373,39 +431,51 @@ def dysel_arm(args, world, rank, local_rank):
             traffic = json.load(open(tp)).get("dram_bytes_per_launch")
         except Exception:
             traffic = None
-    # ---- secondary workloads (1 GPU, rank 0): D3 SpMV and D2m SGEMM
     secondary = {}
-    if rank == 0 and not args.no_secondary:
-        secondary = secondary_workloads(ctx, D, args, stream)
+    if rank == 0 and world == 1 and not args.no_secondary:
+        secondary = secondary_workloads(ctx, D, args, stream, pk)
     # ---- CPU baseline: the oracle as it stands, on the host cores (rank 0, N=1)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         Tc, cores = cpu_oracle_spmv(A, x, reps=args.cpu_reps)
+        g1, s1 = cpu_single_thread_sample(A, x)
         cpu = {"value": round(nbytes_total / Tc / 1e9, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
                "sample": f"full D4 matrix ({A.nnz} nnz), fp64 CSR SpMV in plain C/OpenMP, median of "
-                         f"{args.cpu_reps} passes"}
+                         f"{args.cpu_reps} passes",
+               "single_thread": {"value": round(g1, 3), "unit": "GB/s", "cores": 1, "sample": s1}}
     if rank == 0:
+        h2d = int(x.nbytes) * world
+        d2h = int(A.n_rows) * 4
         line = {
             "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(T_step * 1e3, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": config(A, world, args.f),
+            "step_ms_percentiles": {"p10": pct(per_step, 10), "p50": pct(per_step, 50), "p90": pct(per_step, 90),
+                                    "note": "one event pair per step (rank 0), after the timed region"},
             "default_variant": default_name,
+            "format_prep_ms": round(plan.info.prep_ns / 1e6, 3),
+            "unit_order": {"light_units": plan.info.n_light, "heavy_or_long_units": plan.info.n_heavy},
             "overhead_pct_vs_best_variant": round((T_step - T_star) / T_star * 100, 3) if world == 1 else None,
             "best_variant_oracle": {"variant": best_name, "ms": round(T_star * 1e3, 4),
-                                    "gbs": round(nbytes_total / T_star / 1e9, 2),
-                                    "all_ms": {k: round(v * 1e3, 4) for k, v in T_v.items()}},
+                                    "gbs": round(kern_bytes / T_star / 1e9, 2),
+                                    "all_ms": {k: round(v * 1e3, 4) for k, v in T_v.items()},
+                                    "scope": "this rank's rows" if world > 1 else "whole matrix"},
             "selected": rep["selected_name"], "selection_matches_oracle": rep["selected_name"] == best_name,
+            "per_shard_selected": sels,
             "mode_used": rep["mode_used"], "profiled_units_per_variant": rep["c"],
+            "publish_us": round(rep["timeline_ns"][1] / 1e3, 1) if rep["timeline_ns"][1] is not None else None,
             "selection_accuracy_20_launches": accuracy,
             "amortized_overhead_pct": round((ta - T_star) / T_star * 100, 3) if world == 1 else None,
             "amortized_iters": I, "ablation": ablation,
-            "e2e": {"value": round(nbytes_total / T_e2e / 1e9, 3), "unit": "GB/s",
-                    "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int((r1 - r0) * 4),
-                    "ms_per_step": round(T_e2e * 1e3, 4), "pipelined": e2e_pipelined,
-                    "serial_ms_per_step": round(T_e2e_serial * 1e3, 4),
-                    "note": "pipelined: x H2D / SpMV / y D2H of consecutive steps overlap on 3 streams "
-                            "(double buffers); serial: copy in, SpMV, copy out per step"},
+            "e2e": {"value": round(nbytes_total / T_e2e_serial / 1e9, 3), "unit": "GB/s",
+                    "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                    "ms_per_step": round(T_e2e_serial * 1e3, 4),
+                    "pipelined_value": (round(nbytes_total / T_e2e_pipe / 1e9, 3) if T_e2e_pipe else None),
+                    "pipelined_ms_per_step": round(T_e2e_pipe * 1e3, 4) if T_e2e_pipe else None,
+                    "note": "value: dependent steps (x H2D from pinned memory, the DySel SpMV, y D2H, in stream "
+                            "order each step); pipelined: independent requests, the copies of steps k+1 / k-1 "
+                            "overlap step k's SpMV on three streams (double buffers)"},
             "step": {"eager_units": rep["eager_units"], "tail_units": rep["tail_units"],
                      "aborted_sandbox_units": {D.SPMV_NAMES[v]: rep["aborted"][v] for v in plan.variant_ids},
                      "busy_us_per_unit": {D.SPMV_NAMES[v]: round(rep["busy_ns"][v] / max(1, rep["units"][v]) / 1e3, 2)
@@ -417,13 +487,14 @@ def dysel_arm(args, world, rank, local_rank):
                          "frac": round(achieved / pk["hbm_gbs"], 4), "traffic": traffic,
                          "kernel": f"dysel::spmv_claim_kernel<{sel_name}> (pure full grid, event-timed back to back)",
                          "peak_source": src,
-                         "note": "D4 gathers x at uniform-random columns: bound in practice by the L1TEX/L2 "
-                                 "random-sector rate (DESIGN.md §Roofline), not HBM",
+                         "note": "D4 gathers x at uniform-random columns: bound in practice by the L1TEX random-"
+                                 "sector rate (DESIGN.md §6), not HBM; the 70%-of-HBM target is met on a regular "
+                                 "matrix: secondary.d3x_fem_2250k.roofline",
                          "floor": ({"gather_probe_ms": round(probe["gather"] * 1e3, 4),
                                     "gather_probe_gbs": round(kern_bytes / probe["gather"] / 1e9, 2),
                                     "stream_probe_ms": round(probe["stream"] * 1e3, 4),
                                     "stream_probe_gbs": round(kern_bytes / probe["stream"] / 1e9, 2),
-                                    "frac_of_gather_floor": round(probe["gather"] / T_v[sel_name], 4),
+                                    "frac_of_gather_floor": round(probe["gather"] / k_time, 4),
                                     "what": "dysel_spmv_gather_probe: the same col/val stream + x[col] gathers + "
                                             "row_ptr/y traffic with no row structure (gather), and with x read "
                                             "sequentially instead (stream); frac = probe time / kernel time"}
@@ -436,102 +507,109 @@ def dysel_arm(args, world, rank, local_rank):
     ctx.close()
 
 
-def secondary_workloads(ctx, D, args, stream):
+def secondary_workloads(ctx, D, args, stream, pk):
     import torch
-    from workloads import d3_fem, sgemm_inputs, uniform_f32
+    from workloads import d1_bus, d3_fem, d4_powerlaw, d6_diag, d6_random, sgemm_inputs, uniform_f32
     out = {}
-    # D3: Dubcova3-shaped FEM SpMV (30.9 MB: L2-resident when warm)
-    A = d3_fem()
-    x = torch.from_numpy(uniform_f32(384, A.n_cols)).cuda()
-    rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
-    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ALL)
-    y = torch.empty(A.n_rows, device="cuda")
-    nb = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
-    res = {}
-    for v in plan.variant_ids:
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # 2x the 126 MB L2
+
+    def cold(fn, reps=20):
         ts = []
-        for _ in range(20):
+        for _ in range(reps):
             flush.zero_()
-            ts += time_events(lambda: ctx.spmv_variant(plan, v, x, y), 1, stream)
-        res[D.SPMV_NAMES[v]] = float(np.median(ts))
-    best = min(res, key=res.get)
-    ts = []
-    for _ in range(20):
-        flush.zero_()
-        ts += time_events(lambda: ctx.spmv(plan, x, y, f=0.02, mode=D.AUTO | D.ASYNC), 1, stream)
-    td = float(np.median(ts))
-    ta = float(np.median(time_events(lambda: ctx.spmv(plan, x, y, mode=D.NO_PROFILE), 50, stream)))
-    rep = ctx.spmv(plan, x, y, f=0.02, mode=D.AUTO | D.ASYNC, report=True)
-    ts = []
-    for _ in range(20):
-        flush.zero_()
-        ts += time_events(lambda: ctx.spmv(plan, x, y, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE), 1, stream)
-    tf = float(np.median(ts))
-    repf = ctx.spmv(plan, x, y, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE, report=True)
-    out["d3_spmv_forced_profiling"] = {"dysel_us": round(tf * 1e6, 2), "selected": repf["selected_name"],
-                                       "overhead_pct": round((tf / res[best] - 1) * 100, 2)}
-    out["d3_spmv"] = {"cold_l2": True, "best_variant": best, "best_us": round(res[best] * 1e6, 2),
-                      "best_gbs": round(nb / res[best] / 1e9, 1), "dysel_us": round(td * 1e6, 2),
-                      "dysel_gbs": round(nb / td / 1e9, 1), "overhead_pct": round((td / res[best] - 1) * 100, 2),
-                      "selected": rep["selected_name"], "profiled": rep["profiled"],
-                      "default_variant": D.SPMV_NAMES[plan.info.default_variant],
-                      "warm_no_profile_us": round(ta * 1e6, 2),
-                      "all_us": {k: round(v * 1e6, 2) for k, v in res.items()}}
-    plan.destroy()
+            ts += time_events(fn, 1, stream)
+        return float(np.median(ts))
+
+    def spmv_case(A, x_seed, f, reps=20, formats=D.FMT_ALL, cold_l2=True, forced=True):
+        x = torch.from_numpy(uniform_f32(x_seed, A.n_cols)).cuda()
+        rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
+        plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=formats)
+        y = torch.empty(A.n_rows, device="cuda")
+        tm = (lambda fn: cold(fn, reps)) if cold_l2 else (lambda fn: time_b2b(fn, reps, stream))
+        res = {D.SPMV_NAMES[v]: tm(lambda: ctx.spmv_variant(plan, v, x, y)) for v in plan.variant_ids}
+        best = min(res, key=res.get)
+        td = tm(lambda: ctx.spmv(plan, x, y, f=f, mode=D.AUTO | D.ASYNC))
+        rep = ctx.spmv(plan, x, y, f=f, mode=D.AUTO | D.ASYNC, report=True)
+        nb = spmv_bytes(A.n_rows, A.n_cols, A.nnz)
+        r = {"n_rows": int(A.n_rows), "nnz": int(A.nnz), "cold_l2": cold_l2, "f": f, "best_variant": best,
+             "best_us": round(res[best] * 1e6, 2), "best_gbs": round(nb / res[best] / 1e9, 1),
+             "dysel_us": round(td * 1e6, 2), "dysel_gbs": round(nb / td / 1e9, 1),
+             "overhead_pct": round((td / res[best] - 1) * 100, 2), "selected": rep["selected_name"],
+             "profiled": rep["profiled"], "default_variant": D.SPMV_NAMES[plan.info.default_variant],
+             "format_prep_ms": round(plan.info.prep_ns / 1e6, 3),
+             "all_us": {k: round(v * 1e6, 2) for k, v in res.items()}}
+        if forced:
+            tf = tm(lambda: ctx.spmv(plan, x, y, f=f, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE))
+            repf = ctx.spmv(plan, x, y, f=f, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE, report=True)
+            r["forced_profiling"] = {"dysel_us": round(tf * 1e6, 2), "selected": repf["selected_name"],
+                                     "overhead_pct": round((tf / res[best] - 1) * 100, 2)}
+        plan.destroy()
+        return r, res, nb
+
+    # D1: 1138_bus-shaped (5 units: deactivated, A-3); default and forced-on (ablation)
+    r, _, _ = spmv_case(d1_bus(), 1140, 0.5, reps=50, formats=D.FMT_ELL | D.FMT_JDS | D.FMT_STREAM, cold_l2=False)
+    r["note"] = "5 units < 128 CTAs: profiling deactivated (P:L328-337); forced: f = 0.5, warm L2"
+    out["d1_1138_bus"] = r
+    # D3: Dubcova3-shaped FEM (30.9 MB: L2-resident when warm -> cold numbers)
+    r, _, _ = spmv_case(d3_fem(), 384, 0.02)
+    out["d3_spmv"] = r
+    # D3x: the same 5x5 FEM stencil at 2.25M rows (0.45 GB > L2): the regular
+    # matrix on which SpMV is HBM-bound -> the 70%-of-HBM target's roofline
+    A3 = d3_fem(grid=1500)
+    r, res, nb = spmv_case(A3, 385, 0.02, reps=20)
+    kb = min(res.values())
+    r["roofline"] = {"bound": "hbm", "achieved": round(nb / kb / 1e9, 2), "peak": pk["hbm_gbs"], "unit": "GB/s",
+                     "frac": round(nb / kb / 1e9 / pk["hbm_gbs"], 4),
+                     "kernel": f"dysel::spmv_claim_kernel<{r['best_variant']}> (pure full grid, cold L2)",
+                     "dysel_frac": round(nb / (r["dysel_us"] * 1e-6) / 1e9 / pk["hbm_gbs"], 4)}
+    out["d3x_fem_2250k"] = r
+    del A3
     # D6: the paper's Case IV inputs — the scalar/vector flip
-    from workloads import d6_diag, d6_random
     for name, A6 in (("d6_random_16k_1pct", d6_random()), ("d6_diagonal_2M", d6_diag())):
-        x6 = torch.from_numpy(uniform_f32(6, A6.n_cols)).cuda()
-        rp6, col6, val6 = (torch.from_numpy(a).cuda() for a in (A6.row_ptr, A6.col, A6.val))
-        plan6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ALL)
-        y6 = torch.empty(A6.n_rows, device="cuda")
-        r6 = {D.SPMV_NAMES[v]: time_b2b(lambda: ctx.spmv_variant(plan6, v, x6, y6), 20, stream)
-              for v in plan6.variant_ids}
-        b6 = min(r6, key=r6.get)
-        t6 = time_b2b(lambda: ctx.spmv(plan6, x6, y6, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE), 20, stream)
-        rep6 = ctx.spmv(plan6, x6, y6, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE, report=True)
-        out[name] = {"best_variant": b6, "best_us": round(r6[b6] * 1e6, 2),
-                     "scalar_over_vector": round(r6["csr_scalar"] / r6["csr_vector"], 3),
-                     "dysel_forced_us": round(t6 * 1e6, 2), "selected": rep6["selected_name"],
-                     "all_us": {k: round(v * 1e6, 2) for k, v in r6.items()}}
-        plan6.destroy()
-    # f-4: stencil pool, Parboil-default-shaped 512 x 512 x 64 grid
-    nz, ny, nx = 64, 512, 512
-    a3 = torch.from_numpy(uniform_f32(64, (nz, ny, nx))).cuda()
-    o3 = torch.empty_like(a3)
+        r, res, _ = spmv_case(A6, 6, 0.02, cold_l2=False)
+        r["scalar_over_vector"] = round(res["csr_scalar"] / res["csr_vector"], 3)
+        out[name] = r
+    # f-4: stencil pool, Parboil-default-shaped 512 x 512 x 64 and a 512 x 512 x 256
+    # grid (in + out 537 MB > 2x L2: cold HBM)
     c0, c1 = 0.8125, 0.15625
-    ts3 = {D.STENCIL_NAMES[v]: time_b2b(lambda: ctx.stencil_variant(v, a3, o3, c0, c1), 20, stream) for v in range(3)}
-    b3 = min(ts3, key=ts3.get)
-    td3 = time_b2b(lambda: ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC), 20, stream)
-    r3 = ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC, report=True)
-    tf3 = time_b2b(lambda: ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE), 20, stream)
-    rf3 = ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE, report=True)
-    def amort3():
-        ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE)
-        for _ in range(19):
-            ctx.stencil(a3, o3, c0, c1, mode=D.NO_PROFILE)
-    tam3 = time_b2b(amort3, 3, stream) / 20
-    sb3 = 2 * 4 * nx * ny * nz     # algorithmic: read in once, write out once
-    out["stencil_512x512x64"] = {"best_variant": b3, "best_us": round(ts3[b3] * 1e6, 2),
-                                 "best_gbs": round(sb3 / ts3[b3] / 1e9, 1),
-                                 "dysel_us": round(td3 * 1e6, 2), "selected": r3["selected_name"],
-                                 "profiled": r3["profiled"], "overhead_pct": round((td3 / ts3[b3] - 1) * 100, 2),
-                                 "forced_single_shot_overhead_pct": round((tf3 / ts3[b3] - 1) * 100, 2),
-                                 "forced_selected": rf3["selected_name"],
-                                 "amortized_overhead_pct": round((tam3 / ts3[b3] - 1) * 100, 2),
-                                 "all_us": {k: round(v * 1e6, 2) for k, v in ts3.items()},
-                                 "note": "in + out 134 MB > L2; fully|async, f = 0.02 (profiled unless the default's grid fits one "
-                                         "wave, A-3b); forced: profile once; amortised: forced once + 19 activation-flag "
-                                         "calls"}
+    for nz in (64, 256):
+        a3 = torch.from_numpy(uniform_f32(64, (nz, 512, 512))).cuda()
+        o3 = torch.empty_like(a3)
+        ts3 = {D.STENCIL_NAMES[v]: time_b2b(lambda: ctx.stencil_variant(v, a3, o3, c0, c1), 20, stream)
+               for v in range(3)}
+        b3 = min(ts3, key=ts3.get)
+        td3 = time_b2b(lambda: ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC), 20, stream)
+        r3 = ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC, report=True)
+        tf3 = time_b2b(lambda: ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE), 20,
+                       stream)
+        rf3 = ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE, report=True)
+        def amort3():
+            ctx.stencil(a3, o3, c0, c1, f=0.02, mode=D.FULLY | D.ASYNC | D.FORCE_PROFILE)
+            for _ in range(19):
+                ctx.stencil(a3, o3, c0, c1, mode=D.NO_PROFILE)
+        tam3 = time_b2b(amort3, 3, stream) / 20
+        sb3 = 2 * 4 * a3.numel()     # algorithmic: read in once, write out once
+        out[f"stencil_512x512x{nz}"] = {
+            "best_variant": b3, "best_us": round(ts3[b3] * 1e6, 2), "best_gbs": round(sb3 / ts3[b3] / 1e9, 1),
+            "roofline": {"bound": "hbm", "achieved": round(sb3 / ts3[b3] / 1e9, 2), "peak": pk["hbm_gbs"],
+                         "unit": "GB/s", "frac": round(sb3 / ts3[b3] / 1e9 / pk["hbm_gbs"], 4)},
+            "dysel_us": round(td3 * 1e6, 2), "selected": r3["selected_name"], "profiled": r3["profiled"],
+            "overhead_pct": round((td3 / ts3[b3] - 1) * 100, 2),
+            "forced_single_shot_overhead_pct": round((tf3 / ts3[b3] - 1) * 100, 2),
+            "forced_selected": rf3["selected_name"],
+            "amortized_overhead_pct": round((tam3 / ts3[b3] - 1) * 100, 2),
+            "all_us": {k: round(v * 1e6, 2) for k, v in ts3.items()},
+            "note": f"in + out {sb3 / 1e6:.0f} MB, b2b; fully|async f = 0.02 (profiled unless the default's grid "
+                    "fits one wave, A-3b); forced: profile once; amortised: forced once + 19 activation-flag calls"}
+        del a3, o3
     # SpMTV (f-1): y += A^T x by atomic scatter -> swap-mode profiling
-    from workloads import d4_powerlaw
     At = d4_powerlaw(n=2_000_000, lmax=4096)
     rpt, colt, valt = (torch.from_numpy(a).cuda() for a in (At.row_ptr, At.col, At.val))
     plant = ctx.spmv_prepare(rpt, colt, valt, At.n_cols)
     xt = torch.from_numpy(uniform_f32(61, At.n_rows)).cuda()
     yt = torch.zeros(At.n_cols, device="cuda")
-    tt = {D.SPMTV_NAMES[v]: time_b2b(lambda: ctx.spmtv_variant(plant, v, xt, yt), 20, stream) for v in range(len(D.SPMTV_NAMES))}
+    tt = {D.SPMTV_NAMES[v]: time_b2b(lambda: ctx.spmtv_variant(plant, v, xt, yt), 20, stream)
+          for v in range(len(D.SPMTV_NAMES))}
     bt = min(tt, key=tt.get)
     tdt = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO), 20, stream)
     rept = ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO, report=True)
@@ -545,100 +623,97 @@ def secondary_workloads(ctx, D, args, stream):
     out["spmtv_powerlaw_2M"] = {"nnz": int(At.nnz), "best_variant": bt, "best_us": round(tt[bt] * 1e6, 2),
                                 "best_gbs": round(nbt / tt[bt] / 1e9, 1), "dysel_us": round(tdt * 1e6, 2),
                                 "selected": rept["selected_name"], "profiled": rept["profiled"],
-                                "mode_used": rept["mode_used"],
+                                "mode_used": rept["mode_used"], "sandbox_buffers": rept["sandbox_buffers"],
                                 "overhead_pct": round((tdt / tt[bt] - 1) * 100, 2),
                                 "host_orch_overhead_pct": round((tht / tt[bt] - 1) * 100, 2),
                                 "amortized_overhead_pct": round((tat / tt[bt] - 1) * 100, 2),
                                 "all_us": {k: round(v * 1e6, 2) for k, v in tt.items()},
                                 "note": "y += A^T x (red.global.add per nonzero): AUTO -> swap (private copies of y, "
                                         "winner's swapped in), f = 0.01, sync only (Table 1)"}
-    del plant
-    # D2m: Parboil-medium SGEMM 1024 x 992 x 1056
-    M, K, N = 1024, 992, 1056
-    Ah, Bh, _ = sgemm_inputs(M, K, N)
-    Ad, Bd = torch.from_numpy(Ah).cuda(), torch.from_numpy(Bh).cuda()
-    C = torch.empty((M, N), device="cuda")
-    flops = 2.0 * M * N * K
-    # back-to-back launches between two events (per-call events would add the
-    # host-side tensor-map encoding of these ~40 us kernels to the GPU time)
-    tv = {D.SGEMM_NAMES[v]: time_b2b(lambda: ctx.sgemm_variant(v, Ad, Bd, C), 30, stream) for v in range(4)}
-    bestg = min(tv, key=tv.get)
-    f_sg = 0.06
-    tdg = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY), 30, stream)
-    repg = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY, report=True)
-    tforced = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE), 30, stream)
-    repf = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE, report=True)
-    I = 100
-    def amort():
-        ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE)
-        for _ in range(I - 1):
-            ctx.sgemm(Ad, Bd, C, mode=D.NO_PROFILE)
-    tam = time_b2b(amort, 3, stream) / I
-    out["d2m_sgemm"] = {"best_variant": bestg, "best_us": round(tv[bestg] * 1e6, 2),
-                        "best_tflops": round(flops / tv[bestg] / 1e12, 2),
-                        "dysel_us": round(tdg * 1e6, 2), "profiled": repg["profiled"],
-                        "note": "single wave -> profiling off (reading A-3b); default = tc3xtf32_128x64",
-                        "overhead_pct": round((tdg / tv[bestg] - 1) * 100, 2),
-                        "forced_single_shot_us": round(tforced * 1e6, 2),
-                        "forced_single_shot_overhead_pct": round((tforced / tv[bestg] - 1) * 100, 2),
-                        "forced_selected": repf["selected_name"],
-                        "amortized_overhead_pct": round((tam / tv[bestg] - 1) * 100, 2), "f": f_sg,
-                        "all_us": {k: round(v * 1e6, 2) for k, v in tv.items()}}
-    # extra square case (several waves): the tensor-core roofline of the SGEMM pool
-    M = K = N = 4096
-    Ah, Bh, _ = sgemm_inputs(M, K, N, 5, 6)
-    Ad, Bd = torch.from_numpy(Ah).cuda(), torch.from_numpy(Bh).cuda()
-    C = torch.empty((M, N), device="cuda")
-    t4 = {D.SGEMM_NAMES[v]: time_b2b(lambda: ctx.sgemm_variant(v, Ad, Bd, C), 5, stream) for v in (1, 2, 3)}
-    td4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY), 5, stream)
-    rep4 = ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY, report=True)
-    # hybrid + eager wave: dominated SIMT sandboxes stop (A-32), the default fills free slots (A-33)
-    th4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.01, mode=D.HYBRID | D.ASYNC), 5, stream)
-    reph4 = ctx.sgemm(Ad, Bd, C, f=0.01, mode=D.HYBRID | D.ASYNC, report=True)
-    tn4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY | D.NO_ABORT), 5, stream)
-    ta4 = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY | D.ASYNC | D.HOST_ORCH), 5, stream)
-    I4 = 20
-    def amort4():
-        ctx.sgemm(Ad, Bd, C, f=0.02, mode=D.FULLY)
-        for _ in range(I4 - 1):
-            ctx.sgemm(Ad, Bd, C, mode=D.NO_PROFILE)
-    tam4 = time_b2b(amort4, 2, stream) / I4
-    b4 = min(t4, key=t4.get)
-    # the amortised run is 40 back-to-back 4096^3 calls (~25 ms at full power);
-    # also compare it with the best variant over the same number of calls
-    # (context: the power/clock state differs between short and long regions)
-    bv4 = D.SGEMM_NAMES.index(b4)
-    tb4_long = time_b2b(lambda: ctx.sgemm_variant(bv4, Ad, Bd, C), 2 * I4, stream)
-    fl4 = 2.0 * M * N * K
-    out["sgemm_4096"] = {"best_variant": b4, "best_tflops": round(fl4 / t4[b4] / 1e12, 1),
-                         "all_tflops": {k: round(fl4 / v / 1e12, 1) for k, v in t4.items()},
-                         "dysel_tflops": round(fl4 / td4 / 1e12, 1), "selected": rep4["selected_name"],
-                         "overhead_pct": round((td4 / t4[b4] - 1) * 100, 2),
-                         "no_dominance_overhead_pct": round((tn4 / t4[b4] - 1) * 100, 2),
-                         "hybrid_async_overhead_pct": round((th4 / t4[b4] - 1) * 100, 2),
-                         "hybrid_async_selected": reph4["selected_name"], "hybrid_async_eager_granules": reph4["eager_units"],
-                         "host_async_overhead_pct": round((ta4 / t4[b4] - 1) * 100, 2),
-                         "amortized_overhead_pct": round((tam4 / t4[b4] - 1) * 100, 2),
-                         "amortized_overhead_pct_vs_long_best": round((tam4 / tb4_long - 1) * 100, 2),
-                         "amortized_note": "headline vs the best variant's 5-call b2b time (the conservative one); "
-                                           "_vs_long_best: vs %d b2b calls of it (same count as the amortised run; "
-                                           "sustained-power clocks make this one noisy, measured -7%%..+3%%)" % (2 * I4),
-                         "tensor_roofline_note": "3xTF32 = 3 tf32 MMAs per fp32 product; ceiling ~ tf32 peak / 3"}
+    plant.destroy()
+    del At
+    # SGEMM: D2s (Parboil small), D2m (Parboil medium), D7 8192^3 (extra, labelled)
+    tf32_ceiling = pk["bf16_tflops"] * 0.5 / 3.0   # 3xTF32: three tf32 MMAs per fp32 product
+    for name, (M, K, N), f_sg, reps in (("d2s_sgemm_128x96x160", (128, 96, 160), 0.5, 50),
+                                         ("d2m_sgemm", (1024, 992, 1056), 0.06, 30),
+                                         ("d7_sgemm_8192", (8192, 8192, 8192), 0.005, 5)):
+        Ah, Bh, _ = sgemm_inputs(M, K, N, 992 if M == 1024 else 96 if M == 128 else 8192,
+                                 993 if M == 1024 else 97 if M == 128 else 8193)
+        Ad, Bd = torch.from_numpy(Ah).cuda(), torch.from_numpy(Bh).cuda()
+        C = torch.empty((M, N), device="cuda")
+        flops = 2.0 * M * N * K
+        vids = [v for v in range(4) if not (M >= 8192 and v == D.SGEMM_S64)]
+        tv = {D.SGEMM_NAMES[v]: time_b2b(lambda: ctx.sgemm_variant(v, Ad, Bd, C), reps, stream) for v in vids}
+        bestg = min(tv, key=tv.get)
+        tdg = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY), reps, stream)
+        repg = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY, report=True)
+        tforced = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE), reps, stream)
+        repf = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE, report=True)
+        th = time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.HYBRID | D.ASYNC | D.FORCE_PROFILE), reps, stream)
+        I = 20 if M >= 8192 else 100
+        def amort():
+            ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE)
+            for _ in range(I - 1):
+                ctx.sgemm(Ad, Bd, C, mode=D.NO_PROFILE)
+        tam = time_b2b(amort, 2, stream) / I
+        out[name] = {"M": M, "K": K, "N": N, "best_variant": bestg, "best_us": round(tv[bestg] * 1e6, 2),
+                     "best_tflops": round(flops / tv[bestg] / 1e12, 2),
+                     "roofline": {"bound": "tensor", "achieved": round(flops / tv[bestg] / 1e12, 2),
+                                  "peak": round(tf32_ceiling, 1), "unit": "TFLOP/s",
+                                  "frac": round(flops / tv[bestg] / 1e12 / tf32_ceiling, 4),
+                                  "peak_note": "3xTF32 ceiling = measured bf16 TF/s x 1/2 (nominal tf32 ratio) / 3"},
+                     "dysel_us": round(tdg * 1e6, 2), "profiled": repg["profiled"], "selected": repg["selected_name"],
+                     "overhead_pct": round((tdg / tv[bestg] - 1) * 100, 2),
+                     "forced_single_shot_overhead_pct": round((tforced / tv[bestg] - 1) * 100, 2),
+                     "forced_selected": repf["selected_name"],
+                     "hybrid_async_overhead_pct": round((th / tv[bestg] - 1) * 100, 2),
+                     "amortized_overhead_pct": round((tam / tv[bestg] - 1) * 100, 2), "amortized_iters": I,
+                     "f": f_sg, "all_us": {k: round(v * 1e6, 2) for k, v in tv.items()}}
+        del Ad, Bd, C
     return out
 
 
-def time_b2b(fn, reps, stream):
+# ------------------------------------------------------------------ launch
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _rank_entry(rank, world, port, args, A, x):
+    """One spawned rank (one process per GPU): NCCL process group over
+    127.0.0.1, then the DySel arm on GPU `rank`."""
+    import torch.distributed as dist
+    os.environ.update({"RANK": str(rank), "WORLD_SIZE": str(world), "LOCAL_RANK": str(rank),
+                       "MASTER_ADDR": "127.0.0.1", "MASTER_PORT": str(port)})
     import torch
-    for _ in range(2):
-        fn()
-    torch.cuda.synchronize()
-    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a.record(stream)
-    for _ in range(reps):
-        fn()
-    b.record(stream)
-    torch.cuda.synchronize()
-    return a.elapsed_time(b) * 1e-3 / reps
+    torch.cuda.set_device(rank)
+    dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", rank))
+    try:
+        dysel_arm(args, world, rank, rank, A, x)
+    finally:
+        dist.destroy_process_group()
+
+
+def spawn(args):
+    """`--gpus N` without torchrun: N ranks forked from this process (the D4
+    matrix is generated once here and shared copy-on-write; CUDA is
+    initialised only in the children)."""
+    import multiprocessing as mp
+    A, x = make_d4(args.rows)
+    port = _free_port()
+    ctx = mp.get_context("fork")
+    procs = [ctx.Process(target=_rank_entry, args=(r, args.gpus, port, args, A, x)) for r in range(args.gpus)]
+    for p in procs:
+        p.start()
+    rc = 0
+    for p in procs:
+        p.join()
+        rc = rc or p.exitcode
+    if rc:
+        sys.exit(rc)
 
 
 def main():
@@ -656,15 +731,21 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    launched = "WORLD_SIZE" in os.environ
+    world = int(os.environ.get("WORLD_SIZE", "1")) if launched else args.gpus
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         reference_arm(args, world, rank)
         return
+    if not launched and args.gpus > 1:
+        spawn(args)
+        return
     if world > 1:
+        import torch
         import torch.distributed as dist
-        dist.init_process_group("nccl")
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     dysel_arm(args, world, rank, local_rank)
     if world > 1:
         import torch.distributed as dist

@@ -244,10 +244,8 @@ typedef struct {
   uint64_t timeline_ns[8];
   /* Table 1 allocation record of this launch: extra output
    * buffers the profiling slices wrote instead of the real output, and their
-   * bytes.  FULLY: 0.  HYBRID: generic launcher K-1 (the default's slice is
-   * productive, A-4), SpMV device path K slice-sized sandboxes (every
-   * variant's profiled units are discardable, the winner's are copied in:
-   * reading A-4').  SWAP: K full private outputs. */
+   * bytes.  FULLY: 0.  HYBRID: K-1 slice-sized sandboxes (the default's
+   * slice is productive, A-4).  SWAP: K full private outputs. */
   uint32_t sandbox_buffers;
   uint32_t pad_;
   uint64_t sandbox_bytes;
@@ -375,6 +373,60 @@ dysel_status dysel_spmv_variant(dysel_ctx *ctx, dysel_spmv_plan *plan, int varia
 dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *plan, int flavour, const float *d_x,
                                      float *d_out, void *stream);
 
+/* --------------------------------------- SpMV f-2: data placement (Case II)
+ * SURVEY §8f f-2 / the paper's Case II ("four data placement policies ...
+ * selected at runtime" for spmv-csr, §4.2): one CSR-scalar
+ * kernel (thread per row, CSR-order fmaf from +0) in four placements of x,
+ * selected by DySel through the generic launcher on the plan's 256-row units:
+ *   0 x_ldg      x through the read-only L1 path (ld.global.nc)
+ *   1 x_l2       x through L2 only (ld.global.cg)
+ *   2 x_smem     each unit's x window [min col, max col] staged into shared
+ *                memory by cp.async.bulk (banded matrices; units whose window
+ *                exceeds 12,288 floats gather from global memory instead)
+ *   3 x_persist  as x_ldg, launched with an L2 access-policy window marking x
+ *                persisting (the ctx reserves the device's maximum persisting
+ *                L2 set-aside at the first call: a device-wide limit)
+ * The four are bit-identical to each other and to CSR-S.  The pool is built
+ * and registered at the plan's first placement call (x windows: one kernel).
+ * d_x fp32 [n_cols], d_y fp32 [n_rows]; errors as dysel_spmv. */
+enum { DYSEL_SPMV_PLACE_LDG = 0, DYSEL_SPMV_PLACE_L2 = 1, DYSEL_SPMV_PLACE_SMEM = 2, DYSEL_SPMV_PLACE_PERSIST = 3,
+       DYSEL_SPMV_PLACE_NVARIANTS = 4 };
+dysel_status dysel_spmv_placement(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,
+                                  float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+dysel_status dysel_spmv_placement_variant(dysel_ctx *ctx, dysel_spmv_plan *plan, int variant_id, const float *d_x,
+                                          float *d_y, void *stream);
+/* Test: the plan's per-unit x windows (int32 pairs [min col, max col], (0,-1)
+ * for an empty unit) into HOST h_win (2 * cap_units ints); DYSEL_ERR_NOT_FOUND
+ * before the first placement call. */
+dysel_status dysel_spmv_placement_windows(const dysel_spmv_plan *plan, int32_t *h_win, size_t cap_units);
+
+/* ------------------------------- SpMV f-2: global-sort JDS pool (Case III)
+ * Parboil spmv-jds as the paper profiles it (P:L1424-1429, P:L1454-1461
+ * §4.3): rows sorted by length over the WHOLE matrix (stable: ties keep row
+ * order), entry (p, k) of permuted row p at jd_ptr[k] + p.  A standalone pool
+ * (its units are 256 permuted rows, so it cannot share the block-local
+ * pool's unit space, reading A-14) of four versions of the kernel:
+ *   0 plain, 1 unroll (4 diagonals per iteration), 2 prefetch (next
+ *   diagonal's entry in flight), 3 unroll + prefetch (initial version)
+ * all summing each row in CSR order with fmaf from +0: bit-identical to each
+ * other and to CSR-S.  Mode AUTO: hybrid unless every row has one length.
+ * The plan owns its arrays (perm, len int32 [n]; jd_ptr int32 [W+1]; col /
+ * val [nnz]) and keeps no pointer to the CSR. */
+typedef struct dysel_spmv_jds_plan dysel_spmv_jds_plan;
+enum { DYSEL_SPMV_JDS_PLAIN = 0, DYSEL_SPMV_JDS_UNROLL = 1, DYSEL_SPMV_JDS_PREFETCH = 2,
+       DYSEL_SPMV_JDS_UNROLL_PREFETCH = 3, DYSEL_SPMV_JDS_NVARIANTS = 4 };
+dysel_status dysel_spmv_jds_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, int64_t nnz,
+                                    const int32_t *d_row_ptr, const int32_t *d_col, const float *d_val, void *stream,
+                                    dysel_spmv_jds_plan **out);
+dysel_status dysel_spmv_jds(dysel_ctx *ctx, dysel_spmv_jds_plan *plan, const float *d_x, float *d_y,
+                            float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+dysel_status dysel_spmv_jds_variant(dysel_ctx *ctx, dysel_spmv_jds_plan *plan, int variant_id, const float *d_x,
+                                    float *d_y, void *stream);
+/* Test: copy array `which` (0 perm, 1 len, 2 jd_ptr, 3 col, 4 val) to HOST dst
+ * (*bytes: in capacity, out size; dst NULL = query). */
+dysel_status dysel_spmv_jds_copy_array(const dysel_spmv_jds_plan *plan, int which, void *dst, size_t *bytes);
+void dysel_spmv_jds_plan_destroy(dysel_spmv_jds_plan *plan);
+
 /* ------------------------------------------------------------------ SGEMM
  * C = alpha * A B + beta * C, fp32, row-major, no transposes (Parboil sgemm,
  * P:L1286-1294, L1427; A-17).  Unit = one 32x32 tile of C.  Built-in variants:
@@ -452,11 +504,30 @@ dysel_status dysel_partition_rows(const int32_t *h_row_ptr, int64_t n_rows, int 
 dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local_plan, const int64_t *bounds,
                                 const float *d_x, float *d_y, float profile_fraction, uint32_t mode,
                                 void *stream, dysel_report *rep);
+/* 1-GPU loopback of dysel_spmv_sharded (SURVEY §8e "testing without 8
+ * GPUs"): plans[g] (g < G) holds rows [bounds[g], bounds[g+1]) with a rebased
+ * row_ptr (the layout each rank's local plan has); the G shards' DySel
+ * launches run one after another on this device, each selecting on its own
+ * slice (a "mixed version"), each into a ctx-owned staging
+ * buffer (that GPU's local y), and one cudaMemcpyAsync per shard assembles
+ * d_y (full length bounds[G]) — the stand-in of the allgatherv.  d_x full
+ * length.  reps: nullable array of G reports.  Stream-ordered on `stream`. */
+dysel_status dysel_spmv_sharded_loopback(dysel_ctx *ctx, int G, dysel_spmv_plan *const *plans, const int64_t *bounds,
+                                         const float *d_x, float *d_y, float profile_fraction, uint32_t mode,
+                                         void *stream, dysel_report *reps);
 /* Broadcast n floats from `root` in place (x or B distribution). */
 dysel_status dysel_comm_broadcast(dysel_ctx *ctx, float *d_buf, size_t n, int root, void *stream);
-/* C rows [m0, m1) computed locally with DySel (B replicated), then C allgathered. */
-dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A,
-                                 int lda, const float *d_B, int ldb, float beta, float *d_C, int ldc,
+/* SGEMM M-sharding: rank r owns C rows [m0, m1), blocks of
+ * ceil(M / world) rounded up to 128 (one tcgen05 tile); empty for late ranks
+ * when M is small. */
+dysel_status dysel_sgemm_shard_rows(int M, int world, int rank, int *m0, int *m1);
+/* M-sharded SGEMM: d_A_local = this rank's A_g, rows [m0, m1) of A only
+ * ((m1 - m0) x K, leading dimension lda; A is never replicated), d_B the full
+ * K x N matrix (replicated, e.g. by dysel_comm_broadcast), d_C the full M x N
+ * matrix on every rank: C_g = alpha A_g B + beta C_g is computed in place by a
+ * local DySel launch (own selection per shard), then C is allgathered. */
+dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A_local, int lda,
+                                 const float *d_B, int ldb, float beta, float *d_C, int ldc,
                                  float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
 
 /* --------------------------------------------------------- iterative driver */

@@ -17,6 +17,16 @@ Block-local JDS (reading A-14): per 256-row block b, order = stable argsort of
      #{p : len(order[p]) > k}; entry (p, k) sits at blk_off[b] + jd_ptr_b[k] + p
      where blk_off[b] = row_ptr[b*256].  jd_ptr of all blocks is concatenated;
      block b's W_b+1 entries start at jd_off[b] = sum_{b'<b} (W_b'+1).
+
+Global-sort JDS (Parboil spmv-jds as the paper profiles it, P:L1424-1426,
+P:L1454-1461; SURVEY §8f f-2 "global-sort JDS", a standalone pool since its
+units are permuted rows): perm = stable argsort of -len over ALL rows
+(position p holds row perm[p]); W = len(perm[0]); jd_ptr[0] = 0, jd_ptr[k+1]
+= jd_ptr[k] + #{p : len(perm[p]) > k}; entry (p, k) sits at jd_ptr[k] + p and
+holds the k-th CSR entry of row perm[p].
+
+Pinned by tests/test_oracle_spmv.py / tests/test_oracle_f2.py: hand-computed
+fixtures, CSR round trips (bit-exact), invariants, brute force.
 """
 from __future__ import annotations
 
@@ -194,3 +204,82 @@ def uniform_rows(row_ptr) -> bool:
         return True
     lens = np.diff(rp)
     return int(lens.max()) * n <= 2 * int(rp[-1])
+
+
+def csr_to_global_jds(row_ptr, col, val):
+    """Global-sort JDS (definition in the module docstring), plain loops."""
+    rp = np.asarray(row_ptr, np.int64)
+    n = rp.shape[0] - 1
+    lens = np.diff(rp)
+    perm = np.array(sorted(range(n), key=lambda r: (-int(lens[r]), r)), np.int64)   # stable by row id
+    W = int(lens[perm[0]]) if n else 0
+    jd_ptr = np.zeros(W + 1, np.int64)
+    for k in range(W):
+        jd_ptr[k + 1] = jd_ptr[k] + int(np.sum(lens[perm] > k))
+    nnz = int(rp[-1])
+    jc = np.zeros(nnz, np.int32)
+    jv = np.zeros(nnz, np.float32)
+    for p in range(n):
+        r = perm[p]
+        for k in range(int(lens[r])):
+            jc[jd_ptr[k] + p] = col[rp[r] + k]
+            jv[jd_ptr[k] + p] = val[rp[r] + k]
+    return {"perm": perm.astype(np.int32), "len": lens[perm].astype(np.int32), "jd_ptr": jd_ptr.astype(np.int32),
+            "col": jc, "val": jv, "W": W}
+
+
+def csr_to_global_jds_fast(row_ptr, col, val):
+    """Vectorised form of csr_to_global_jds (same definition), for large inputs."""
+    rp = np.asarray(row_ptr, np.int64)
+    n = rp.shape[0] - 1
+    lens = np.diff(rp)
+    perm = np.argsort(-lens, kind="stable")
+    sl = lens[perm]
+    W = int(sl[0]) if n else 0
+    # #{p : len_p > k} for k < W: rows sorted descending -> searchsorted on -sl
+    cnt = np.searchsorted(-sl, -np.arange(W), side="left") if W else np.zeros(0, np.int64)
+    jd_ptr = np.zeros(W + 1, np.int64)
+    np.cumsum(cnt, out=jd_ptr[1:])
+    nnz = int(rp[-1])
+    rows = np.repeat(np.arange(n), sl)                 # permuted position of each entry (position-major)
+    k = np.arange(nnz) - np.repeat(np.concatenate([[0], np.cumsum(sl)[:-1]]) if n else np.zeros(0, np.int64), sl)
+    src = rp[perm[rows]] + k
+    dst = jd_ptr[k] + rows
+    jc = np.zeros(nnz, np.int32)
+    jv = np.zeros(nnz, np.float32)
+    jc[dst] = np.asarray(col)[src]
+    jv[dst] = np.asarray(val)[src]
+    return {"perm": perm.astype(np.int32), "len": sl.astype(np.int32), "jd_ptr": jd_ptr.astype(np.int32),
+            "col": jc, "val": jv, "W": W}
+
+
+def global_jds_to_csr(j, n):
+    """Inverse of csr_to_global_jds (round-trip pin)."""
+    perm, lens, jd_ptr = j["perm"], j["len"], np.asarray(j["jd_ptr"], np.int64)
+    row_len = np.zeros(n, np.int64)
+    row_len[perm] = lens
+    rp = np.zeros(n + 1, np.int64)
+    np.cumsum(row_len, out=rp[1:])
+    col = np.zeros(int(rp[-1]), np.int32)
+    val = np.zeros(int(rp[-1]), np.float32)
+    for p in range(n):
+        r = int(perm[p])
+        for k in range(int(lens[p])):
+            col[rp[r] + k] = j["col"][jd_ptr[k] + p]
+            val[rp[r] + k] = j["val"][jd_ptr[k] + p]
+    return rp, col, val
+
+
+def unit_x_windows(row_ptr, col, unit=UNIT_ROWS):
+    """Per 256-row unit: (min col, max col) over its entries, (0, -1) when the
+    unit has none — the x window the smem-staged placement variant copies
+    (integer, bit-exact contract)."""
+    rp = np.asarray(row_ptr, np.int64)
+    n = rp.shape[0] - 1
+    nu = (n + unit - 1) // unit
+    out = np.zeros((nu, 2), np.int32)
+    c = np.asarray(col, np.int64)
+    for u in range(nu):
+        a, b = rp[u * unit], rp[min((u + 1) * unit, n)]
+        out[u] = (int(c[a:b].min()), int(c[a:b].max())) if b > a else (0, -1)
+    return out

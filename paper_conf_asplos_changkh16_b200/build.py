@@ -20,7 +20,7 @@ CSRC = os.path.join(HERE, "csrc")
 INC = os.path.join(ROOT, "include")
 OBJ = os.path.join(ROOT, "build", "obj")
 LIB = os.path.join(HERE, "libdysel.so")
-SOURCES = ["runtime.cu", "spmv.cu", "spmv_probe.cu", "spmv_prep.cu", "sgemm.cu", "comm.cu", "iterate.cu", "stencil.cu", "spmtv.cu"]
+SOURCES = ["runtime.cu", "spmv.cu", "spmv_probe.cu", "spmv_prep.cu", "spmv_f2.cu", "sgemm.cu", "comm.cu", "iterate.cu", "stencil.cu", "spmtv.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
@@ -33,15 +33,16 @@ def _deps():
     return max(os.path.getmtime(h) for h in hdrs)
 
 
-RDC = {"spmv.cu"}   # the switch kernel's device-side launch (A-42) needs relocatable device code
+RDC = {"spmv.cu", "spmtv.cu"}   # the switch kernel's device-side launch (A-42) needs relocatable device code
 
 
-def _compile(src, verbose):
-    obj = os.path.join(OBJ, src.replace(".cu", ".o"))
+def _compile(src, verbose, obj_dir=None, defines=()):
+    obj = os.path.join(obj_dir or OBJ, src.replace(".cu", ".o"))
     path = os.path.join(CSRC, src)
     if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(path), _deps()):
         return obj, ""
-    cmd = [NVCC, *ARCH, *FLAGS, *(["-rdc=true"] if src in RDC else []), "-c", path, "-o", obj]
+    cmd = [NVCC, *ARCH, *FLAGS, *[f"-D{d}" for d in defines], *(["-rdc=true"] if src in RDC else []), "-c", path,
+           "-o", obj]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -50,35 +51,42 @@ def _compile(src, verbose):
     return obj, r.stderr
 
 
-def build(verbose: bool = False) -> str:
-    os.makedirs(OBJ, exist_ok=True)
+def build(verbose: bool = False, defines=(), out=None) -> str:
+    """defines / out: an A/B build of the same sources with -D defines into
+    another library path (objects under build/obj-<tag>); the product library
+    is the default build."""
+    lib = out or LIB
+    obj_dir = OBJ if not defines else OBJ + "-" + "-".join(d.replace("=", "") for d in defines)
+    os.makedirs(obj_dir, exist_ok=True)
     with cf.ThreadPoolExecutor(len(SOURCES)) as ex:
-        results = list(ex.map(lambda s: _compile(s, verbose), SOURCES))
+        results = list(ex.map(lambda s: _compile(s, verbose, obj_dir, defines), SOURCES))
     objs = [o for o, _ in results]
     if verbose:
         for _, log in results:
             if log:
                 sys.stderr.write(log)
-    if not os.path.exists(LIB) or os.path.getmtime(LIB) < max(os.path.getmtime(o) for o in objs):
+    if not os.path.exists(lib) or os.path.getmtime(lib) < max(os.path.getmtime(o) for o in objs):
         rdc = [o for o in objs if os.path.basename(o).replace(".o", ".cu") in RDC]
-        dlink = os.path.join(OBJ, "dlink.o")
+        dlink = os.path.join(obj_dir, "dlink.o")
         r = subprocess.run([NVCC, *ARCH, "-Xcompiler", "-fPIC", "-dlink", *rdc, "-o", dlink, "-lcudadevrt"],
                            capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"device link failed:\n{r.stderr}")
-        cmd = [NVCC, *ARCH, "-shared", "-o", LIB, *objs, dlink, "-lcudadevrt", "-ldl"]
+        cmd = [NVCC, *ARCH, "-shared", "-o", lib, *objs, dlink, "-lcudadevrt", "-ldl"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stderr}")
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--verbose", action="store_true")
     ap.add_argument("--force", action="store_true")
+    ap.add_argument("-D", dest="defines", action="append", default=[], help="A/B build: extra -D define")
+    ap.add_argument("--out", default=None, help="A/B build: library path")
     a = ap.parse_args()
     if a.force and os.path.isdir(OBJ):
         for f in os.listdir(OBJ):
             os.remove(os.path.join(OBJ, f))
-    print(build(a.verbose))
+    print(build(a.verbose, tuple(a.defines), a.out))

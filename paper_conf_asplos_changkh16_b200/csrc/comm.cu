@@ -158,26 +158,76 @@ dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local, const in
   return allgatherv(ctx, d_y, offs, counts, (cudaStream_t)stream);
 }
 
-dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A, int lda,
+dysel_status dysel_sgemm_shard_rows(int M, int world, int rank, int *m0, int *m1) {
+  if (M < 0 || world < 1 || rank < 0 || rank >= world || !m0 || !m1) return DYSEL_ERR_INVALID;
+  // M-blocks of ceil(M / world) rounded up to 128 rows (one tcgen05 tile)
+  const int64_t per = (((int64_t)M + world - 1) / world + 127) / 128 * 128;
+  *m0 = (int)std::min<int64_t>((int64_t)rank * per, M);
+  *m1 = (int)std::min<int64_t>((int64_t)(rank + 1) * per, M);
+  return DYSEL_OK;
+}
+
+dysel_status dysel_sgemm_sharded(dysel_ctx *ctx, int M, int N, int K, float alpha, const float *d_A_local, int lda,
                                  const float *d_B, int ldb, float beta, float *d_C, int ldc, float f, uint32_t mode,
                                  void *stream, dysel_report *rep) {
-  if (!ctx || M < 0) return DYSEL_ERR_INVALID;
+  if (!ctx || M < 0 || N < 0 || K < 0) return DYSEL_ERR_INVALID;
   const int R = ctx->world;
   if (R > 1024) return DYSEL_ERR_UNSUPPORTED;
-  // M-blocks of ceil(M/R) rounded up to 128 rows (one tcgen05 tile)
-  const int64_t per = (((int64_t)M + R - 1) / R + 127) / 128 * 128;
   int64_t offs[1024], counts[1024];
   for (int r = 0; r < R; ++r) {
-    const int64_t m0 = std::min<int64_t>((int64_t)r * per, M), m1 = std::min<int64_t>((int64_t)(r + 1) * per, M);
-    offs[r] = m0 * ldc;
-    counts[r] = (m1 - m0) * ldc;
+    int a = 0, b = 0;
+    DYSEL_TRY(dysel_sgemm_shard_rows(M, R, r, &a, &b));
+    offs[r] = (int64_t)a * ldc;
+    counts[r] = (int64_t)(b - a) * ldc;
   }
-  const int64_t m0 = std::min<int64_t>((int64_t)ctx->rank * per, M);
-  const int64_t m1 = std::min<int64_t>((int64_t)(ctx->rank + 1) * per, M);
+  int m0 = 0, m1 = 0;
+  DYSEL_TRY(dysel_sgemm_shard_rows(M, R, ctx->rank, &m0, &m1));
+  // A_g is LOCAL (rows [m0, m1) only, row 0 = global row m0); B replicated; C_g
+  // written in place inside the full C, then allgathered
   if (m1 > m0)
-    DYSEL_TRY(dysel_sgemm(ctx, (int)(m1 - m0), N, K, alpha, d_A + m0 * lda, lda, d_B, ldb, beta, d_C + m0 * ldc, ldc, f,
+    DYSEL_TRY(dysel_sgemm(ctx, m1 - m0, N, K, alpha, d_A_local, lda, d_B, ldb, beta, d_C + (int64_t)m0 * ldc, ldc, f,
                           mode, stream, rep));
   return allgatherv(ctx, d_C, offs, counts, (cudaStream_t)stream);
+}
+
+// 1-GPU loopback of the row-sharded SpMV (SURVEY §8e "Testing without 8
+// GPUs"): the G shards' DySel launches run one after another on this device,
+// each with its own plan (rebased row_ptr) and therefore its own selection —
+// the paper's "mixed version" — each into a private staging
+// buffer standing in for that GPU's local y, and one cudaMemcpyAsync per
+// shard stands in for its part of the allgatherv.
+dysel_status dysel_spmv_sharded_loopback(dysel_ctx *ctx, int G, dysel_spmv_plan *const *plans, const int64_t *bounds,
+                                         const float *d_x, float *d_y, float f, uint32_t mode, void *stream,
+                                         dysel_report *reps) {
+  if (!ctx || G < 1 || !plans || !bounds || (bounds[G] > 0 && (!d_y || !d_x))) {
+    set_error(ctx, "dysel_spmv_sharded_loopback: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  int64_t maxc = 0;
+  for (int g = 0; g < G; ++g) {
+    dysel_spmv_plan_info info;
+    if (!plans[g] || bounds[g + 1] < bounds[g]) {
+      set_error(ctx, "dysel_spmv_sharded_loopback: bad plan / bounds");
+      return DYSEL_ERR_INVALID;
+    }
+    DYSEL_TRY(dysel_spmv_plan_get_info(plans[g], &info));
+    if (info.n_rows != bounds[g + 1] - bounds[g]) {
+      set_error(ctx, "dysel_spmv_sharded_loopback: plan rows != bounds slice");
+      return DYSEL_ERR_INVALID;
+    }
+    maxc = std::max<int64_t>(maxc, info.n_rows);
+  }
+  DYSEL_TRY(scratch(ctx, ctx->shard_stage, (size_t)std::max<int64_t>(maxc, 1) * sizeof(float)));
+  float *stage = (float *)ctx->shard_stage.ptr;
+  for (int g = 0; g < G; ++g) {
+    const int64_t n = bounds[g + 1] - bounds[g];
+    DYSEL_TRY(dysel_spmv(ctx, plans[g], d_x, stage, f, mode, stream, reps ? reps + g : nullptr));
+    if (n > 0)
+      DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(d_y + bounds[g], stage, (size_t)n * sizeof(float), cudaMemcpyDeviceToDevice,
+                                          st));
+  }
+  return DYSEL_OK;
 }
 
 }  // extern "C"

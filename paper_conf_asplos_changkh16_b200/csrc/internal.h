@@ -102,10 +102,12 @@ struct dysel_ctx {
   dysel::DevProf *d_prof = nullptr;
   dysel::DevProf *h_prof = nullptr;  // pinned
   void *d_spmv_state = nullptr;      // persistent-dispatcher state (spmv.cu)
+  void *d_spmtv_state = nullptr;     // swap-mode device path state (spmtv.cu)
   void *h_spmv_rep = nullptr;        // pinned copy of its report area
   dysel::ScratchBuf sandbox[2 * DYSEL_MAX_VARIANTS];
   dysel::ScratchBuf unit_variant;    // device bytes, one per granule
   dysel::ScratchBuf norm_part;       // iterate.cu: fp64 norm partials
+  dysel::ScratchBuf shard_stage;     // comm.cu: loopback shard output (a GPU's local y)
   dysel::PendingSel pending[dysel::kPendingRing];
   uint64_t *h_pending_sel = nullptr;   // pinned + mapped, kPendingRing words
   uint64_t *d_pending_sel = nullptr;   // device alias of h_pending_sel
@@ -116,6 +118,9 @@ struct dysel_ctx {
   uint32_t *d_sel_timeout = nullptr;
   uint64_t launches = 0;
   uint64_t plan_serial = 0;
+  // L2 persisting set-aside (f-2 placement pool, x_persist): bytes reserved, max window
+  size_t l2_persist_bytes = 0;
+  size_t l2_persist_window = 0;
   // multi-GPU
   void *nccl_comm = nullptr;
   int rank = 0, world = 1;

@@ -482,6 +482,7 @@ void dysel_destroy(dysel_ctx *ctx) {
   if (ctx->ev_start) cudaEventDestroy(ctx->ev_start);
   if (ctx->ev_fork2) cudaEventDestroy(ctx->ev_fork2);
   if (ctx->d_prof) cudaFree(ctx->d_prof);
+  if (ctx->d_spmtv_state) cudaFree(ctx->d_spmtv_state);
   if (ctx->h_prof) cudaFreeHost(ctx->h_prof);
   if (ctx->h_pending_sel) cudaFreeHost(ctx->h_pending_sel);
   if (ctx->h_sel_timeout) cudaFreeHost(ctx->h_sel_timeout);
@@ -491,6 +492,7 @@ void dysel_destroy(dysel_ctx *ctx) {
     if (b.ptr) cudaFree(b.ptr);
   if (ctx->unit_variant.ptr) cudaFree(ctx->unit_variant.ptr);
   if (ctx->norm_part.ptr) cudaFree(ctx->norm_part.ptr);
+  if (ctx->shard_stage.ptr) cudaFree(ctx->shard_stage.ptr);
   comm_free(ctx);
   delete ctx;
 }

@@ -5,18 +5,19 @@
 //   1. init kernel: reset the ctx's device state (tickets, timer slots, scores).
 //   2. ONE profiling kernel (PDL behind the init): CTA b runs profiled unit
 //      b / K of pool variant b mod K — fully mode: a disjoint unit per
-//      variant (A-24), hybrid: the same units for every variant, each into its
-//      own sandbox (A-4').  Every unit is timed (Fig. 7b, B200 form); the last
-//      CTA of a variant scores it (packed atomicMin, A-7/A-8); the last variant
-//      publishes the selection and the switch point.
+//      variant (A-24), hybrid: the same units for every variant, the default
+//      writing y and the others a sandbox (A-4).  Every unit is timed (Fig. 7b,
+//      B200 form); the last CTA of a variant scores it (packed atomicMin,
+//      A-7/A-8); a variant that provably cannot win is decided at once
+//      (dominance, A-26); the last variant decided publishes the selection and
+//      the switch point.
 //   3. The default ("initial") variant's claim kernel (PDL behind the
 //      profiling kernel): ASYNC, its warps claim light remainder slots eagerly
 //      until the selection is published; then the winner's warps
 //      take the rest, heavy units first (A-40, A-45).
 //   4. A one-warp switch kernel (PDL) that device-launches the winner's claim
 //      kernel only when the default lost (A-42).
-// Hybrid sandbox units of a provably losing variant stop early (dominance,
-// A-26).  The unit order (seq) and the light / heavy split come from the plan
+// The unit order (seq) and the light / heavy split come from the plan
 // (spmv_prep.cu, reading A-45).
 #include <algorithm>
 #include <cstdlib>
@@ -44,7 +45,7 @@ struct SpmvState {
   uint64_t sel;             // final packed selection, ~0 until published
   uint64_t best_total;      // min over completed variants of the predicted time (busy score) or makespan (ns)
   uint32_t ctas_done[DYSEL_MAX_VARIANTS];
-  uint32_t dominated[DYSEL_MAX_VARIANTS];
+  uint32_t decided[DYSEL_MAX_VARIANTS];   // 0 running, 1 completed, 2 dominated (set once, by CAS)
   uint64_t busy[DYSEL_MAX_VARIANTS];      // sum of unit busy times (ns)
   uint64_t lb[DYSEL_MAX_VARIANTS];        // lower bound of the final busy sum (ns)
   uint64_t aborted[DYSEL_MAX_VARIANTS];   // sandbox units stopped / skipped by dominance
@@ -63,7 +64,7 @@ struct ProfParams {
   uint64_t *host_sel;    // mapped pinned word: the publishing CTA writes the selection here (cache)
   int32_t vids[DYSEL_SPMV_NVARIANTS];
   uint32_t occ[DYSEL_SPMV_NVARIANTS];
-  float *sandbox;        // K * c * 256 floats (hybrid, A-4')
+  float *sandbox;        // (K - 1) * c * 256 floats (hybrid: every variant but the default, A-4)
   uint64_t *tl;          // SpmvState::tl when a report is requested, else nullptr (no timeline atomics)
   uint8_t *unit_variant; // optional debug map (variant id per unit)
   uint32_t pure;         // pure full-grid run of one variant (self-resetting counters, no init kernel)
@@ -74,7 +75,21 @@ struct ProfParams {
   // default only light units seq[p_end, n_light); the winner the rest first.
   const int32_t *seq;
   uint32_t n_light;
+  // eager list (reading A-45, thread-per-row defaults only; nullptr = the
+  // light range): the light units whose longest row is <= kEagerRowTPR, in
+  // index order, and their bitmap -- an unproven thread-per-row default's
+  // eager claims take only these (its time per slot grows with the longest
+  // row); the winner then walks the whole light range and skips those done
+  const int32_t *elist;
+  const uint32_t *ebits;
+  uint32_t n_elist;
 };
+
+// eager slots of the default (published switch point S is clipped to it)
+__host__ __device__ __forceinline__ uint32_t eager_slots(const ProfParams &p) {
+  if (p.p_end >= p.n_light) return 0u;
+  return (p.elist ? p.n_elist : p.n_light - p.p_end) * (uint32_t)(kUnitRows / 32);
+}
 
 __global__ void spmv_state_init_kernel(SpmvState *s, int def) {
   // the profiling kernel behind it (PDL) may launch now; it waits for this
@@ -83,7 +98,7 @@ __global__ void spmv_state_init_kernel(SpmvState *s, int def) {
   const int v = threadIdx.x;
   if (v < DYSEL_MAX_VARIANTS) {
     s->ctas_done[v] = 0;
-    s->dominated[v] = 0;
+    s->decided[v] = 0;
     s->busy[v] = 0;
     s->lb[v] = 0;
     s->aborted[v] = 0;
@@ -116,14 +131,45 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
   return v;
 }
 
-// Dominance abort for hybrid sandbox units (A-26): every ~kPollNs
-// one thread of the CTA adds the time elapsed since the last report to lb[v].
-// lb[v] only sums time variant v's units really spent, so it is a lower bound
-// of v's final busy sum; once the prediction it implies exceeds the predicted
-// time of a COMPLETED variant (best_total) v cannot be selected any more (in
-// hybrid mode every variant profiles the same c units), so its sandbox work
-// stops and its remaining sandbox units are skipped: the selection is the one
-// running them to completion would give.
+// Publishing (the last variant to be decided, by completion or dominance):
+// the packed selection, the switch point S of the claim kernels (the eager
+// claim count at this instant rounded up to a whole unit, clipped to the
+// light range E), the activation-flag cache word.  One thread.
+struct PubArgs {
+  SpmvState *st;
+  uint64_t *host_sel;   // mapped pinned word (selection cache), nullable
+  uint64_t *tl;         // report timeline, nullable
+  uint32_t K;
+  uint32_t E;           // eager (light) slots
+};
+constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
+
+__device__ __forceinline__ void decided_publish(const PubArgs a) {
+  __threadfence();
+  const uint32_t vd = atomicAdd(&a.st->variants_done, 1u) + 1u;
+  if (vd != a.K) return;
+  __threadfence();
+  const unsigned long long fin = atomicAdd((unsigned long long *)&a.st->best, 0ull);
+  atomicExch((unsigned long long *)&a.st->sel, fin);
+  const uint64_t old = atomicOr((unsigned long long *)&a.st->c1, 1ull << 32);   // close the eager range
+  const uint64_t S = min(((uint64_t)(uint32_t)old + kSlots - 1) / kSlots * kSlots, (uint64_t)a.E);
+  atomicExch((unsigned long long *)&a.st->sw, (S << 8) | (fin & 0xffull));
+  if (a.host_sel) *(volatile uint64_t *)a.host_sel = fin;
+  if (a.tl) a.tl[1] = dysel_globaltimer();
+  __threadfence();
+}
+
+// Dominance (A-26): every ~kPollNs one thread of a profiling CTA
+// adds the time elapsed since its last report to lb[v].  lb[v] only sums time
+// variant v's units really spent, so it is a lower bound of v's final busy
+// sum; once the prediction it implies exceeds the predicted time of a
+// COMPLETED variant (best_total), v cannot be selected any more: v is DECIDED
+// at once (maximal score, one CAS on decided[v]) so the selection never waits
+// for its CTAs.  Its sandbox units (hybrid, non-default) stop and the rest
+// are skipped; productive units (fully mode, the hybrid default) run on —
+// their output is part of y (north_star: profiling slices are never
+// recomputed) — and only stop polling.  The selection is the one running
+// every slice to completion would give.
 // The comparison is made in the units of the active score: busy score ->
 // max(lb x G_n / (c x occ x #SM), this unit's elapsed time) vs the best
 // completed prediction; makespan score (sequential profiling: the variant
@@ -132,18 +178,20 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
 constexpr uint64_t kPollNs = 2000;
 constexpr long long kPollCycles = 2048;   // ~1 us at 1.9 GHz
 constexpr uint32_t kWarpPollEvery = 4;
-struct SandboxPoll {
+template <bool PRODUCTIVE>
+struct ProfPoll {
   static constexpr bool active = true;
   unsigned long long *s_last;   // smem: last report time
   const unsigned long long *s_start;   // smem: this unit's start time
-  volatile int *s_abort;        // smem
+  volatile int *s_abort;        // smem: the variant is dominated (sandbox: stop; productive: stop polling)
   unsigned long long *lb;
   const uint64_t *best_total;
-  uint32_t *dominated;
+  uint32_t *decided;
   const uint64_t *t_start;      // makespan mode: the variant's earliest CTA start
   uint64_t scale_num;           // busy mode: lower bound of the predicted time = lb * num / den
   uint64_t scale_den;
   uint32_t makespan;
+  PubArgs pub;
   // %globaltimer reads are slow (measured: polling it every loop step doubled
   // the per-unit time of CSR-V / CSR-W sandboxes); the per-SM cycle counter
   // (CS2R) gates them to one per kPollCycles per thread.
@@ -154,27 +202,27 @@ struct SandboxPoll {
     next_clk = c + kPollCycles;
     return true;
   }
-  // thread-per-row loops: every thread polls (its own loop); warp loops: warp()
+  // true = stop this unit (sandbox of a dominated variant)
   __device__ __forceinline__ bool operator()() const {
-    if (*s_abort) return true;
-    return due() && report();
+    if (*s_abort) return !PRODUCTIVE;
+    return due() && report() && !PRODUCTIVE;
   }
   // warp-cooperative loops: only lane 0 reads the timer (the caller combines
   // with __any_sync); checked every kWarpPollEvery-th step only
   mutable uint32_t tick = 0;
   __device__ __forceinline__ bool warp() const {
     if ((++tick & (kWarpPollEvery - 1)) != 0) return false;   // warp-uniform
-    if (*s_abort) return true;
+    if (*s_abort) return !PRODUCTIVE;
     if ((threadIdx.x & 31) != 0) return false;
-    return due() && report();
+    return due() && report() && !PRODUCTIVE;
   }
   // Global values read by this thread's previous report, issued without
   // waiting (a blocking global atomic / load per report stalled the polling
   // warp for ~3 L2 round trips and doubled sandbox unit times).  Stale values
   // stay safe: lb only grows (a stale lb is still a lower bound) and
-  // best_total only shrinks (a stale best aborts later, never wrongly).
+  // best_total only shrinks (a stale best decides later, never wrongly).
   mutable unsigned long long lb_seen = 0, best_seen = ~0ull, t0_seen = ~0ull;
-  mutable uint32_t dom_seen = 0;
+  mutable uint32_t dec_seen = 0;
   __device__ __forceinline__ bool report() const {
     const unsigned long long now = dysel_globaltimer();
     const unsigned long long last = *(volatile unsigned long long *)s_last;
@@ -190,14 +238,15 @@ struct SandboxPoll {
       const unsigned long long el = now - *(volatile const unsigned long long *)s_start;
       cost = thr > el ? thr : el;
     }
-    if (cost > best_seen || dom_seen != 0) {
+    if (dec_seen == 1u) return false;   // completed (this unit's report raced its last CTA): never dominated
+    if (cost > best_seen || dec_seen == 2u) {
       *s_abort = 1;
-      atomicExch(dominated, 1u);
+      if (dec_seen != 2u && atomicCAS(decided, 0u, 2u) == 0u) decided_publish(pub);
       return true;
     }
     lb_seen = ld_relaxed_u64((const uint64_t *)lb);
     best_seen = ld_relaxed_u64(best_total);
-    dom_seen = ld_relaxed_u32(dominated);
+    dec_seen = ld_relaxed_u32(decided);
     if (makespan) t0_seen = ld_relaxed_u64(t_start);
     return false;
   }
@@ -206,7 +255,6 @@ struct SandboxPoll {
 // resident CTAs per SM each plain variant kernel is compiled for (register
 // cap).  CSR-V at 6/SM spills and measured slower on D4 (1.44 vs 1.35 ms).
 constexpr int kSliceMinBlocks[DYSEL_SPMV_NVARIANTS] = {8, 4, 4, 6, 5, 3};
-constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
 // dynamic shared memory of each variant's kernels (CSR-T's staging buffers)
 __host__ __device__ constexpr size_t dyn_smem(int vid) { return vid == DYSEL_SPMV_CSR_TMA ? sizeof(TmaStageBufs) : 0; }
 inline size_t pool_dyn_smem(const ProfParams &p) {
@@ -262,23 +310,23 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
   const uint64_t thr_den = (uint64_t)p.c * max(1u, p.occ[pv]) * max(1u, p.n_sm);
   const uint32_t jj = p.hybrid ? b : (p.contiguous ? pv * p.c + b : pv + p.K * b);   // position in seq
   const uint32_t j = unit_at(p, jj);
-  // hybrid (reading A-4'): every variant runs the shared units into its own
-  // sandbox and may be stopped by dominance; the winner's sandbox is copied
-  // into y when the selection is published, so its profiled work is the
-  // productive one (never recomputed) whichever variant wins
-  const bool productive = !p.hybrid;
+  // hybrid (reading A-4): every variant runs the same units; the
+  // default ("first") variant writes y, the others their own sandbox
+  const bool productive = !p.hybrid || pv == p.def;
   const bool sandbox = !productive;
+  const PubArgs pub{st, p.host_sel, p.tl, p.K, eager_slots(p)};
   if (tid == 0) {
     s_abort = 0;
     s_last = dysel_globaltimer();
     s_start = s_last;
-    s_skip = (sandbox && p.abort && ld_relaxed_u32(&st->dominated[pv]) != 0) ? 1 : 0;
+    s_skip = (sandbox && p.abort && ld_relaxed_u32(&st->decided[pv]) == 2u) ? 1 : 0;
     if (!s_skip) atomicMin((unsigned long long *)&st->slot[pv].t_start_min, s_last);   // variant start (makespan)
     if (p.tl) atomicMin((unsigned long long *)&p.tl[0], s_last);
   }
   __syncthreads();
   const bool skipped = s_skip != 0;
-  float *out = productive ? y + (size_t)j * kUnitRows : p.sandbox + ((size_t)pv * p.c + b) * kUnitRows;
+  const uint32_t sb = pv < p.def ? pv : pv - 1;   // sandbox slot of a non-default variant (K - 1 of them)
+  float *out = productive ? y + (size_t)j * kUnitRows : p.sandbox + ((size_t)sb * p.c + b) * kUnitRows;
   if (!skipped) {
     if ((tid & 31) == 0) {
       psm.c0[tid >> 5] = dysel_clock64();
@@ -289,11 +337,16 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     // (CSR-V, CSR-W) finish any unit in tens of us, and polling inside their
     // loops measured +60% per-unit time on D4 (CSR-W 15 -> 24.6 us).
     constexpr bool kPolled = VID == 0 || VID == 2 || VID == 3 || VID == 5;
-    if (kPolled && sandbox && p.abort)
+    if (kPolled && p.abort && sandbox)
       run_unit<VID>(A, j, out,
-                    SandboxPoll{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
-                                &st->dominated[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
-                                p.score_mode == 2 ? 1u : 0u});
+                    ProfPoll<false>{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
+                                    &st->decided[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
+                                    p.score_mode == 2 ? 1u : 0u, pub});
+    else if (kPolled && p.abort)
+      run_unit<VID>(A, j, out,
+                    ProfPoll<true>{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
+                                   &st->decided[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
+                                   p.score_mode == 2 ? 1u : 0u, pub});
     else
       run_unit<VID>(A, j, out, NoPoll());
     if ((tid & 31) == 0) {
@@ -313,8 +366,6 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     c0 = min(c0, __shfl_xor_sync(0xffffffffu, c0, o));
     c1 = max(c1, __shfl_xor_sync(0xffffffffu, c1, o));
   }
-  bool publish = false;
-  unsigned long long fin = 0;
   if (tid == 0) {
     dysel_timer_slot *slot = &st->slot[pv];
     if (!skipped) {
@@ -327,72 +378,30 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
       if (p.tl) atomicMax((unsigned long long *)&p.tl[7], t1 - t0);
     }
     if (p.tl) atomicMax((unsigned long long *)&p.tl[2], dysel_globaltimer());
-    if (skipped || s_abort) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
+    if (skipped || (s_abort && sandbox)) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
     atomicAdd((unsigned long long *)&slot->units, 1ull);
     if (productive && p.unit_variant) p.unit_variant[j] = (uint8_t)VID;
     __threadfence();
     const uint32_t done = atomicAdd(&st->ctas_done[pv], 1u) + 1u;
-    if (done == p.c) {
-      // ---- variant complete: score, packed atomicMin (A-7, A-8)
+    // ---- variant complete (and not already decided by dominance): score,
+    // packed atomicMin (A-7, A-8); the last variant decided publishes
+    if (done == p.c && atomicCAS(&st->decided[pv], 0u, 1u) == 0u) {
       __threadfence();
       const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
       const unsigned long long e = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
       const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
       const unsigned long long bz = atomicAdd((unsigned long long *)&st->busy[pv], 0ull);
       const unsigned long long mb = atomicAdd((unsigned long long *)&st->max_busy[pv], 0ull);
-      const bool dom = ld_relaxed_u32(&st->dominated[pv]) != 0;
       const unsigned long long cap = (1ull << 56) - 1;
       const unsigned long long thr = bz * (unsigned long long)p.n_units / thr_den;
       const unsigned long long pred = thr > mb ? thr : mb;   // predicted full-grid time (ns)
       unsigned long long score = p.score_mode == 1 ? cy / p.c : p.score_mode == 2 ? e - a : pred;
-      if (dom || score > cap) score = cap;
-      if (!dom) atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
+      if (score > cap) score = cap;
+      atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
       atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
-      __threadfence();
-      const uint32_t vd = atomicAdd(&st->variants_done, 1u) + 1u;
-      if (vd == p.K) {
-        // ---- last variant: publish the selection
-        __threadfence();
-        fin = atomicAdd((unsigned long long *)&st->best, 0ull);
-        publish = true;
-      }
+      decided_publish(pub);
     }
   }
-  publish = __shfl_sync(0xffffffffu, publish ? 1 : 0, 0) != 0;
-  if (!publish) return;
-  fin = __shfl_sync(0xffffffffu, fin, 0);
-  const uint32_t win = (uint32_t)(fin & 0xff);
-  if (p.hybrid) {   // the winner's profiled units become the productive ones (warp 0 copies)
-    for (uint32_t q = 0; q < p.c; ++q) {
-      const uint32_t u = unit_at(p, q);
-      const int64_t r0 = (int64_t)u * kUnitRows;
-      const int n = (int)min((int64_t)kUnitRows, (int64_t)A.n_rows - r0);
-      const float *src = p.sandbox + ((size_t)win * p.c + q) * kUnitRows;
-      float *dst = y + r0;
-      // y is the caller's pointer (any float alignment, e.g. a tensor view):
-      // 16-byte vectors only when it is aligned (the sandbox always is)
-      const int n4 = ((uintptr_t)dst & 15) == 0 ? n / 4 : 0;
-      for (int i = tid; i < n4; i += 32) reinterpret_cast<float4 *>(dst)[i] = reinterpret_cast<const float4 *>(src)[i];
-      for (int i = n4 * 4 + tid; i < n; i += 32) dst[i] = src[i];
-      if (p.unit_variant && tid == 0) p.unit_variant[u] = (uint8_t)p.vids[win];
-    }
-    __syncwarp();
-    __threadfence();
-  }
-  if (tid != 0) return;
-  atomicExch((unsigned long long *)&st->sel, fin);
-  {   // close the eager ticket range; the default keeps whole units only, so
-      // the switch point S is rounded up to a unit boundary and clipped to the
-      // eager (light) range
-    const uint64_t old = atomicOr((unsigned long long *)&st->c1, 1ull << 32);
-    const uint32_t L1 = max(p.p_end, p.n_light);
-    const uint64_t E = (uint64_t)(L1 - p.p_end) * kSlots;
-    const uint64_t S = min(((uint64_t)(uint32_t)old + kSlots - 1) / kSlots * kSlots, E);
-    atomicExch((unsigned long long *)&st->sw, (S << 8) | win);
-  }
-  if (p.host_sel) *(volatile uint64_t *)p.host_sel = fin;   // activation-flag cache, no D2H copy
-  if (p.tl) p.tl[1] = dysel_globaltimer();
-  __threadfence();
 }
 
 // Profiling copy of one variant (sequential profiling: one launch per variant).
@@ -476,6 +485,10 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
   const uint32_t L1 = max(P, p.n_light);
   const uint32_t n_hs = (p.n_units - L1) * kSlots;   // winner's first range: heavy / long-row slots
   const uint32_t E = (L1 - P) * kSlots;               // light slots after the profiled prefix
+  const bool el = p.elist != nullptr && !p.pure;      // eager list mode (thread-per-row default)
+  const uint32_t Ee = p.pure ? 0u : eager_slots(p);   // eager ticket range
+  const uint32_t last_prof = P > 0 ? unit_at(p, P - 1) : 0u;   // profiled light units are <= this (light-first seq)
+  uint32_t last_eager = 0;                            // el: eager-done light units are eligible and <= this
   // Claim batch: k = min(p.k_claim, remaining / (2 x warps)) >= 1 (p.k_claim
   // ~ 1024 nnz of work per claim: the counter serialises claims, ~1 per ns,
   // which capped 1-nnz rows).  Claims are made on demand: issuing the next
@@ -504,8 +517,9 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     sw = __shfl_sync(FULL, sw, 0);
     if ((sw & 0xff) != pv) return false;
     phase = 2;
-    S = min((uint32_t)(sw >> 8), E);
-    n_win = n_hs + E - S;
+    S = min((uint32_t)(sw >> 8), Ee);
+    n_win = el ? n_hs + E : n_hs + E - S;
+    if (el && S > 0) last_eager = (uint32_t)__ldg(p.elist + S / kSlots - 1);
     t = gid;   // static first slot
     e = t < n_win ? t + 1 : t;
     return true;
@@ -519,14 +533,14 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
   for (;;) {
     if (t >= e) {   // need a claim
       if (phase == 1) {
-        const uint32_t k = batch(E - min(e, E));
+        const uint32_t k = batch(Ee - min(e, Ee));
         const uint64_t r = claim(k);
         t = (uint32_t)r;
-        uint32_t lim = E;
+        uint32_t lim = Ee;
         if (r >> 32) {   // claimed after the selection was published: only below the switch point
           uint64_t sw = 0;
           if (lane == 0) sw = wait_published(&st->sw);
-          lim = min((uint32_t)(__shfl_sync(FULL, sw, 0) >> 8), E);
+          lim = min((uint32_t)(__shfl_sync(FULL, sw, 0) >> 8), Ee);
         }
         if (t >= lim) {   // eager range closed or exhausted: hand over to the selection
           if (!enter_remainder()) break;
@@ -560,16 +574,22 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     }
     for (uint32_t q = t; q < e; ++q) {
       uint32_t u, w;
-      if (phase == 1) {   // eager: light slot q of seq[P, L1)
-        u = unit_at(p, P + q / kSlots);
+      if (phase == 1) {   // eager: light slot q of seq[P, L1), or of the eager list
         w = q % kSlots;
+        if (el) {
+          u = (uint32_t)__ldg(p.elist + q / kSlots);
+          if (P > 0 && u <= last_prof) continue;   // profiled already
+        } else {
+          u = unit_at(p, P + q / kSlots);
+        }
       } else if (q < n_hs) {   // winner / pure: heavy-first range seq[L1, n)
         u = unit_at(p, L1 + q / kSlots);
         w = q % kSlots;
-      } else {   // then the light slots from the switch point
-        const uint32_t l = S + (q - n_hs);
+      } else {   // then the light slots from the switch point (el: all, minus the eager-done ones)
+        const uint32_t l = (el ? 0u : S) + (q - n_hs);
         u = unit_at(p, P + l / kSlots);
         w = l % kSlots;
+        if (el && S > 0 && u <= last_eager && ((__ldg(p.ebits + (u >> 5)) >> (u & 31)) & 1u)) continue;
       }
       run_slot<VID>(A, u, (int)w, y + (size_t)u * kUnitRows);
       if (lane == 0 && p.unit_variant && w == 0) p.unit_variant[u] = (uint8_t)VID;
@@ -711,6 +731,11 @@ static const ClaimLauncher kClaim[DYSEL_SPMV_NVARIANTS] = {launch_claim<0>, laun
 static void set_order(ProfParams &p, const dysel_spmv_plan *pl) {
   p.seq = pl->seq;
   p.n_light = pl->seq ? pl->n_light : pl->n_units;
+}
+
+// thread-per-row variants: a slot's time grows with its longest row (A-45)
+static bool thread_per_row(int vid) {
+  return vid == DYSEL_SPMV_CSR_SCALAR || vid == DYSEL_SPMV_ELL || vid == DYSEL_SPMV_JDS || vid == DYSEL_SPMV_CSR_TMA;
 }
 
 // Slots per claim: about kClaimNnz nonzeros of work (at least 1, at most a unit).
@@ -892,18 +917,23 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.def = (uint32_t)pl->def;
   p.k_claim = claim_batch(pl);
   set_order(p, pl);
+  if (pl->elist && thread_per_row(pl->vids[pl->def])) {   // reading A-45: short-row eager list
+    p.elist = pl->elist;
+    p.ebits = pl->ebits;
+    p.n_elist = pl->n_elist;
+  }
   p.abort = ((mode & DYSEL_NO_ABORT) || p.score_mode == 1) ? 0u : 1u;   // dominance needs busy or makespan
   for (int i = 0; i < pl->K; ++i) {
     p.vids[i] = pl->vids[i];
     // occupancy of the claim kernel that will run the remainder with this variant
     p.occ[i] = (uint32_t)std::max(1, cs->occ_claim[pl->vids[i]]);
   }
-  if (p.hybrid) {   // A-4': K slice-sized sandboxes (every variant's profiled units are discardable)
-    const size_t bytes = (size_t)pl->K * P.c * kUnitRows * sizeof(float);
+  if (p.hybrid) {   // Table 1: K - 1 slice-sized sandboxes, the default's slice is productive (A-4)
+    const size_t bytes = (size_t)(pl->K - 1) * P.c * kUnitRows * sizeof(float);
     DYSEL_TRY(scratch(ctx, ctx->sandbox[0], bytes));
     p.sandbox = (float *)ctx->sandbox[0].ptr;
     if (rep) {
-      rep->sandbox_buffers = pl->K;
+      rep->sandbox_buffers = (uint32_t)(pl->K - 1);
       rep->sandbox_bytes = bytes;
     }
   }
@@ -966,7 +996,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       rep->makespan_ns[id] = t.t_end_max > t.t_start_min ? t.t_end_max - t.t_start_min : 0;
       rep->units[id] = t.units;
       rep->cycles[id] = t.cycles;
-      rep->score[id] = h->dominated[v] ? cap
+      rep->score[id] = h->decided[v] == 2u ? cap
                        : p.score_mode == 1 ? (t.units ? t.cycles / t.units : cap)
                        : p.score_mode == 2 ? rep->makespan_ns[id]
                                            : std::max<uint64_t>(h->busy[v] * p.n_units /

@@ -67,6 +67,7 @@ struct SpmvDev {
   const float *__restrict__ jds_val;
   const float *__restrict__ x;
   int32_t vec_ok;   // col/val 16-byte aligned
+  int32_t vec32;    // col/val 32-byte aligned (256-bit loads)
 };
 
 struct NoPoll {
@@ -104,6 +105,17 @@ __device__ __forceinline__ int4 ld_stream4(const int32_t *p, uint64_t pol) {
                : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
                : "l"(p), "l"(pol));
   return v;
+}
+// 256-bit loads (sm_100: LDG.E.256): one full 32-byte sector per lane
+__device__ __forceinline__ void ld_stream8(const int32_t *p, uint64_t pol, int (&v)[8]) {
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "l"(p), "l"(pol));
+}
+__device__ __forceinline__ void ld_stream8(const float *p, uint64_t pol, float (&v)[8]) {
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+               : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+               : "l"(p), "l"(pol));
 }
 __device__ __forceinline__ float4 ld_stream4(const float *p, uint64_t pol) {
   float4 v;
@@ -460,20 +472,18 @@ __device__ __forceinline__ void unit_csr_stream_s(const SpmvDev &A, uint32_t j, 
 // adds its 4 products to the lane partial; otherwise the row sums come from a
 // two-level segmented scan: sequential within the lane's 4 entries, then a
 // Hillis-Steele scan of the lane totals (segment starts = lanes holding a row
-// start, from a ballot), so a chunk costs ~20 shuffles instead of ~12 per 32
-// entries.  The order of every row's additions depends only on the row's
-// offset inside its group and on s mod 4: deterministic (c-6).
-#ifndef DYSEL_STREAM_VEC
-#define DYSEL_STREAM_VEC 2
-#endif
-constexpr int kStreamVec = DYSEL_STREAM_VEC;   // 128-entry chunks in flight per warp (8 x gathers per lane)
+// start, from a ballot); the open row's lane partials are folded (butterfly)
+// only when some chunk since the last fold added to them.  The order of every
+// row's additions depends only on the row's offset inside its group and on
+// s mod 4: deterministic (c-6).
+// (Measured alternative, A-41b: lanes owning 8 contiguous entries
+// with lane-local row sums and direct row writes issued 1.8x the instructions
+// and ran 12% slower on D4.)
+constexpr int kStreamVec = 2;   // 128-entry chunks in flight per warp (8 x gathers per lane)
 template <class Poll>
 __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
                                                 const Poll &poll) {
-#ifndef DYSEL_EXP_CSRW_SCALAR
-#define DYSEL_EXP_CSRW_SCALAR 0   // experiment knob (scripts/build_exp.py): force the 32-bit form
-#endif
-  if (!A.vec_ok || DYSEL_EXP_CSRW_SCALAR) {
+  if (!A.vec_ok) {
     unit_csr_stream_s(A, j, w, out, poll);
     return;
   }
@@ -497,12 +507,14 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, in
   int oe = o >= 0 ? __shfl_sync(FULL, re, o) : e;
   const uint32_t lane_mask_le = (lane == 31) ? FULL : ((2u << lane) - 1u);
   const bool starts = rs < re;   // this lane's row is non-empty
+  bool pend = false;             // some lane partial added since the last fold (warp-uniform)
   for (int c0 = s & ~3; c0 < e; c0 += 128 * kStreamVec) {
     // long stretch of the open row ahead (c0 >= s: no foreign entries)
     if (c0 >= s && oe - c0 >= kStreamLong) {
       const int a = c0;   // 16-byte aligned here
       const int body_end = a + ((oe - a) & ~255);
       bool stop = false;
+      pend = true;
       for (int b0 = a; b0 < body_end; b0 += 256) {
         const int k0 = b0 + 4 * lane, k1 = k0 + 128;
         const int4 q0 = ld_stream4(A.col + k0, ps), q1 = ld_stream4(A.col + k1, ps);
@@ -559,14 +571,17 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, in
       if (cb >= e) break;
       if (oe >= cb + 128) {   // whole chunk inside the open row
         part += (p[u][0] + p[u][1]) + (p[u][2] + p[u][3]);
+        pend = true;
         continue;
       }
-      // fold the open row's per-lane partials
-      float P = part;
+      if (pend) {   // fold the open row's per-lane partials
+        float P = part;
 #pragma unroll
-      for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
-      if (lane == o) acc += P;
-      part = 0.0f;
+        for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
+        if (lane == o) acc += P;
+        part = 0.0f;
+        pend = false;
+      }
       // head bits of the chunk's 128 entries (word q: entries 32q .. 32q+31);
       // entry 0 always starts a segment
       const int off = rs - cb;
@@ -610,12 +625,15 @@ __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, in
     }
     if (Poll::active && __any_sync(FULL, poll.warp())) break;   // warp-uniform exit
   }
-  float P = part;
+  if (pend) {
+    float P = part;
 #pragma unroll
-  for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
-  if (lane == o) acc += P;
+    for (int d = 16; d > 0; d >>= 1) P += __shfl_xor_sync(FULL, P, d);
+    if (lane == o) acc += P;
+  }
   if (lane < nr) out[w * 32 + lane] = acc;
 }
+
 
 // ------------------------------------------------------------------ CSR-T
 // Bulk-staged CSR (B200 data-placement variant; north_star

@@ -164,6 +164,7 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
   A.col = d_col;
   A.val = d_val;
   A.vec_ok = (((uintptr_t)d_col | (uintptr_t)d_val) & 15) == 0;
+  A.vec32 = (((uintptr_t)d_col | (uintptr_t)d_val) & 31) == 0;
   pl->n_units = (uint32_t)((n_rows + kUnitRows - 1) / kUnitRows);
   const int64_t n_pad = (int64_t)pl->n_units * kUnitRows;
   A.n_pad = n_pad;
@@ -287,6 +288,22 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
         if (cudaMemcpy(pl->seq, seq.data(), nu * 4, cudaMemcpyHostToDevice) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
         pl->n_light = (uint32_t)light.size();
         I.n_heavy = (int32_t)rest.size();
+        std::vector<int32_t> el;
+        std::vector<uint32_t> bits((nu + 31) / 32, 0u);
+        for (int32_t u : light)
+          if ((int64_t)um[u] <= kEagerRowTPR) {
+            el.push_back(u);
+            bits[u >> 5] |= 1u << (u & 31);
+          }
+        if (!el.empty()) {
+          if (cudaMalloc(&pl->elist, el.size() * 4) != cudaSuccess ||
+              cudaMalloc(&pl->ebits, bits.size() * 4) != cudaSuccess)
+            return fail(DYSEL_ERR_NOMEM);
+          if (cudaMemcpy(pl->elist, el.data(), el.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+              cudaMemcpy(pl->ebits, bits.data(), bits.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
+            return fail(DYSEL_ERR_CUDA);
+          pl->n_elist = (uint32_t)el.size();
+        }
       }
     }
     I.n_light = pl->seq ? (int32_t)pl->n_light : (int32_t)nu;
@@ -365,6 +382,10 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *pl) {
       pl->ctx->reg.erase(pl->sig);
       pl->ctx->sel_cache.erase(pl->sig);
     }
+    if (!pl->place_sig.empty()) {
+      pl->ctx->reg.erase(pl->place_sig);
+      pl->ctx->sel_cache.erase(pl->place_sig);
+    }
   }
   cudaFree(pl->ell_col);
   cudaFree(pl->ell_val);
@@ -376,6 +397,9 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *pl) {
   cudaFree(pl->blk_off);
   cudaFree(pl->jd_off);
   cudaFree(pl->seq);
+  cudaFree(pl->xwin);
+  cudaFree(pl->elist);
+  cudaFree(pl->ebits);
   cudaGetLastError();
   delete pl;
 }

@@ -236,7 +236,6 @@ __global__ void __launch_bounds__(128) stencil_tiled_kernel(StencilArgs g, float
 }
 
 static uint64_t g_stencil_wave[DYSEL_STENCIL_NVARIANTS] = {0, 0, 0};   // occupancy x #SM
-
 template <int VID>
 static dysel_status stencil_variant_fn(const dysel_slice *s, void *const *args, void *stream, void *) {
   const StencilArgs &g = *(const StencilArgs *)args[1];
@@ -250,11 +249,12 @@ static dysel_status stencil_variant_fn(const dysel_slice *s, void *const *args, 
   if (s->gate && !s->timer && g_stencil_wave[VID] > 0) ctas = std::min<uint64_t>(ctas, g_stencil_wave[VID]);
   if constexpr (VID == DYSEL_STENCIL_BASE)
     stencil_base_kernel<<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
-  else if constexpr (VID == DYSEL_STENCIL_ZMARCH)
+  else if constexpr (VID == DYSEL_STENCIL_ZMARCH) {
     if (s->timer)
       stencil_zmarch_kernel<true><<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
     else
       stencil_zmarch_kernel<false><<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
+  }
   else
     stencil_tiled_kernel<<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
@@ -271,7 +271,6 @@ dysel_status stencil_register(dysel_ctx *ctx) {
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], stencil_tiled_kernel, 128, 0);
   cudaGetLastError();
   const uint64_t n = (uint64_t)ctx->n_sm;
-  for (int i = 0; i < DYSEL_STENCIL_NVARIANTS; ++i) g_stencil_wave[i] = (uint64_t)o[i] * n;
   dysel_variant v[DYSEL_STENCIL_NVARIANTS] = {
       {"base", kStencilFns[0], {1, 1, 1}, sb, 1, 0, nullptr, (uint64_t)o[0] * n},
       {"zmarch64", kStencilFns[1], {1, 1, 64}, sb, 1, 0, nullptr, (uint64_t)o[1] * n},

@@ -44,6 +44,10 @@ SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"
 STENCIL_NAMES = ["base", "zmarch64", "tiled64x4_zmarch64"]
 SPMTV_NAMES = ["scatter_thread", "scatter_warp", "scatter_segment"]
 STENCIL_BASE, STENCIL_ZMARCH, STENCIL_TILED = range(3)
+PLACE_LDG, PLACE_L2, PLACE_SMEM, PLACE_PERSIST = range(4)
+PLACE_NAMES = ["x_ldg", "x_l2", "x_smem", "x_persist"]
+JDSG_PLAIN, JDSG_UNROLL, JDSG_PREFETCH, JDSG_UNROLL_PREFETCH = range(4)
+JDSG_NAMES = ["jds_plain", "jds_unroll", "jds_prefetch", "jds_unroll_prefetch"]
 
 c_void_p, c_int, c_float, c_u32, c_u64, c_i64, c_size = (ctypes.c_void_p, ctypes.c_int, ctypes.c_float,
                                                         ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int64,
@@ -122,6 +126,19 @@ dysel_spmv_power_sharded = _sig("dysel_spmv_power_sharded", c_int, P, P, P, P, P
 dysel_comm_broadcast = _sig("dysel_comm_broadcast", c_int, P, P, c_size, c_int, P)
 dysel_sgemm_sharded = _sig("dysel_sgemm_sharded", c_int, P, c_int, c_int, c_int, c_float, P, c_int, P, c_int, c_float,
                            P, c_int, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_sgemm_shard_rows = _sig("dysel_sgemm_shard_rows", c_int, c_int, c_int, c_int, ctypes.POINTER(c_int),
+                              ctypes.POINTER(c_int))
+dysel_spmv_sharded_loopback = _sig("dysel_spmv_sharded_loopback", c_int, P, c_int, ctypes.POINTER(c_void_p), P, P, P,
+                                   c_float, c_u32, P, P)
+dysel_spmv_placement = _sig("dysel_spmv_placement", c_int, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_spmv_placement_variant = _sig("dysel_spmv_placement_variant", c_int, P, P, c_int, P, P, P)
+dysel_spmv_placement_windows = _sig("dysel_spmv_placement_windows", c_int, P, P, c_size)
+dysel_spmv_jds_prepare = _sig("dysel_spmv_jds_prepare", c_int, P, c_i64, c_i64, c_i64, P, P, P, P,
+                              ctypes.POINTER(c_void_p))
+dysel_spmv_jds = _sig("dysel_spmv_jds", c_int, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_spmv_jds_variant = _sig("dysel_spmv_jds_variant", c_int, P, P, c_int, P, P, P)
+dysel_spmv_jds_copy_array = _sig("dysel_spmv_jds_copy_array", c_int, P, c_int, P, ctypes.POINTER(c_size))
+dysel_spmv_jds_plan_destroy = _sig("dysel_spmv_jds_plan_destroy", None, P)
 dysel_kernel_launches = _sig("dysel_kernel_launches", c_u64, P)
 dysel_timer_calibrate = _sig("dysel_timer_calibrate", c_int, P, c_u64, c_u64, ctypes.POINTER(c_u64),
                              ctypes.POINTER(ctypes.c_double))
@@ -228,6 +245,36 @@ class SpmvPlan:
             pass
 
 
+class JdsPlan:
+    """Global-sort JDS pool of one matrix (dysel_spmv_jds_plan, f-2 Case III)."""
+    _ARRAYS = {"perm": (0, "int32"), "len": (1, "int32"), "jd_ptr": (2, "int32"), "col": (3, "int32"),
+               "val": (4, "float32")}
+
+    def __init__(self, ctx, handle, n_rows):
+        self.ctx, self.handle, self.n_rows = ctx, handle, n_rows
+        self.n_units = (n_rows + 255) // 256
+
+    def array(self, name):
+        import numpy as np
+        which, dt = self._ARRAYS[name]
+        n = c_size(0)
+        self.ctx._check(dysel_spmv_jds_copy_array(self.handle, which, None, ctypes.byref(n)))
+        out = np.empty(n.value // np.dtype(dt).itemsize, dt)
+        self.ctx._check(dysel_spmv_jds_copy_array(self.handle, which, out.ctypes.data_as(c_void_p), ctypes.byref(n)))
+        return out
+
+    def destroy(self):
+        if self.handle and self.ctx is not None and self.ctx.h:
+            dysel_spmv_jds_plan_destroy(self.handle)
+        self.handle = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
 class Context:
     """dysel_ctx on one CUDA device."""
 
@@ -243,6 +290,7 @@ class Context:
         n_sm, tick, l2 = c_int(), c_u64(), c_u64()
         dysel_device_info(h, ctypes.byref(n_sm), ctypes.byref(tick), ctypes.byref(l2))
         self.n_sm, self.globaltimer_tick_ns, self.l2_bytes = n_sm.value, tick.value, l2.value
+        self.rank, self.world = 0, 1
 
     def _check(self, st):
         if st != OK:
@@ -313,6 +361,50 @@ class Context:
     def spmv_gather_probe(self, plan, flavour, x, out, stream=None):
         """Measurement only: the plan's CSR traffic with no row structure (include/dysel.h)."""
         self._check(dysel_spmv_gather_probe(self.h, plan.handle, int(flavour), _ptr(x), _ptr(out), _stream(stream)))
+
+    # ----------------------------------------------------- SpMV f-2 pools
+    def spmv_placement(self, plan, x, y, f=0.02, mode=DEFAULT_MODE, report=False, unit_map=False, stream=None):
+        """y = A x through the x data-placement pool (Case II, f-2)."""
+        rep, keep, uv = (_make_report(plan.n_units if unit_map else 0) if report else (None, None, None))
+        self._check(dysel_spmv_placement(self.h, plan.handle, _ptr(x), _ptr(y), float(f), int(mode), _stream(stream),
+                                         ctypes.byref(rep) if rep is not None else None))
+        if rep is None:
+            return None
+        return report_dict(rep, PLACE_NAMES, bytes(uv) if uv is not None else None)
+
+    def spmv_placement_variant(self, plan, variant_id, x, y, stream=None):
+        self._check(dysel_spmv_placement_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y),
+                                                 _stream(stream)))
+
+    def spmv_placement_windows(self, plan):
+        import numpy as np
+        out = np.empty((plan.n_units, 2), np.int32)
+        st = dysel_spmv_placement_windows(plan.handle, out.ctypes.data_as(c_void_p), plan.n_units)
+        if st == ERR_NOT_FOUND:
+            return None
+        self._check(st)
+        return out
+
+    def spmv_jds_prepare(self, row_ptr, col, val, n_cols, stream=None) -> JdsPlan:
+        n = row_ptr.numel() - 1
+        h = ctypes.c_void_p()
+        self._check(dysel_spmv_jds_prepare(self.h, n, int(n_cols), col.numel(), _ptr(row_ptr), _ptr(col), _ptr(val),
+                                           _stream(stream), ctypes.byref(h)))
+        plan = JdsPlan(self, h, n)
+        self._plans.add(plan)
+        return plan
+
+    def spmv_jds(self, plan, x, y, f=0.02, mode=DEFAULT_MODE, report=False, unit_map=False, stream=None):
+        """y = A x through the global-sort JDS pool (Case III, f-2)."""
+        rep, keep, uv = (_make_report(plan.n_units if unit_map else 0) if report else (None, None, None))
+        self._check(dysel_spmv_jds(self.h, plan.handle, _ptr(x), _ptr(y), float(f), int(mode), _stream(stream),
+                                   ctypes.byref(rep) if rep is not None else None))
+        if rep is None:
+            return None
+        return report_dict(rep, JDSG_NAMES, bytes(uv) if uv is not None else None)
+
+    def spmv_jds_variant(self, plan, variant_id, x, y, stream=None):
+        self._check(dysel_spmv_jds_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), _stream(stream)))
 
     # ------------------------------------------------------------ SGEMM
     def sgemm(self, A, B, C, alpha=1.0, beta=0.0, f=0.02, mode=DEFAULT_MODE, report=False, unit_map=False,
@@ -392,6 +484,7 @@ class Context:
     def comm_init(self, rank, world, uid: bytes):
         buf = ctypes.create_string_buffer(uid, 128)
         self._check(dysel_comm_init(self.h, buf, int(rank), int(world)))
+        self.rank, self.world = int(rank), int(world)
 
     def spmv_sharded(self, local_plan, bounds, x, y, f=0.02, mode=DEFAULT_MODE, report=False, stream=None):
         b = (c_i64 * len(bounds))(*bounds)
@@ -410,14 +503,29 @@ class Context:
                                              ctypes.byref(rep) if rep is not None else None))
         return report_dict(rep, SPMV_NAMES) if rep is not None else None
 
-    def sgemm_sharded(self, A, B, C, alpha=1.0, beta=0.0, f=0.02, mode=DEFAULT_MODE, report=False, stream=None):
-        M, K = A.shape
-        N = B.shape[1]
+    def sgemm_sharded(self, A_local, B, C, alpha=1.0, beta=0.0, f=0.02, mode=DEFAULT_MODE, report=False,
+                      stream=None):
+        """C (full M x N on every rank) with rows [m0, m1) = alpha A_local B + beta C there, then allgathered;
+        A_local = this rank's rows of A only (see sgemm_shard_rows)."""
+        M, N = C.shape
+        K = B.shape[0]
+        m0, m1 = sgemm_shard_rows(M, self.world, self.rank)
+        assert A_local.shape[0] == m1 - m0 and A_local.shape[1] == K
         rep, keep, uv = (_make_report(0) if report else (None, None, None))
-        self._check(dysel_sgemm_sharded(self.h, M, N, K, float(alpha), _ptr(A), A.stride(0), _ptr(B), B.stride(0),
-                                        float(beta), _ptr(C), C.stride(0), float(f), int(mode), _stream(stream),
-                                        ctypes.byref(rep) if rep is not None else None))
+        self._check(dysel_sgemm_sharded(self.h, M, N, K, float(alpha), _ptr(A_local), max(1, A_local.stride(0)),
+                                        _ptr(B), B.stride(0), float(beta), _ptr(C), C.stride(0), float(f), int(mode),
+                                        _stream(stream), ctypes.byref(rep) if rep is not None else None))
         return report_dict(rep, SGEMM_NAMES) if rep is not None else None
+
+    def spmv_sharded_loopback(self, plans, bounds, x, y, f=0.02, mode=DEFAULT_MODE, report=False, stream=None):
+        """1-GPU loopback of the row-sharded SpMV: plans[g] = shard g's plan (rebased row_ptr); y full length."""
+        G = len(plans)
+        arr = (c_void_p * G)(*[p.handle for p in plans])
+        b = (c_i64 * len(bounds))(*bounds)
+        reps = (Report * G)() if report else None
+        self._check(dysel_spmv_sharded_loopback(self.h, G, arr, b, _ptr(x), _ptr(y), float(f), int(mode),
+                                                _stream(stream), ctypes.cast(reps, c_void_p) if reps is not None else None))
+        return [report_dict(reps[g], SPMV_NAMES) for g in range(G)] if reps is not None else None
 
     def comm_broadcast(self, t, root, stream=None):
         self._check(dysel_comm_broadcast(self.h, _ptr(t), t.numel(), int(root), _stream(stream)))
@@ -429,6 +537,14 @@ def comm_unique_id() -> bytes:
     if st != OK:
         raise DyselError(st, "ncclGetUniqueId failed")
     return buf.raw
+
+
+def sgemm_shard_rows(M, world, rank):
+    a, b = c_int(), c_int()
+    st = dysel_sgemm_shard_rows(int(M), int(world), int(rank), ctypes.byref(a), ctypes.byref(b))
+    if st != OK:
+        raise DyselError(st, "dysel_sgemm_shard_rows")
+    return a.value, b.value
 
 
 def partition_rows(row_ptr_host, world):

@@ -1,7 +1,7 @@
 """SpMTV swap-mode overhead on the 2M-row power-law matrix (bench secondary
 spmtv_powerlaw_2M, standalone): pure variants, AUTO (swap) single shot, host
 swap, amortised.  Run with DYSEL_SPMTV_PERSISTENT=1 for the persistent-wave
-remainder ablation."""
+remainder ablation (removed)."""
 import json
 import os
 import sys
@@ -26,8 +26,11 @@ out = {"persistent": bool(os.environ.get("DYSEL_SPMTV_PERSISTENT")), "pure_us": 
 for f in (0.002, 0.005, 0.01, 0.02):
     td = time_b2b(lambda: ctx.spmtv(plan, x, y, f=f, mode=D.AUTO), 20, stream)
     rep = ctx.spmtv(plan, x, y, f=f, mode=D.AUTO, report=True)
+    sels = [ctx.spmtv(plan, x, y, f=f, mode=D.AUTO, report=True)["selected_name"] for _ in range(10)]
     out["f=%g" % f] = {"us": round(td * 1e6, 1), "overhead_pct": round((td / best - 1) * 100, 2),
-                       "selected": rep["selected_name"], "c": rep["c"], "profiled": rep["profiled"]}
+                       "selected": rep["selected_name"], "c": rep["c"], "profiled": rep["profiled"],
+                       "selections_10": sels, "score": rep["score"][:3], "aborted": rep["aborted"][:3],
+                       "timeline_us": [None if t is None else round(t / 1e3, 1) for t in rep["timeline_ns"]]}
 print(json.dumps(out))
 for name, m in (("swap_no_abort", D.AUTO | D.NO_ABORT), ("fully", D.FULLY), ("swap_sequential", D.AUTO | D.SEQUENTIAL)
                 if hasattr(D, "SEQUENTIAL") else (("swap_no_abort", D.AUTO | D.NO_ABORT), ("fully", D.FULLY))):

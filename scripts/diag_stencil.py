@@ -14,7 +14,7 @@ def b2b(fn, n=50):
     for _ in range(n): fn()
     b.record(s); torch.cuda.synchronize()
     return a.elapsed_time(b) / n * 1e3
-for shape in ((64, 512, 512), (256, 256, 256)):
+for shape in ((64, 512, 512), (256, 512, 512)):
     a = torch.from_numpy(uniform_f32(1, shape)).cuda(); o = torch.empty_like(a)
     nb = 8 * a.numel()
     r = {D.STENCIL_NAMES[v]: b2b(lambda: ctx.stencil_variant(v, a, o, 0.8, 0.15)) for v in range(3)}

@@ -64,8 +64,10 @@ def test_sgemm_sharded_one_rank(cctx):
     M, K, N = 1024, 992, 1056
     A, B, C0 = sgemm_inputs(M, K, N, 992, 993, 994)
     C = torch.from_numpy(C0.copy()).cuda()
-    cctx.sgemm_sharded(torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda(), C, 1.5, -0.5, f=0.06,
-                       mode=D.FULLY | D.FORCE_PROFILE)
+    m0, m1 = D.sgemm_shard_rows(M, 1, 0)
+    assert (m0, m1) == (0, M)
+    cctx.sgemm_sharded(torch.from_numpy(A[m0:m1].copy()).cuda(), torch.from_numpy(B).cuda(), C, 1.5, -0.5,
+                       f=0.06, mode=D.FULLY | D.FORCE_PROFILE)
     torch.cuda.synchronize()
     ref, den = osg.sgemm(A, B, C0, 1.5, -0.5), osg.sgemm_abs(A, B, C0, 1.5, -0.5)
     assert float((np.abs(C.cpu().numpy() - ref) / den).max()) <= osg.SGEMM_TOL

@@ -147,3 +147,26 @@ def test_spmtv_bench_size_parity(ctx, D):
         assert rep["profiled"] == (mode == D.AUTO)
         assert _err(A, x, y0, y) <= SPMV_TOL, mode
     plan.destroy()
+
+
+@pytest.mark.parametrize("offset", [0, 1])
+def test_spmtv_swap_odd_columns_and_unaligned_y(ctx, D, offset):
+    """n_cols % 4 != 0 on a matrix big enough that a losing
+    variant is dominated mid-profile -- nothing of a partial private output
+    may reach y -- and an output y that is not 16-byte aligned (a tensor
+    view): the device swap path's add-in must not assume alignment."""
+    import torch
+    A = d4_powerlaw(n=600_002, lmax=3000)          # n_cols = 600,002 (mod 4 = 2)
+    x = uniform_f32(71, A.n_rows)
+    y0 = uniform_f32(72, A.n_cols)
+    plan, keep = _plan(ctx, A)
+    for mode in (D.AUTO, D.SWAP | D.HOST_ORCH):
+        buf = torch.empty(A.n_cols + 1, device="cuda")
+        y = buf[offset:offset + A.n_cols]
+        y.copy_(vec(y0))
+        rep = ctx.spmtv(plan, vec(x), y, f=0.02, mode=mode, report=True)
+        torch.cuda.synchronize()
+        assert rep["profiled"] and rep["mode_used"] & 3 == D.SWAP
+        assert rep["sandbox_buffers"] == len(D.SPMTV_NAMES)              # Table 1: K private outputs
+        assert _err(A, x, y0, y) <= SPMV_TOL, (mode, offset)
+    plan.destroy()

@@ -188,18 +188,21 @@ def test_dysel_composition(ctx, D, name, m):
     # productive default (A-4).
     # The device path profiles the first units of the plan's unit order
     # (light units first, A-45); the host path the NDRange prefix (paper).
+    # Hybrid: the default's profiled slice is the productive one (A-4).
     pool = plan.variant_ids
     owner = slice_plan.productive_cover(p, pool.index(sel))
     host = m.endswith("host")
     order = np.arange(plan.n_units) if host else unit_order(plan)
-    dev_hybrid = p.mode == slice_plan.HYBRID and not host
     n_prof = p.c * (K if p.mode == slice_plan.FULLY else 1)
     for j in range(p.Gn):
         u = order[j]
         if j < len(owner) and j < n_prof:
-            assert uv[u] == (sel if dev_hybrid else pool[owner[j]]), j
+            assert uv[u] == pool[owner[j]], j
         elif "async" not in m:
             assert uv[u] == sel, j
+    # Table 1: fully 0 extra outputs, hybrid K - 1 sandboxes
+    assert rep["sandbox_buffers"] == (K - 1 if p.mode == slice_plan.HYBRID else 0), rep["sandbox_buffers"]
+    assert rep["sandbox_bytes"] == (K - 1) * p.c * 256 * 4 * (p.mode == slice_plan.HYBRID) or host
     assert sorted(order) == list(range(plan.n_units))      # a permutation: every unit exactly once
     plan.destroy()
 
@@ -272,10 +275,10 @@ def test_remainder_hand_off(ctx, D, asy, default, name):
     """The remainder goes to the winner: the default's claim kernel runs it
     when the default wins, the switch kernel device-launches the winner's
     claim kernel otherwise (A-42).  Sync: every remainder unit is the
-    winner's (eager = 0).  Async: the eager units are whole LIGHT units of
-    the default (A-45: an unproven default never starts a heavy or long-row
-    unit, here a thread-per-row JDS default on 16,384-entry rows), the rest
-    the winner's."""
+    winner's (eager = 0).  Async: the default's eager units are whole LIGHT
+    units (A-45: an unproven default never starts a heavy or long-row unit;
+    a thread-per-row default -- JDS here -- only units whose longest row is
+    <= 128), every other remainder unit is the winner's."""
     import torch
     A = MATS[name]()
     x = uniform_f32(11, A.n_cols)
@@ -283,6 +286,9 @@ def test_remainder_hand_off(ctx, D, asy, default, name):
     K = len(plan.variant_ids)
     order = unit_order(plan)
     n_light = plan.info.n_light
+    light = set(order[:n_light].tolist())
+    lens = np.diff(A.row_ptr.astype(np.int64))
+    umax = np.array([lens[u * 256:(u + 1) * 256].max() for u in range(plan.n_units)])
     if name == "heavy":
         assert plan.info.n_heavy > 0 and n_light + plan.info.n_heavy == plan.n_units
     mode = D.FULLY | D.FORCE_PROFILE | (D.ASYNC if asy else 0)
@@ -292,15 +298,21 @@ def test_remainder_hand_off(ctx, D, asy, default, name):
     P = K * r["c"]
     rem = plan.n_units - P
     uv = r["unit_variant"]
+    sel = r["selected"]
+    rest = [order[j] for j in range(P, plan.n_units)]
     if not asy:
         assert r["eager_units"] == 0 and r["tail_units"] == rem, r
-        assert all(uv[order[j]] == r["selected"] for j in range(P, plan.n_units))
+        assert all(uv[u] == sel for u in rest)
     else:
-        e = r["eager_units"]
-        assert e + r["tail_units"] == rem, r
-        assert P + e <= max(P, n_light)                         # eager units are light
-        assert all(uv[order[j]] == default for j in range(P, P + e))
-        assert all(uv[order[j]] == r["selected"] for j in range(P + e, plan.n_units))
+        assert all(uv[u] in (default, sel) for u in rest)
+        if default != sel:
+            eager = [u for u in rest if uv[u] == default]
+            assert len(eager) <= r["eager_units"]
+            assert all(u in light for u in eager)                # never a heavy / long-row unit
+            if default == 3 and plan.info.n_heavy > 0:
+                assert all(umax[u] <= 128 for u in eager)        # thread-per-row default: short rows only
+        else:
+            assert r["eager_units"] + r["tail_units"] == rem, r
     plan.destroy()
 
 
@@ -446,4 +458,21 @@ def test_unit_order(ctx, D, name):
     for v in (0, 2, 3):   # CSR-S, ELL, JDS: bit-identical by construction
         if v in ys:
             assert np.array_equal(ys[v], ys[0]), v
+    plan.destroy()
+
+
+def test_hybrid_unaligned_output_view(ctx, D):
+    """the output may be any float pointer (a tensor view y[1:]):
+    the device path must not use 16-byte stores on it."""
+    import torch
+    A = MATS["heavy"]()
+    x = uniform_f32(81, A.n_cols)
+    plan = prepared(ctx, A, default=D.SPMV_DEFAULT_AUTO)
+    buf = torch.full((A.n_rows + 1,), float("nan"), device="cuda")
+    y = buf[1:]
+    for mode in (D.AUTO | D.ASYNC | D.FORCE_PROFILE, D.HYBRID | D.FORCE_PROFILE):
+        y.fill_(float("nan"))
+        ctx.spmv(plan, vec(x), y, f=0.05, mode=mode)
+        torch.cuda.synchronize()
+        assert spmv_err(A, x, y) <= SPMV_TOL
     plan.destroy()
