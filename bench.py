@@ -563,11 +563,21 @@ def secondary_workloads(ctx, D, args, stream, pk):
                      "kernel": f"dysel::spmv_claim_kernel<{r['best_variant']}> (pure full grid, cold L2)",
                      "dysel_frac": round(nb / (r["dysel_us"] * 1e-6) / 1e9 / pk["hbm_gbs"], 4)}
     out["d3x_fem_2250k"] = r
-    del A3
+    A3_keep = A3
     # D6: the paper's Case IV inputs — the scalar/vector flip
     for name, A6 in (("d6_random_16k_1pct", d6_random()), ("d6_diagonal_2M", d6_diag())):
         r, res, _ = spmv_case(A6, 6, 0.02, cold_l2=False)
         r["scalar_over_vector"] = round(res["csr_scalar"] / res["csr_vector"], 3)
+        x6 = torch.from_numpy(uniform_f32(6, A6.n_cols)).cuda()
+        rp6, col6, val6 = (torch.from_numpy(a).cuda() for a in (A6.row_ptr, A6.col, A6.val))
+        p6 = ctx.spmv_prepare(rp6, col6, val6, A6.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ALL)
+        y6 = torch.empty(A6.n_rows, device="cuda")
+        def am6():
+            ctx.spmv(p6, x6, y6, f=0.02, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE)
+            for _ in range(19):
+                ctx.spmv(p6, x6, y6, mode=D.NO_PROFILE)
+        r["amortized_overhead_pct"] = round((time_b2b(am6, 3, stream) / 20 / min(res.values()) - 1) * 100, 2)
+        p6.destroy()
         out[name] = r
     # f-4: stencil pool, Parboil-default-shaped 512 x 512 x 64 and a 512 x 512 x 256
     # grid (in + out 537 MB > 2x L2: cold HBM)
@@ -619,6 +629,7 @@ def secondary_workloads(ctx, D, args, stream, pk):
         for _ in range(19):
             ctx.spmtv(plant, xt, yt, mode=D.AUTO | D.NO_PROFILE)
     tat = time_b2b(amortt, 3, stream) / 20
+    sels_t = [ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO, report=True)["selected_name"] for _ in range(10)]
     nbt = spmv_bytes(At.n_rows, At.n_cols, At.nnz)
     out["spmtv_powerlaw_2M"] = {"nnz": int(At.nnz), "best_variant": bt, "best_us": round(tt[bt] * 1e6, 2),
                                 "best_gbs": round(nbt / tt[bt] / 1e9, 1), "dysel_us": round(tdt * 1e6, 2),
@@ -627,9 +638,11 @@ def secondary_workloads(ctx, D, args, stream, pk):
                                 "overhead_pct": round((tdt / tt[bt] - 1) * 100, 2),
                                 "host_orch_overhead_pct": round((tht / tt[bt] - 1) * 100, 2),
                                 "amortized_overhead_pct": round((tat / tt[bt] - 1) * 100, 2),
+                                "selections_10": {n: sels_t.count(n) for n in sorted(set(sels_t))},
                                 "all_us": {k: round(v * 1e6, 2) for k, v in tt.items()},
-                                "note": "y += A^T x (red.global.add per nonzero): AUTO -> swap (private copies of y, "
-                                        "winner's swapped in), f = 0.01, sync only (Table 1)"}
+                                "note": "y += A^T x (red.global.add per nonzero): AUTO -> swap, device path (A-47: "
+                                        "zeroed private outputs, the winner's reduced into y), f = 0.01, sync only "
+                                        "(Table 1); host_orch = the paper's copy-based swap"}
     plant.destroy()
     del At
     # SGEMM: D2s (Parboil small), D2m (Parboil medium), D7 8192^3 (extra, labelled)
@@ -670,6 +683,47 @@ def secondary_workloads(ctx, D, args, stream, pk):
                      "amortized_overhead_pct": round((tam / tv[bestg] - 1) * 100, 2), "amortized_iters": I,
                      "f": f_sg, "all_us": {k: round(v * 1e6, 2) for k, v in tv.items()}}
         del Ad, Bd, C
+    # (last: the x_persist placement sets a device-wide persisting L2 set-aside)
+    # f-2, Case II: x data placement pool of a CSR-scalar kernel;
+    # Case III: global-sort JDS optimisation versions
+    f2 = {}
+    for mname, Am in (("d3x_fem_2250k", A3_keep), ("d6_random_16k_1pct", d6_random()),
+                      ("powerlaw_2M_lmax256", d4_powerlaw(n=2_000_000, lmax=256))):
+        xm = torch.from_numpy(uniform_f32(7, Am.n_cols)).cuda()
+        rpm, colm, valm = (torch.from_numpy(a).cuda() for a in (Am.row_ptr, Am.col, Am.val))
+        ym = torch.empty(Am.n_rows, device="cuda")
+        plm = ctx.spmv_prepare(rpm, colm, valm, Am.n_cols)
+        jpm = ctx.spmv_jds_prepare(rpm, colm, valm, Am.n_cols)
+        for pool, names, var, run in (("placement", D.PLACE_NAMES, lambda v: ctx.spmv_placement_variant(plm, v, xm, ym),
+                                       lambda md: ctx.spmv_placement(plm, xm, ym, f=0.02, mode=md)),
+                                      ("global_jds", D.JDSG_NAMES, lambda v: ctx.spmv_jds_variant(jpm, v, xm, ym),
+                                       lambda md: ctx.spmv_jds(jpm, xm, ym, f=0.02, mode=md))):
+            tv = {names[v]: cold(lambda: var(v), 10) for v in range(4)}
+            bv = min(tv, key=tv.get)
+            md = D.AUTO | D.ASYNC | D.FORCE_PROFILE
+            td = cold(lambda: run(md), 10)
+            sels = []
+            for _ in range(10):
+                rr = (ctx.spmv_placement(plm, xm, ym, f=0.02, mode=md, report=True) if pool == "placement"
+                      else ctx.spmv_jds(jpm, xm, ym, f=0.02, mode=md, report=True))
+                sels.append(rr["selected_name"])
+            def amf2():   # the paper's Case II protocol: profiled on the first iteration only
+                run(md)
+                for _ in range(19):
+                    run(D.NO_PROFILE)
+            tam = cold(amf2, 3) / 20
+            f2[f"{pool}/{mname}"] = {"best_variant": bv, "best_us": round(tv[bv] * 1e6, 2),
+                                     "amortized_overhead_pct": round((tam / tv[bv] - 1) * 100, 2),
+                                     "all_us": {k: round(v * 1e6, 2) for k, v in tv.items()},
+                                     "dysel_us": round(td * 1e6, 2), "overhead_pct": round((td / tv[bv] - 1) * 100, 2),
+                                     "selections_10": {n: sels.count(n) for n in sorted(set(sels))},
+                                     "selected_within_5pct": round(sum(tv[n] <= 1.05 * tv[bv] for n in sels) / 10, 2)}
+        jpm.destroy()
+        plm.destroy()
+    f2["note"] = ("cold L2, AUTO|ASYNC, f = 0.02, profiling forced on; all 8 variants are bit-identical to CSR-S "
+                  "(tests/test_spmv_f2_gpu.py)")
+    out["f2_pools"] = f2
+    del A3_keep
     return out
 
 

@@ -179,6 +179,11 @@ typedef struct {
   uint64_t grid_ctas;        /* CTAs of the variant's full grid (G_n x CTAs per granule) */
   uint64_t wave_ctas;        /* CTAs resident at once (occupancy x #SM) */
   uint32_t units_per_cta;    /* wa[0] x wa[1] x wa[2] */
+  /* gated batch hint: 1 = the launcher expects this copy to win (the default
+   * variant's, launched first at high priority): launch the full grid (the
+   * block scheduler balances it); 0 = a variant that will most likely exit at
+   * the gate: one wave of CTAs walking the slice is enough */
+  uint32_t gate_full_grid;
 } dysel_slice;
 
 /* A variant = a host function that launches its kernel(s) over a slice on
@@ -384,8 +389,9 @@ dysel_status dysel_spmv_gather_probe(dysel_ctx *ctx, dysel_spmv_plan *plan, int 
  *                memory by cp.async.bulk (banded matrices; units whose window
  *                exceeds 12,288 floats gather from global memory instead)
  *   3 x_persist  as x_ldg, launched with an L2 access-policy window marking x
- *                persisting (the ctx reserves the device's maximum persisting
- *                L2 set-aside at the first call: a device-wide limit)
+ *                persisting (the ctx sets the device-wide persisting L2
+ *                set-aside to the plan's x size, 1 MB granules, capped by the
+ *                device maximum; grown per plan, released at dysel_destroy)
  * The four are bit-identical to each other and to CSR-S.  The pool is built
  * and registered at the plan's first placement call (x windows: one kernel).
  * d_x fp32 [n_cols], d_y fp32 [n_rows]; errors as dysel_spmv. */

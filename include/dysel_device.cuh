@@ -110,6 +110,7 @@ __device__ __forceinline__ void dysel_variant_decided(const dysel_slice &s) {
   if (vd == s.n_variants) {           /* last variant: publish the selection */
     __threadfence();
     const unsigned long long fin = atomicAdd((unsigned long long *)s.best, 0ull);
+    s.sel[1] = dysel_globaltimer();   /* the library's state block keeps the publish time right after sel */
     atomicExch((unsigned long long *)s.sel, fin);
   }
 }

@@ -57,6 +57,7 @@ struct DevProf {
   uint32_t pad;
   uint64_t best;
   uint64_t sel;
+  uint64_t t_publish;   // %globaltimer when the selection was published (written at sel + 1, dysel_device.cuh)
 };
 
 struct Registered {

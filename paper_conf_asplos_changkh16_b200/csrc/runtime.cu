@@ -6,6 +6,8 @@
 // (§3.3); safe-point / uniform / side-effect analyses
 // (§3.4); orchestration (§2.4); Table 1.
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <chrono>
 #include <cmath>
 #include <cstring>
@@ -201,6 +203,7 @@ __global__ void init_prof_kernel(DevProf *p, int K, int def) {
     p->variants_done = 0;
     p->best = (((1ull << 56) - 1) << 8) | (uint64_t)def;
     p->sel = ~0ull;
+    p->t_publish = 0;
   }
 }
 
@@ -469,6 +472,11 @@ void dysel_destroy(dysel_ctx *ctx) {
   if (!ctx) return;
   cudaSetDevice(ctx->device);
   cudaDeviceSynchronize();
+  if (ctx->l2_persist_bytes > 0) {   // give the L2 set-aside of the x_persist placement back
+    cudaCtxResetPersistingL2Cache();
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+    cudaGetLastError();
+  }
   spmv_ctx_free(ctx);
   for (int i = 0; i < DYSEL_MAX_VARIANTS; ++i) {
     if (ctx->fork[i]) cudaStreamDestroy(ctx->fork[i]);
@@ -709,6 +717,12 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     }
   }
   // ---- profiling copies, concurrently on forked streams
+  // diagnostics (report requested): timing events on the launching stream,
+  // the gate stream and after each phase (dysel_report.timeline_ns[2..5])
+  cudaEvent_t tev[6] = {};
+  if (rep)
+    for (auto &e : tev) cudaEventCreate(&e);
+  if (rep) cudaEventRecord(tev[0], st);
   init_prof_kernel<<<1, 32, 0, st>>>(ctx->d_prof, K, def);
   DYSEL_TRY(check_launch(ctx, "init_prof_kernel"));
   DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_start, st));
@@ -752,6 +766,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->fork[v], ctx->ev_start, 0));
     DYSEL_TRY(R.v[v].fn(&s, vargs[v].data(), ctx->fork[v], R.v[v].user));
     DYSEL_TRY(check_launch(ctx, "variant profiling copy"));
+
     DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join[v], ctx->fork[v]));
     add_slice_rec(rep, s);
     if (s.role == DYSEL_ROLE_PRODUCTIVE) mark_units(rep, s);
@@ -801,6 +816,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
       for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_join[v], 0));
     }
     DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_fork2, gate_st));
+    if (rep) cudaEventRecord(tev[1], gate_st);   // selection known
     if (P.mode == DYSEL_SWAP) {   // winner's private output copied in (after every private copy is complete)
       DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_fork2, 0));
       for (int v = 0; v < K; ++v)
@@ -825,15 +841,27 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
         s.granule_begin = rem_begin;
         s.granule_count = rem_end - rem_begin;
         s.gate = &ctx->d_prof->sel;
+        s.gate_full_grid = k == 0 ? 1u : 0u;
         DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(rs, ctx->ev_fork2, 0));
         DYSEL_TRY(R.v[v].fn(&s, base_args.data(), rs, R.v[v].user));
         DYSEL_TRY(check_launch(ctx, "variant gated batch"));
         DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join2[v], rs));
+
+      }
+      if (rep) {   // each remainder stream's completion
+        cudaEventRecord(tev[2], ctx->rem_hi);
+        for (int v = 0; v < K; ++v) cudaStreamWaitEvent(ctx->query, ctx->ev_join2[v], 0);
+        cudaEventRecord(tev[3], ctx->query);
       }
       for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join2[v], 0));
     }
     // the call completes with every profiling copy (stream semantics)
+    if (rep) {
+      for (int v = 0; v < K; ++v) cudaStreamWaitEvent(ctx->query, ctx->ev_join[v], 0);
+      cudaEventRecord(tev[4], ctx->query);   // every profiling copy done
+    }
     for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(st, ctx->ev_join[v], 0));
+    if (rep) cudaEventRecord(tev[5], st);
     // selection for the activation-flag cache: async D2H, resolved lazily
     DYSEL_TRY(push_pending_sel(ctx, key, &ctx->d_prof->sel, st));
     if (rep) {   // a report costs a D2H copy + sync
@@ -946,6 +974,26 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     }
     rep->selected = selected;
     rep->eager_units = eager_units;
+    {   // timeline: [0] first profiling CTA, [1] selection published (device paths);
+        // event-timed from the call's first kernel: [2] selection known on the
+        // gate stream, [3] the default's remainder done, [4] every remainder
+        // done, [5] every profiling copy done, [6] the call done
+      uint64_t t0 = ~0ull;
+      for (int v = 0; v < K; ++v) t0 = std::min<uint64_t>(t0, ctx->h_prof->slot[v].t_start_min);
+      for (int i = 0; i < 8; ++i) rep->timeline_ns[i] = ~0ull;
+      if (t0 != ~0ull) {
+        rep->timeline_ns[0] = 0;
+        if (!host_orch && ctx->h_prof->t_publish > t0) rep->timeline_ns[1] = ctx->h_prof->t_publish - t0;
+      }
+      if (!host_orch) {
+        cudaStreamSynchronize(st);
+        for (int i = 1; i < 6; ++i) {
+          float ms = 0.0f;
+          if (tev[i] && cudaEventElapsedTime(&ms, tev[0], tev[i]) == cudaSuccess) rep->timeline_ns[i + 1] = (uint64_t)(ms * 1e6);
+        }
+        cudaGetLastError();
+      }
+    }
     for (int v = 0; v < K; ++v) {
       const dysel_timer_slot &t = ctx->h_prof->slot[v];
       rep->makespan_ns[v] = t.t_end_max - t.t_start_min;
@@ -957,5 +1005,7 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     }
     rep->host_ns = now_ns() - t_host0;
   }
+  for (auto &e : tev)
+    if (e) cudaEventDestroy(e);
   return DYSEL_OK;
 }

@@ -83,7 +83,7 @@ static dysel_status sgemm_variant_fn(const dysel_slice *s, void *const *args, vo
   const uint64_t ctas = dysel_slice_ctas(*s, wa);
   if (ctas == 0) return DYSEL_OK;
   // gated remainder of a SIMT variant: one persistent wave (sgemm_simt_kernel)
-  const uint64_t grid = (s->gate && s->timer == nullptr && g_simt_wave[VID & 1] > 0)
+  const uint64_t grid = (s->gate && s->timer == nullptr && !s->gate_full_grid && g_simt_wave[VID & 1] > 0)
                             ? std::min<uint64_t>(ctas, g_simt_wave[VID & 1]) : ctas;
   if constexpr (VID == DYSEL_SGEMM_S64) {
     sgemm_simt_kernel<64, 64, 16, 4, 4><<<(unsigned)grid, 256, 0, st>>>(g, C, *s);

@@ -75,20 +75,17 @@ struct ProfParams {
   // default only light units seq[p_end, n_light); the winner the rest first.
   const int32_t *seq;
   uint32_t n_light;
-  // eager list (reading A-45, thread-per-row defaults only; nullptr = the
-  // light range): the light units whose longest row is <= kEagerRowTPR, in
-  // index order, and their bitmap -- an unproven thread-per-row default's
-  // eager claims take only these (its time per slot grows with the longest
-  // row); the winner then walks the whole light range and skips those done
-  const int32_t *elist;
-  const uint32_t *ebits;
-  uint32_t n_elist;
+  // reading A-45: no eager execution (ASYNC behaves as SYNC) when the
+  // initial version is a thread-per-row variant and the matrix has long-row
+  // units -- an unproven thread-per-row default is slow on exactly the rows
+  // that dominate such a matrix, and its eager work only delays the selection
+  uint32_t no_eager;
 };
 
 // eager slots of the default (published switch point S is clipped to it)
 __host__ __device__ __forceinline__ uint32_t eager_slots(const ProfParams &p) {
-  if (p.p_end >= p.n_light) return 0u;
-  return (p.elist ? p.n_elist : p.n_light - p.p_end) * (uint32_t)(kUnitRows / 32);
+  if (p.no_eager || p.p_end >= p.n_light) return 0u;
+  return (p.n_light - p.p_end) * (uint32_t)(kUnitRows / 32);
 }
 
 __global__ void spmv_state_init_kernel(SpmvState *s, int def) {
@@ -485,10 +482,7 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
   const uint32_t L1 = max(P, p.n_light);
   const uint32_t n_hs = (p.n_units - L1) * kSlots;   // winner's first range: heavy / long-row slots
   const uint32_t E = (L1 - P) * kSlots;               // light slots after the profiled prefix
-  const bool el = p.elist != nullptr && !p.pure;      // eager list mode (thread-per-row default)
   const uint32_t Ee = p.pure ? 0u : eager_slots(p);   // eager ticket range
-  const uint32_t last_prof = P > 0 ? unit_at(p, P - 1) : 0u;   // profiled light units are <= this (light-first seq)
-  uint32_t last_eager = 0;                            // el: eager-done light units are eligible and <= this
   // Claim batch: k = min(p.k_claim, remaining / (2 x warps)) >= 1 (p.k_claim
   // ~ 1024 nnz of work per claim: the counter serialises claims, ~1 per ns,
   // which capped 1-nnz rows).  Claims are made on demand: issuing the next
@@ -518,8 +512,7 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     if ((sw & 0xff) != pv) return false;
     phase = 2;
     S = min((uint32_t)(sw >> 8), Ee);
-    n_win = el ? n_hs + E : n_hs + E - S;
-    if (el && S > 0) last_eager = (uint32_t)__ldg(p.elist + S / kSlots - 1);
+    n_win = n_hs + E - S;
     t = gid;   // static first slot
     e = t < n_win ? t + 1 : t;
     return true;
@@ -574,22 +567,16 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
     }
     for (uint32_t q = t; q < e; ++q) {
       uint32_t u, w;
-      if (phase == 1) {   // eager: light slot q of seq[P, L1), or of the eager list
+      if (phase == 1) {   // eager: light slot q of seq[P, L1)
+        u = unit_at(p, P + q / kSlots);
         w = q % kSlots;
-        if (el) {
-          u = (uint32_t)__ldg(p.elist + q / kSlots);
-          if (P > 0 && u <= last_prof) continue;   // profiled already
-        } else {
-          u = unit_at(p, P + q / kSlots);
-        }
       } else if (q < n_hs) {   // winner / pure: heavy-first range seq[L1, n)
         u = unit_at(p, L1 + q / kSlots);
         w = q % kSlots;
-      } else {   // then the light slots from the switch point (el: all, minus the eager-done ones)
-        const uint32_t l = (el ? 0u : S) + (q - n_hs);
+      } else {   // then the light slots from the switch point
+        const uint32_t l = S + (q - n_hs);
         u = unit_at(p, P + l / kSlots);
         w = l % kSlots;
-        if (el && S > 0 && u <= last_eager && ((__ldg(p.ebits + (u >> 5)) >> (u & 31)) & 1u)) continue;
       }
       run_slot<VID>(A, u, (int)w, y + (size_t)u * kUnitRows);
       if (lane == 0 && p.unit_variant && w == 0) p.unit_variant[u] = (uint8_t)VID;
@@ -917,11 +904,10 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   p.def = (uint32_t)pl->def;
   p.k_claim = claim_batch(pl);
   set_order(p, pl);
-  if (pl->elist && thread_per_row(pl->vids[pl->def])) {   // reading A-45: short-row eager list
-    p.elist = pl->elist;
-    p.ebits = pl->ebits;
-    p.n_elist = pl->n_elist;
-  }
+  // reading A-45: an unproven thread-per-row default gets no eager range on a
+  // matrix with long-row units (measured on D4, JDS default: +12.9% with a
+  // short-row eager range, +9.5% without eager work)
+  p.no_eager = (pl->seq != nullptr && thread_per_row(pl->vids[pl->def])) ? 1u : 0u;
   p.abort = ((mode & DYSEL_NO_ABORT) || p.score_mode == 1) ? 0u : 1u;   // dominance needs busy or makespan
   for (int i = 0; i < pl->K; ++i) {
     p.vids[i] = pl->vids[i];

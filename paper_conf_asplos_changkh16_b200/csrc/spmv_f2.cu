@@ -198,7 +198,7 @@ static dysel_status place_variant_fn(const dysel_slice *s, void *const *args, vo
   PlaceArgs a{pl->dev, (const int2 *)pl->xwin};
   a.A.x = (const float *)args[1];
   uint64_t grid = s->granule_count;
-  if (s->timer == nullptr && s->gate != nullptr && g_place_occ[PL] > 0)   // gated remainder: one wave
+  if (s->timer == nullptr && s->gate != nullptr && !s->gate_full_grid && g_place_occ[PL] > 0)   // likely loser: one wave
     grid = std::min<uint64_t>(grid, (uint64_t)g_place_occ[PL] * pl->ctx->n_sm);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
@@ -252,12 +252,19 @@ static dysel_status place_pool(dysel_ctx *ctx, dysel_spmv_plan *pl, cudaStream_t
                                                                         pl->dev.n_rows, nu, (int2 *)pl->xwin);
     DYSEL_TRY(check_launch(ctx, "unit_window_kernel"));
   }
-  if (ctx->l2_persist_bytes == 0) {   // persisting L2 set-aside for x (placement 3)
+  {   // persisting L2 set-aside for x (placement 3): a DEVICE-wide limit that
+      // takes that much L2 from every other kernel (measured: a full-size
+      // set-aside slowed a later L2-sized stencil 2x), so it is sized to this
+      // plan's x (1 MB granules), grown only when a plan needs more, and
+      // released when the ctx is destroyed
     int maxp = 0, maxw = 0;
     cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, ctx->device);
     cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, ctx->device);
-    if (maxp > 0 && maxw > 0 && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp) == cudaSuccess) {
-      ctx->l2_persist_bytes = (size_t)maxp;
+    const size_t want = std::min<size_t>((size_t)std::max(maxp, 0),
+                                         ((size_t)pl->dev.n_cols * sizeof(float) + (1u << 20) - 1) & ~(size_t)((1u << 20) - 1));
+    if (maxw > 0 && want > ctx->l2_persist_bytes &&
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want) == cudaSuccess) {
+      ctx->l2_persist_bytes = want;
       ctx->l2_persist_window = (size_t)maxw;
     }
     cudaGetLastError();
@@ -383,7 +390,7 @@ static dysel_status jds_variant_fn(const dysel_slice *s, void *const *args, void
   if (s->granule_count == 0) return DYSEL_OK;
   JdsArgs a{jp->n_rows, jp->perm, jp->len, jp->jd_ptr, jp->col, jp->val, (const float *)args[1]};
   uint64_t grid = s->granule_count;
-  if (s->timer == nullptr && s->gate != nullptr && g_jds_occ[V] > 0)
+  if (s->timer == nullptr && s->gate != nullptr && !s->gate_full_grid && g_jds_occ[V] > 0)
     grid = std::min<uint64_t>(grid, (uint64_t)g_jds_occ[V] * jp->ctx->n_sm);
   cudaStream_t st = (cudaStream_t)stream;
   float *y = (float *)args[0];

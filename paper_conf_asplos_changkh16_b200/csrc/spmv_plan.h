@@ -27,11 +27,6 @@ struct dysel_spmv_plan {
   // light (uniform matrices, single-wave grids).
   int32_t *seq = nullptr;
   uint32_t n_light = 0;
-  // eager list for thread-per-row defaults (A-45): light units whose longest
-  // row is <= kEagerRowTPR, index order, + bitmap over units
-  int32_t *elist = nullptr;
-  uint32_t *ebits = nullptr;
-  uint32_t n_elist = 0;
   std::string sig;                    // generic-registry signature (host path)
   // f-2 placement pool (spmv_f2.cu): per-unit x windows (int2 [n_units]), registry sig
   void *xwin = nullptr;
@@ -41,7 +36,6 @@ struct dysel_spmv_plan {
 namespace dysel {
 constexpr int64_t kHeavyUnitNnz = 8192;   // a unit with >= max(this, 4 x mean) nonzeros is heavy (A-40)
 constexpr int64_t kLongRow = 1024;        // a unit with a row longer than max(this, 8 x mean row) is long (A-45)
-constexpr int64_t kEagerRowTPR = 128;     // eager units of a thread-per-row default: longest row <= this (A-45)
 int spmv_pool_index(const dysel_spmv_plan *pl, int vid);
 // register the plan's pool with the generic launcher (host-orchestrated path)
 dysel_status spmv_register_pool(dysel_ctx *ctx, dysel_spmv_plan *pl);

@@ -288,22 +288,6 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
         if (cudaMemcpy(pl->seq, seq.data(), nu * 4, cudaMemcpyHostToDevice) != cudaSuccess) return fail(DYSEL_ERR_CUDA);
         pl->n_light = (uint32_t)light.size();
         I.n_heavy = (int32_t)rest.size();
-        std::vector<int32_t> el;
-        std::vector<uint32_t> bits((nu + 31) / 32, 0u);
-        for (int32_t u : light)
-          if ((int64_t)um[u] <= kEagerRowTPR) {
-            el.push_back(u);
-            bits[u >> 5] |= 1u << (u & 31);
-          }
-        if (!el.empty()) {
-          if (cudaMalloc(&pl->elist, el.size() * 4) != cudaSuccess ||
-              cudaMalloc(&pl->ebits, bits.size() * 4) != cudaSuccess)
-            return fail(DYSEL_ERR_NOMEM);
-          if (cudaMemcpy(pl->elist, el.data(), el.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
-              cudaMemcpy(pl->ebits, bits.data(), bits.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
-            return fail(DYSEL_ERR_CUDA);
-          pl->n_elist = (uint32_t)el.size();
-        }
       }
     }
     I.n_light = pl->seq ? (int32_t)pl->n_light : (int32_t)nu;
@@ -398,8 +382,6 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *pl) {
   cudaFree(pl->jd_off);
   cudaFree(pl->seq);
   cudaFree(pl->xwin);
-  cudaFree(pl->elist);
-  cudaFree(pl->ebits);
   cudaGetLastError();
   delete pl;
 }

@@ -246,7 +246,8 @@ static dysel_status stencil_variant_fn(const dysel_slice *s, void *const *args, 
   if (ctas == 0) return DYSEL_OK;
   // gated remainder: one persistent wave (a variant that lost the selection
   // then costs one wave of exiting CTAs instead of one per tile: 130K for base)
-  if (s->gate && !s->timer && g_stencil_wave[VID] > 0) ctas = std::min<uint64_t>(ctas, g_stencil_wave[VID]);
+  if (s->gate && !s->timer && !s->gate_full_grid && g_stencil_wave[VID] > 0)
+    ctas = std::min<uint64_t>(ctas, g_stencil_wave[VID]);
   if constexpr (VID == DYSEL_STENCIL_BASE)
     stencil_base_kernel<<<(unsigned)ctas, 128, 0, st>>>(g, out, *s);
   else if constexpr (VID == DYSEL_STENCIL_ZMARCH) {
@@ -271,6 +272,7 @@ dysel_status stencil_register(dysel_ctx *ctx) {
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], stencil_tiled_kernel, 128, 0);
   cudaGetLastError();
   const uint64_t n = (uint64_t)ctx->n_sm;
+  for (int i = 0; i < DYSEL_STENCIL_NVARIANTS; ++i) g_stencil_wave[i] = (uint64_t)o[i] * n;
   dysel_variant v[DYSEL_STENCIL_NVARIANTS] = {
       {"base", kStencilFns[0], {1, 1, 1}, sb, 1, 0, nullptr, (uint64_t)o[0] * n},
       {"zmarch64", kStencilFns[1], {1, 1, 64}, sb, 1, 0, nullptr, (uint64_t)o[1] * n},
