@@ -726,7 +726,10 @@ static bool thread_per_row(int vid) {
 }
 
 // Slots per claim: about kClaimNnz nonzeros of work (at least 1, at most a unit).
-constexpr int64_t kClaimNnz = 1024;
+#ifndef DYSEL_CLAIM_NNZ
+#define DYSEL_CLAIM_NNZ 4096
+#endif
+constexpr int64_t kClaimNnz = DYSEL_CLAIM_NNZ;
 static uint32_t claim_batch(const dysel_spmv_plan *pl) {
   const int64_t slots = (int64_t)pl->n_units * kSlots;
   const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
