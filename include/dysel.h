@@ -459,8 +459,10 @@ dysel_status dysel_sgemm_variant(dysel_ctx *ctx, int variant_id, int M, int N, i
  * variants are bit-identical); boundary points (any coordinate 0 or n-1):
  * out = in (reading A-37).  Unit = 32 x 4 x 1 points.  Built-in variants:
  * 0 base (thread per point, wa 1x1x1), 1 z-march (thread per (x, y) column
- * over 64 z-planes, wa 1x1x64), 2 tiled (64x4 tile staged plane by plane in
- * shared memory + z-march, wa 2x1x64).  nx, ny, nz >= 0 (0 volume: no-op);
+ * over 64 z-planes, wa 1x1x64), 2 TMA tile (128x8x16 points: each z-plane of
+ * the tile plus its y / x halo streamed by TMA into a shared-memory ring,
+ * persistent CTAs, wa 4x2x16; needs nx % 4 == 0 and 16-byte aligned buffers,
+ * else the same items run the z-march column code).  nx, ny, nz >= 0 (0 volume: no-op);
  * DYSEL_ERR_INVALID for NULL or aliased buffers. */
 enum { DYSEL_STENCIL_BASE = 0, DYSEL_STENCIL_ZMARCH = 1, DYSEL_STENCIL_TILED = 2, DYSEL_STENCIL_NVARIANTS = 3 };
 dysel_status dysel_stencil(dysel_ctx *ctx, int nx, int ny, int nz, float c0, float c1, const float *d_in,

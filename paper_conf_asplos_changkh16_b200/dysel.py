@@ -41,7 +41,7 @@ FMT_DEFAULT = FMT_ELL | FMT_JDS | FMT_STREAM
 SPMV_DEFAULT_AUTO = -1
 SGEMM_S64, SGEMM_S128, SGEMM_T128x64, SGEMM_T128x128 = range(4)
 SGEMM_NAMES = ["simt64x64", "simt128x128", "tc3xtf32_128x64", "tc3xtf32_128x128"]
-STENCIL_NAMES = ["base", "zmarch64", "tiled64x4_zmarch64"]
+STENCIL_NAMES = ["base", "zmarch64", "tma128x8x16"]
 SPMTV_NAMES = ["scatter_thread", "scatter_warp", "scatter_segment"]
 STENCIL_BASE, STENCIL_ZMARCH, STENCIL_TILED = range(3)
 PLACE_LDG, PLACE_L2, PLACE_SMEM, PLACE_PERSIST = range(4)

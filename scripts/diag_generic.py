@@ -21,20 +21,28 @@ def show(name, T, run, modes):
               f"eager {r['eager_units']} tl_us {[None if v is None else round(v/1e3,1) for v in r['timeline_ns']]}", flush=True)
 modes = [("fully_sync", D.FULLY | D.FORCE_PROFILE), ("fully_async", D.FULLY | D.ASYNC | D.FORCE_PROFILE),
          ("hybrid_async", D.HYBRID | D.ASYNC | D.FORCE_PROFILE), ("no_abort", D.FULLY | D.NO_ABORT | D.FORCE_PROFILE)]
-a3 = torch.from_numpy(uniform_f32(64, (256, 512, 512))).cuda(); o3 = torch.empty_like(a3)
-T = {D.STENCIL_NAMES[v]: time_b2b(lambda: ctx.stencil_variant(v, a3, o3, 0.8, 0.15), 10, s) for v in range(3)}
-show("stencil 512x512x256", T, lambda md, rep: ctx.stencil(a3, o3, 0.8, 0.15, f=0.02, mode=md, report=rep), modes)
-del a3, o3
-A = d3_fem(grid=1500)
-x = torch.from_numpy(uniform_f32(7, A.n_cols)).cuda()
-rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
-y = torch.empty(A.n_rows, device="cuda")
-pl = ctx.spmv_prepare(rp, col, val, A.n_cols)
-T = {D.PLACE_NAMES[v]: time_b2b(lambda: ctx.spmv_placement_variant(pl, v, x, y), 10, s) for v in range(4)}
-show("placement d3x", T, lambda md, rep: ctx.spmv_placement(pl, x, y, f=0.02, mode=md, report=rep), modes)
-jp = ctx.spmv_jds_prepare(rp, col, val, A.n_cols)
-T = {D.JDSG_NAMES[v]: time_b2b(lambda: ctx.spmv_jds_variant(jp, v, x, y), 10, s) for v in range(4)}
-show("global jds d3x", T, lambda md, rep: ctx.spmv_jds(jp, x, y, f=0.02, mode=md, report=rep), modes)
+ONLY = sys.argv[1] if len(sys.argv) > 1 else None   # stencil | f2 | sgemm
+for nz in (64, 256):
+    if ONLY not in (None, "stencil"):
+        break
+    a3 = torch.from_numpy(uniform_f32(64, (nz, 512, 512))).cuda(); o3 = torch.empty_like(a3)
+    T = {D.STENCIL_NAMES[v]: time_b2b(lambda: ctx.stencil_variant(v, a3, o3, 0.8, 0.15), 10, s) for v in range(3)}
+    show(f"stencil 512x512x{nz}", T, lambda md, rep: ctx.stencil(a3, o3, 0.8, 0.15, f=0.02, mode=md, report=rep),
+         modes)
+    del a3, o3
+if ONLY == "stencil":
+    sys.exit(0)
+if ONLY != "sgemm":
+  A = d3_fem(grid=1500)
+  x = torch.from_numpy(uniform_f32(7, A.n_cols)).cuda()
+  rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
+  y = torch.empty(A.n_rows, device="cuda")
+  pl = ctx.spmv_prepare(rp, col, val, A.n_cols)
+  T = {D.PLACE_NAMES[v]: time_b2b(lambda: ctx.spmv_placement_variant(pl, v, x, y), 10, s) for v in range(4)}
+  show("placement d3x", T, lambda md, rep: ctx.spmv_placement(pl, x, y, f=0.02, mode=md, report=rep), modes)
+  jp = ctx.spmv_jds_prepare(rp, col, val, A.n_cols)
+  T = {D.JDSG_NAMES[v]: time_b2b(lambda: ctx.spmv_jds_variant(jp, v, x, y), 10, s) for v in range(4)}
+  show("global jds d3x", T, lambda md, rep: ctx.spmv_jds(jp, x, y, f=0.02, mode=md, report=rep), modes)
 M = K = N = 4096
 Ah, Bh, _ = sgemm_inputs(M, K, N, 5, 6)
 Ad, Bd = torch.from_numpy(Ah).cuda(), torch.from_numpy(Bh).cuda()

@@ -20,3 +20,7 @@ for shape in ((64, 512, 512), (256, 512, 512)):
     r = {D.STENCIL_NAMES[v]: b2b(lambda: ctx.stencil_variant(v, a, o, 0.8, 0.15)) for v in range(3)}
     t = b2b(lambda: ctx.stencil(a, o, 0.8, 0.15, f=0.02, mode=D.FULLY | D.ASYNC))
     print(shape, {k: f"{v:.1f}us {nb / v / 1e3:.0f}GB/s" for k, v in r.items()}, f"dysel {t:.1f}us", flush=True)
+    for m, mn in ((D.FULLY, "fully"), (D.FULLY | D.ASYNC, "fully_async")):
+        rep = ctx.stencil(a, o, 0.8, 0.15, f=0.02, mode=m | D.FORCE_PROFILE, report=True)
+        print("  ", mn, rep["selected_name"], "c", rep["c"], "score", rep["score"][:3], "units", rep["units"][:3],
+              "busy_us", [round(b / 1e3, 1) for b in rep["busy_ns"][:3]], flush=True)

@@ -84,7 +84,7 @@ def test_deactivated_small_and_invalid(ctx):
     inp = torch.from_numpy(a).cuda()
     out = torch.empty_like(inp)
     rep = ctx.stencil(inp, out, C0, C1, report=True)
-    assert not rep["profiled"] and rep["selected"] == D.STENCIL_ZMARCH   # < 128 CTAs: default
+    assert not rep["profiled"] and rep["selected"] == D.STENCIL_TILED   # < 128 CTAs: default
     assert ost.rel_error(out.cpu().numpy(), ost.stencil(a, C0, C1), ost.stencil_abs(a, C0, C1)) <= ost.STENCIL_TOL
     with pytest.raises(Exception):
         ctx.stencil(inp, inp, C0, C1)                            # in-place is not a Jacobi step
@@ -93,7 +93,7 @@ def test_deactivated_small_and_invalid(ctx):
 @pytest.mark.parametrize("shape,f,mode_name", [((256, 64, 512), 0.1, "fully"), ((130, 37, 700), 0.05, "hybrid"),
                                                ((64, 256, 256), 0.3, "fully_contig")])
 def test_stencil_plan_matches_oracle(ctx, shape, f, mode_name):
-    """a-2 with a 3-D LCM granule (2 x 1 x 64 units): the library's slice plan
+    """a-2 with a 3-D LCM granule (4 x 2 x 64 units): the library's slice plan
     and per-granule producers equal the oracle's (c-5, c-6)."""
     import torch
     from paper_conf_asplos_changkh16_b200 import dysel as D
@@ -104,7 +104,7 @@ def test_stencil_plan_matches_oracle(ctx, shape, f, mode_name):
     rep = ctx.stencil(inp, out, C0, C1, f=f, mode=mode, report=True, unit_map=True)
     torch.cuda.synchronize()
     U = (-(-nx // 32), -(-ny // 4), nz)
-    p = slice_plan.plan(U, [(1, 1, 1), (1, 1, 64), (2, 1, 64)], f, ctx.n_sm, D.STENCIL_ZMARCH, mode)
+    p = slice_plan.plan(U, [(1, 1, 1), (1, 1, 64), (4, 2, 16)], f, ctx.n_sm, D.STENCIL_TILED, mode)
     assert rep["c"] == p.c and rep["n_granules"] == p.Gn and rep["profiled"] == p.active
     owner = slice_plan.productive_cover(p, rep["selected"])
     assert list(rep["unit_variant"][:p.Gn]) == owner     # sync: profiled slices + the winner's remainder
