@@ -526,7 +526,11 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
   for (;;) {
     if (t >= e) {   // need a claim
       if (phase == 1) {
-        const uint32_t k = batch(Ee - min(e, Ee));
+        // CSR-V's warp walks its slot's 32 rows one after another (~1 us each):
+        // an eager batch of several slots would hold a losing default's warps
+        // (and their SM slots) for ~100 us after the selection; one slot per
+        // claim bounds that drain to one slot
+        const uint32_t k = VID == DYSEL_SPMV_CSR_VECTOR ? 1u : batch(Ee - min(e, Ee));
         const uint64_t r = claim(k);
         t = (uint32_t)r;
         uint32_t lim = Ee;

@@ -7,6 +7,7 @@ import numpy as np, torch
 from paper_conf_asplos_changkh16_b200 import dysel as D
 from workloads import d3_fem, uniform_f32
 grid = int(sys.argv[1]) if len(sys.argv) > 1 else 1500
+FS = [float(v) for v in sys.argv[2].split(",")] if len(sys.argv) > 2 else (0.02, 0.05)
 ctx = D.Context(0)
 A = d3_fem(grid=grid)
 x = torch.from_numpy(uniform_f32(385, A.n_cols)).cuda()
@@ -29,7 +30,7 @@ for fm, name in ((D.FMT_ALL, "all"), (D.FMT_DEFAULT, "default")):
     for mname, mode in (("fully_async", D.FULLY | D.ASYNC), ("fully_sync", D.FULLY), ("makespan", D.FULLY | D.ASYNC |
                          D.SCORE_MAKESPAN), ("cycles", D.FULLY | D.ASYNC | D.SCORE_CYCLES),
                         ("seq", D.FULLY | D.SEQUENTIAL), ("hybrid_async", D.HYBRID | D.ASYNC)):
-        for f in (0.02, 0.05):
+        for f in FS:
             t = cold(lambda: ctx.spmv(plan, x, y, f=f, mode=mode))
             sels = [ctx.spmv(plan, x, y, f=f, mode=mode, report=True) for _ in range(5)]
             r = sels[-1]
