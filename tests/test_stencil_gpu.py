@@ -8,9 +8,9 @@ from oracle import stencil as ost
 
 pytestmark = pytest.mark.gpu
 
-# (nz, ny, nx); nx % 4 == 0 takes the TMA z-march (plane ring), the others its register form
+# (nz, ny, nx); nx % 4 == 0 takes V2's TMA plane ring, the others its z-march column fallback
 SHAPES = [(130, 37, 70), (64, 64, 64), (3, 5, 33), (1, 1, 1), (4, 3, 2), (70, 9, 200), (65, 6, 36), (200, 3, 8),
-          (2, 2, 4)]
+          (2, 2, 4), (37, 100, 260), (17, 8, 128), (16, 9, 132)]
 C0, C1 = 0.8125, 0.15625
 
 
@@ -110,11 +110,12 @@ def test_stencil_plan_matches_oracle(ctx, shape, f, mode_name):
     assert list(rep["unit_variant"][:p.Gn]) == owner     # sync: profiled slices + the winner's remainder
 
 
-def test_tma_zmarch_multi_tile_ring(ctx):
-    """A grid of 8,192 z-march tiles (> one wave of 16 CTAs/SM): every CTA of
-    the persistent TMA z-march walks several tiles, its mbarrier phase
-    sequence running on across them.  All variants stay bit-identical; the
-    oracle is checked on sampled z-planes (boundary, granule edges, interior)."""
+def test_tma_tile_multi_item_ring(ctx):
+    """2,048 V2 items over one persistent wave (4 full round-robin rounds and
+    a last round split in z over all CTAs): every CTA's plane ring and its
+    mbarrier phases run on across items.  All variants stay bit-identical; the
+    oracle is checked on sampled z-planes (boundary, item / granule edges,
+    interior)."""
     import torch
     from paper_conf_asplos_changkh16_b200 import dysel as D
     shape = (256, 256, 512)
@@ -138,3 +139,28 @@ def test_tma_zmarch_multi_tile_ring(ctx):
             assert ost.rel_error(o[z], ref, den) <= ost.STENCIL_TOL, z
         else:
             assert np.array_equal(o[z], a[z]), z
+
+
+def test_tma_tile_unaligned_view_fallback(ctx):
+    """V2 on buffers that are not 16-byte aligned (a view one float into the
+    allocation) cannot use TMA: the same items run the z-march column code,
+    bit-identical to the other variants and to V2 on aligned buffers."""
+    import torch
+    shape = (40, 24, 136)
+    a = field(shape, 12)
+    n = a.size
+    big_in = torch.zeros(n + 4, device="cuda")
+    big_out = torch.full((n + 4,), float("nan"), device="cuda")
+    inp = big_in[1:n + 1].view(shape)
+    inp.copy_(torch.from_numpy(a))
+    out_u = big_out[1:n + 1].view(shape)
+    ctx.stencil_variant(2, inp, out_u, C0, C1)
+    out_a = torch.empty(shape, device="cuda")
+    ctx.stencil_variant(2, inp.contiguous().clone(), out_a, C0, C1)
+    out_z = torch.empty(shape, device="cuda")
+    ctx.stencil_variant(1, inp, out_z, C0, C1)
+    torch.cuda.synchronize()
+    assert torch.equal(out_u.view(torch.int32), out_a.view(torch.int32))
+    assert torch.equal(out_u.view(torch.int32), out_z.view(torch.int32))
+    assert ost.rel_error(out_u.cpu().numpy(), ost.stencil(a, C0, C1), ost.stencil_abs(a, C0, C1)) <= ost.STENCIL_TOL
+    assert torch.isnan(big_out[0]) and torch.isnan(big_out[n + 1])   # nothing written outside the view
