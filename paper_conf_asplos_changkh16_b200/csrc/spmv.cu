@@ -63,7 +63,9 @@ struct ProfParams {
   uint32_t hybrid, async, contiguous, score_mode, def, abort;
   uint64_t *host_sel;    // mapped pinned word: the publishing CTA writes the selection here (cache)
   int32_t vids[DYSEL_SPMV_NVARIANTS];
-  uint32_t occ[DYSEL_SPMV_NVARIANTS];
+  uint32_t occ[DYSEL_SPMV_NVARIANTS];     // claim-kernel occupancy (remainder grids)
+  uint32_t occ_t[DYSEL_SPMV_NVARIANTS];   // score normalisation: the co-residency the units were timed at
+                                          // (grouped profiling: min(occ, units per CTA), A-49), else occ
   float *sandbox;        // (K - 1) * c * 256 floats (hybrid: every variant but the default, A-4)
   uint64_t *tl;          // SpmvState::tl when a report is requested, else nullptr (no timeline atomics)
   uint8_t *unit_variant; // optional debug map (variant id per unit)
@@ -80,6 +82,9 @@ struct ProfParams {
   // units -- an unproven thread-per-row default is slow on exactly the rows
   // that dominate such a matrix, and its eager work only delays the selection
   uint32_t no_eager;
+  uint32_t part_first;   // grouped profiling (A-49): pool index of the first launch (it waits for the init kernel)
+  uint32_t n_grp;        // ... pool indices profiled by the combined grouped kernel
+  uint32_t grp_pv[DYSEL_SPMV_NVARIANTS];
 };
 
 // eager slots of the default (published switch point S is clipped to it)
@@ -294,17 +299,33 @@ __device__ __forceinline__ uint32_t unit_at(const ProfParams &p, uint32_t i) {
   return p.seq ? (uint32_t)__ldg(p.seq + i) : i;
 }
 
-// One profiling unit of variant VID (pool index pv): the b-th unit of its slice.
+// Shared state of one profiled unit (one per 256-thread unit group).
+struct ProfUnitSmem {
+  unsigned long long s_last, s_start;
+  int s_abort, s_skip;
+  dysel_prof_smem psm;
+};
+// barrier of a unit group: the whole CTA (grp 0) or named barrier grp (256 threads)
+__device__ __forceinline__ void unit_sync(int grp) {
+  if (grp == 0)
+    __syncthreads();
+  else
+    asm volatile("bar.sync %0, 256;" ::"r"(grp) : "memory");
+}
+
+// One profiling unit of variant VID (pool index pv): the b-th unit of its
+// slice, run by the 256 threads of unit group grp (threadIdx.x / 256).
 template <int VID>
 __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ y, SpmvState *st,
-                                          const ProfParams &p, uint32_t pv, uint32_t b) {
-  __shared__ unsigned long long s_last, s_start;
-  __shared__ int s_abort, s_skip;
-  __shared__ dysel_prof_smem psm;
-  const uint32_t tid = threadIdx.x;
+                                          const ProfParams &p, uint32_t pv, uint32_t b, ProfUnitSmem &sm,
+                                          int grp) {
+  unsigned long long &s_last = sm.s_last, &s_start = sm.s_start;
+  int &s_abort = sm.s_abort, &s_skip = sm.s_skip;
+  dysel_prof_smem &psm = sm.psm;
+  const uint32_t tid = threadIdx.x & (kUnitRows - 1);
   // predicted full-grid time of a variant (A-6): max(throughput bound, longest
   // unit); throughput bound = busy_sum * G_n / (c * occupancy * #SM)
-  const uint64_t thr_den = (uint64_t)p.c * max(1u, p.occ[pv]) * max(1u, p.n_sm);
+  const uint64_t thr_den = (uint64_t)p.c * max(1u, p.occ_t[pv]) * max(1u, p.n_sm);
   const uint32_t jj = p.hybrid ? b : (p.contiguous ? pv * p.c + b : pv + p.K * b);   // position in seq
   const uint32_t j = unit_at(p, jj);
   // hybrid (reading A-4): every variant runs the same units; the
@@ -320,7 +341,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     if (!s_skip) atomicMin((unsigned long long *)&st->slot[pv].t_start_min, s_last);   // variant start (makespan)
     if (p.tl) atomicMin((unsigned long long *)&p.tl[0], s_last);
   }
-  __syncthreads();
+  unit_sync(grp);
   const bool skipped = s_skip != 0;
   const uint32_t sb = pv < p.def ? pv : pv - 1;   // sandbox slot of a non-default variant (K - 1 of them)
   float *out = productive ? y + (size_t)j * kUnitRows : p.sandbox + ((size_t)sb * p.c + b) * kUnitRows;
@@ -335,23 +356,23 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     // loops measured +60% per-unit time on D4 (CSR-W 15 -> 24.6 us).
     constexpr bool kPolled = VID == 0 || VID == 2 || VID == 3 || VID == 5;
     if (kPolled && p.abort && sandbox)
-      run_unit<VID>(A, j, out,
+      run_slot<VID>(A, j, (int)(tid >> 5), out,
                     ProfPoll<false>{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
                                     &st->decided[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
                                     p.score_mode == 2 ? 1u : 0u, pub});
     else if (kPolled && p.abort)
-      run_unit<VID>(A, j, out,
+      run_slot<VID>(A, j, (int)(tid >> 5), out,
                     ProfPoll<true>{&s_last, &s_start, &s_abort, (unsigned long long *)&st->lb[pv], &st->best_total,
                                    &st->decided[pv], &st->slot[pv].t_start_min, (uint64_t)p.n_units, thr_den,
                                    p.score_mode == 2 ? 1u : 0u, pub});
     else
-      run_unit<VID>(A, j, out, NoPoll());
+      run_slot<VID>(A, j, (int)(tid >> 5), out, NoPoll());
     if ((tid & 31) == 0) {
       psm.t1[tid >> 5] = dysel_globaltimer();
       psm.c1[tid >> 5] = dysel_clock64();
     }
   }
-  __syncthreads();
+  unit_sync(grp);
   if (tid >= 32) return;
   // warp-shuffle reduction of the per-warp samples (min start, max end)
   unsigned long long t0 = tid < 8 ? psm.t0[tid] : ~0ull, t1 = tid < 8 ? psm.t1[tid] : 0ull;
@@ -406,7 +427,52 @@ template <int VID>
 __global__ void __launch_bounds__(kUnitRows, kSliceMinBlocks[VID])
     spmv_prof_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
   if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
-  prof_unit<VID>(A, y, st, p, pv, blockIdx.x);
+  __shared__ ProfUnitSmem sm;
+  prof_unit<VID>(A, y, st, p, pv, blockIdx.x, sm, 0);
+}
+
+// Grouped profiling copy of one variant (reading A-49): each CTA runs
+// kProfGroups(VID) profiled units at once, one per 256-thread group (named
+// barriers), so a unit is timed beside as many units of its own variant as
+// the claim kernel keeps resident per SM (up to 4; CSR-T's staging buffers
+// allow one) — the per-SM load of the full run (L1 / LSU / gather rate)
+// instead of one unit alone on an SM, which hid CSR-S's LSU saturation on
+// regular matrices.  The K launches are chained by PDL and run concurrently;
+// only the first waits for the init kernel (the others start after all of
+// its CTAs passed that wait).
+__host__ __device__ constexpr int kProfGroups(int vid) { return vid == DYSEL_SPMV_CSR_TMA ? 3 : 4; }
+// The K_g variants without staging buffers in ONE grouped launch (CTA b:
+// variant grp_pv[b % K_g], its units 4 (b / K_g) .. + 3), so the PDL chain in
+// front of the eager claim kernel is one or two launches, not K.
+__global__ void __launch_bounds__(kUnitRows * 4, 1)
+    spmv_prof_grp_all_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  __shared__ ProfUnitSmem sm[4];
+  const uint32_t pv = p.grp_pv[blockIdx.x % p.n_grp];
+  const int g = (int)(threadIdx.x / kUnitRows);
+  const uint32_t b = (blockIdx.x / p.n_grp) * 4 + (uint32_t)g;
+  if (b >= p.c) return;
+  switch (p.vids[pv]) {
+    case 0: prof_unit<0>(A, y, st, p, pv, b, sm[g], g + 1); break;
+    case 1: prof_unit<1>(A, y, st, p, pv, b, sm[g], g + 1); break;
+    case 2: prof_unit<2>(A, y, st, p, pv, b, sm[g], g + 1); break;
+    case 3: prof_unit<3>(A, y, st, p, pv, b, sm[g], g + 1); break;
+    default: prof_unit<4>(A, y, st, p, pv, b, sm[g], g + 1); break;
+  }
+}
+
+template <int VID>
+__global__ void __launch_bounds__(kUnitRows * kProfGroups(VID), 1)
+    spmv_prof_grp_kernel(SpmvDev A, float *__restrict__ y, SpmvState *st, ProfParams p, uint32_t pv) {
+  constexpr int G = kProfGroups(VID);
+  if constexpr (VID == DYSEL_SPMV_CSR_TMA) tma_stage_prologue();
+  if (pv == p.part_first) asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  __shared__ ProfUnitSmem sm[G];
+  const int g = (int)(threadIdx.x / kUnitRows);
+  const uint32_t b = blockIdx.x * G + (uint32_t)g;
+  if (b < p.c) prof_unit<VID>(A, y, st, p, pv, b, sm[g], G > 1 ? g + 1 : 0);
 }
 
 // All K profiling slices in ONE launch (no forked streams / joins): CTA b runs
@@ -426,13 +492,14 @@ __global__ void __launch_bounds__(kUnitRows, 1)
   // may start as soon as every profiling CTA is resident
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const uint32_t pv = blockIdx.x % p.K, b = blockIdx.x / p.K;
+  __shared__ ProfUnitSmem sm;
   switch (p.vids[pv]) {
-    case 0: prof_unit<0>(A, y, st, p, pv, b); break;
-    case 1: prof_unit<1>(A, y, st, p, pv, b); break;
-    case 2: prof_unit<2>(A, y, st, p, pv, b); break;
-    case 3: prof_unit<3>(A, y, st, p, pv, b); break;
-    case 4: prof_unit<4>(A, y, st, p, pv, b); break;
-    default: prof_unit<5>(A, y, st, p, pv, b); break;
+    case 0: prof_unit<0>(A, y, st, p, pv, b, sm, 0); break;
+    case 1: prof_unit<1>(A, y, st, p, pv, b, sm, 0); break;
+    case 2: prof_unit<2>(A, y, st, p, pv, b, sm, 0); break;
+    case 3: prof_unit<3>(A, y, st, p, pv, b, sm, 0); break;
+    case 4: prof_unit<4>(A, y, st, p, pv, b, sm, 0); break;
+    default: prof_unit<5>(A, y, st, p, pv, b, sm, 0); break;
   }
 }
 
@@ -530,7 +597,11 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
         // an eager batch of several slots would hold a losing default's warps
         // (and their SM slots) for ~100 us after the selection; one slot per
         // claim bounds that drain to one slot
-        const uint32_t k = VID == DYSEL_SPMV_CSR_VECTOR ? 1u : batch(Ee - min(e, Ee));
+        // Other variants but CSR-W (whose slots take a few us): at most 2 slots
+        // per eager claim, which bounds a losing default's drain to ~2 slots.
+        const uint32_t k = VID == DYSEL_SPMV_CSR_VECTOR ? 1u
+                           : VID == DYSEL_SPMV_CSR_STREAM ? batch(Ee - min(e, Ee))
+                                                          : min(2u, batch(Ee - min(e, Ee)));
         const uint64_t r = claim(k);
         t = (uint32_t)r;
         uint32_t lim = Ee;
@@ -606,6 +677,9 @@ __global__ void spmv_switch_kernel(SpmvDev A, float *__restrict__ y, SpmvState *
   const uint64_t sw = wait_published(&st->sw);
   const uint32_t w = (uint32_t)(sw & 0xff);
   if (w == p.def || w >= p.K || p.p_end >= p.n_units) return;
+  // CSR-T's claim kernel is host-launched behind this one (its shared-memory
+  // carveout is not applied to a device-side launch: it ran at half speed)
+  if (p.vids[w] == DYSEL_SPMV_CSR_TMA) return;
   const unsigned g = (unsigned)min((uint64_t)p.occ[w] * p.n_sm, (uint64_t)(p.n_units - p.p_end));
   const cudaStream_t ff = cudaStreamFireAndForget;
   switch (p.vids[w]) {
@@ -658,13 +732,19 @@ dysel_status spmv_ctx_init(dysel_ctx *ctx) {
   const void *claim[DYSEL_SPMV_NVARIANTS] = {(const void *)spmv_claim_kernel<0>, (const void *)spmv_claim_kernel<1>,
                                             (const void *)spmv_claim_kernel<2>, (const void *)spmv_claim_kernel<3>,
                                             (const void *)spmv_claim_kernel<4>, (const void *)spmv_claim_kernel<5>};
+  const void *part[DYSEL_SPMV_NVARIANTS] = {
+      (const void *)spmv_prof_grp_kernel<0>, (const void *)spmv_prof_grp_kernel<1>,
+      (const void *)spmv_prof_grp_kernel<2>, (const void *)spmv_prof_grp_kernel<3>,
+      (const void *)spmv_prof_grp_kernel<4>, (const void *)spmv_prof_grp_kernel<5>};
   {   // CSR-T's staging buffers exceed the 48 KB default dynamic limit
     const int m = (int)dyn_smem(DYSEL_SPMV_CSR_TMA);
     const void *k5[] = {(const void *)spmv_slice_kernel<5>, (const void *)spmv_slice_timed_kernel<5>,
                         (const void *)spmv_claim_kernel<5>, (const void *)spmv_prof_kernel<5>,
-                        (const void *)spmv_prof_all_kernel};
+                        (const void *)spmv_prof_all_kernel, (const void *)spmv_prof_grp_kernel<5>};
     for (const void *k : k5)
-      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, m) != cudaSuccess) return DYSEL_ERR_CUDA;
+      if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               k == (const void *)spmv_prof_grp_kernel<5> ? m * kProfGroups(5) : m) != cudaSuccess)
+        return DYSEL_ERR_CUDA;
   }
   for (int v = 0; v < DYSEL_SPMV_NVARIANTS; ++v) {
     // largest L1 for the gathers; CSR-T holds its staging buffers in shared
@@ -676,6 +756,7 @@ dysel_status spmv_ctx_init(dysel_ctx *ctx) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_slice[v], slice[v], kUnitRows, dyn_smem(v));
     cudaFuncSetAttribute(claim[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&s->occ_claim[v], claim[v], kUnitRows, dyn_smem(v));
+    cudaFuncSetAttribute(part[v], cudaFuncAttributePreferredSharedMemoryCarveout, carve);
   }
   return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
 }
@@ -734,6 +815,10 @@ static bool thread_per_row(int vid) {
 #define DYSEL_CLAIM_NNZ 4096
 #endif
 constexpr int64_t kClaimNnz = DYSEL_CLAIM_NNZ;
+#ifndef DYSEL_GROUPED_PROFILING
+#define DYSEL_GROUPED_PROFILING 1
+#endif
+constexpr bool kGroupedProfiling = DYSEL_GROUPED_PROFILING != 0;   // reading A-49
 static uint32_t claim_batch(const dysel_spmv_plan *pl) {
   const int64_t slots = (int64_t)pl->n_units * kSlots;
   const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
@@ -767,6 +852,23 @@ static void launch_prof(const SpmvDev &A, float *y, SpmvState *st, const ProfPar
   spmv_prof_kernel<VID><<<p.c, kUnitRows, dyn_smem(VID), s>>>(A, y, st, p, pv);
 }
 typedef void (*ProfLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, uint32_t, cudaStream_t);
+static cudaError_t launch_pdl(const void *fn, dim3 grid, dim3 block, size_t smem, cudaStream_t st, void **args);
+template <int VID>
+static cudaError_t launch_part(const SpmvDev &A, float *y, SpmvState *st, const ProfParams &p, uint32_t pv,
+                               unsigned grid, cudaStream_t s) {
+  SpmvDev a = A;
+  float *yy = y;
+  SpmvState *ss = st;
+  ProfParams pp = p;
+  uint32_t v = pv;
+  void *args[] = {&a, &yy, &ss, &pp, &v};
+  return launch_pdl((const void *)spmv_prof_grp_kernel<VID>, dim3(grid), dim3(kUnitRows * kProfGroups(VID)),
+                    dyn_smem(VID) * kProfGroups(VID), s, args);
+}
+typedef cudaError_t (*PartLauncher)(const SpmvDev &, float *, SpmvState *, const ProfParams &, uint32_t, unsigned,
+                                    cudaStream_t);
+static const PartLauncher kPart[DYSEL_SPMV_NVARIANTS] = {launch_part<0>, launch_part<1>, launch_part<2>,
+                                                         launch_part<3>, launch_part<4>, launch_part<5>};
 static const ProfLauncher kProf[DYSEL_SPMV_NVARIANTS] = {launch_prof<0>, launch_prof<1>, launch_prof<2>, launch_prof<3>,
                                                          launch_prof<4>, launch_prof<5>};
 
@@ -916,10 +1018,13 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   // short-row eager range, +9.5% without eager work)
   p.no_eager = (pl->seq != nullptr && thread_per_row(pl->vids[pl->def])) ? 1u : 0u;
   p.abort = ((mode & DYSEL_NO_ABORT) || p.score_mode == 1) ? 0u : 1u;   // dominance needs busy or makespan
+  const bool grouped = kGroupedProfiling && !sequential;
   for (int i = 0; i < pl->K; ++i) {
     p.vids[i] = pl->vids[i];
-    // occupancy of the claim kernel that will run the remainder with this variant
+    // occupancy of the claim kernel that will run the remainder with this
+    // variant (the busy-time score normalises by it, A-6)
     p.occ[i] = (uint32_t)std::max(1, cs->occ_claim[pl->vids[i]]);
+    p.occ_t[i] = grouped ? std::min<uint32_t>(p.occ[i], (uint32_t)kProfGroups(pl->vids[i])) : p.occ[i];
   }
   if (p.hybrid) {   // Table 1: K - 1 slice-sized sandboxes, the default's slice is productive (A-4)
     const size_t bytes = (size_t)(pl->K - 1) * P.c * kUnitRows * sizeof(float);
@@ -944,6 +1049,25 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       kProf[pl->vids[i]](A, d_y, dst, p, (uint32_t)i, st);
       DYSEL_TRY(check_launch(ctx, "spmv_prof_kernel"));
     }
+  } else if (grouped) {   // grouped profiling (reading A-49): one combined launch + CSR-T's, PDL-chained
+    p.n_grp = 0;
+    for (int i = 0; i < pl->K; ++i)
+      if (pl->vids[i] != DYSEL_SPMV_CSR_TMA) p.grp_pv[p.n_grp++] = (uint32_t)i;
+    p.part_first = DYSEL_SPMV_NVARIANTS;   // the combined kernel waits for the init kernel
+    if (p.n_grp > 0) {
+      void *args[] = {&A, &d_y, &dst, &p};
+      DYSEL_CUDA_TRY(ctx, launch_pdl((const void *)spmv_prof_grp_all_kernel, dim3(p.n_grp * ((p.c + 3) / 4)),
+                                     dim3(kUnitRows * 4), 0, st, args));
+      DYSEL_TRY(check_launch(ctx, "spmv_prof_grp_all_kernel"));
+    }
+    for (int i = 0; i < pl->K; ++i) {
+      if (pl->vids[i] != DYSEL_SPMV_CSR_TMA) continue;
+      if (p.n_grp == 0) p.part_first = (uint32_t)i;
+      const int G = kProfGroups(pl->vids[i]);
+      const unsigned g = (unsigned)((p.c + G - 1) / G);
+      DYSEL_CUDA_TRY(ctx, kPart[pl->vids[i]](A, d_y, dst, p, (uint32_t)i, g, st));
+      DYSEL_TRY(check_launch(ctx, "spmv_prof_grp_kernel"));
+    }
   } else {   // all K profiling slices in one launch, PDL behind the init kernel
     void *args[] = {&A, &d_y, &dst, &p};
     DYSEL_CUDA_TRY(ctx, launch_pdl((const void *)spmv_prof_all_kernel, dim3(p.K * p.c), dim3(kUnitRows),
@@ -967,6 +1091,17 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
         spmv_switch_kernel<<<1, 32, 0, st>>>(A, d_y, dst, p);
       DYSEL_TRY(check_launch(ctx, "spmv_switch_kernel"));
     }
+    // a non-default CSR-T: its claim kernel in plain stream order behind the
+    // switch kernel (it enters the winner's phase at the published switch
+    // point, or exits when another variant won)
+    for (int i = 0; i < pl->K; ++i)
+      if (i != pl->def && pl->vids[i] == DYSEL_SPMV_CSR_TMA) {
+        const int v2 = pl->vids[i];
+        const uint64_t g2 =
+            std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[v2]) * ctx->n_sm, p.n_units - p.p_end);
+        DYSEL_TRY(kClaim[v2](A, d_y, dst, p, (uint32_t)i, (unsigned)g2, st, false));
+        DYSEL_TRY(check_launch(ctx, "spmv_claim_kernel (CSR-T, host-gated)"));
+      }
   }
   DYSEL_TRY(commit_pending_sel(ctx, pend, pl->sig, st));
   if (rep) {
@@ -993,7 +1128,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
                        : p.score_mode == 1 ? (t.units ? t.cycles / t.units : cap)
                        : p.score_mode == 2 ? rep->makespan_ns[id]
                                            : std::max<uint64_t>(h->busy[v] * p.n_units /
-                                                                    ((uint64_t)p.c * p.occ[v] * p.n_sm),
+                                                                    ((uint64_t)p.c * p.occ_t[v] * p.n_sm),
                                                                 h->max_busy[v]);
     }
     if (sel_pool < pl->K) ctx->sel_cache[pl->sig] = sel_pool;

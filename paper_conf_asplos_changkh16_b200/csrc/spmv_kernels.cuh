@@ -656,10 +656,11 @@ struct TmaStageBufs {
 };
 
 // dynamic shared memory (kernels that can run CSR-T are launched with
-// sizeof(TmaStageBufs) bytes of it, spmv.cu kDynSmem)
+// sizeof(TmaStageBufs) bytes of it per 256-thread unit group, spmv.cu dyn_smem):
+// group threadIdx.x / 256 uses the group-th set (grouped profiling, A-49)
 __device__ __forceinline__ TmaStageBufs &tma_stage_bufs() {
   extern __shared__ __align__(128) unsigned char spmv_dyn_smem[];
-  return *reinterpret_cast<TmaStageBufs *>(spmv_dyn_smem);
+  return *reinterpret_cast<TmaStageBufs *>(spmv_dyn_smem + (threadIdx.x / kUnitRows) * sizeof(TmaStageBufs));
 }
 
 __device__ __forceinline__ uint32_t spmv_smem_u32(const void *p) {
@@ -672,11 +673,12 @@ __device__ __forceinline__ uint32_t spmv_smem_u32(const void *p) {
 __device__ __forceinline__ void tma_stage_prologue() {
   uint32_t dyn;
   asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(dyn));
-  if (dyn < sizeof(TmaStageBufs)) return;
+  if (dyn < (threadIdx.x / kUnitRows + 1) * sizeof(TmaStageBufs)) return;   // (uniform per CTA in practice)
   TmaStageBufs &t = tma_stage_bufs();
-  if (threadIdx.x < kTmaWarps) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(spmv_smem_u32(&t.bar[threadIdx.x])) : "memory");
-    t.phase[threadIdx.x] = 0;
+  const uint32_t i = threadIdx.x % kUnitRows;
+  if (i < kTmaWarps) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(spmv_smem_u32(&t.bar[i])) : "memory");
+    t.phase[i] = 0;
   }
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
