@@ -46,6 +46,7 @@ struct SpmvState {
   uint64_t best_total;      // min over completed variants of the predicted time (busy score) or makespan (ns)
   uint32_t ctas_done[DYSEL_MAX_VARIANTS];
   uint32_t decided[DYSEL_MAX_VARIANTS];   // 0 running, 1 completed, 2 dominated (set once, by CAS)
+  uint64_t vscore[DYSEL_MAX_VARIANTS];    // packed final score of each completed variant (~0: dominated / none)
   uint64_t busy[DYSEL_MAX_VARIANTS];      // sum of unit busy times (ns)
   uint64_t lb[DYSEL_MAX_VARIANTS];        // lower bound of the final busy sum (ns)
   uint64_t aborted[DYSEL_MAX_VARIANTS];   // sandbox units stopped / skipped by dominance
@@ -101,6 +102,7 @@ __global__ void spmv_state_init_kernel(SpmvState *s, int def) {
   if (v < DYSEL_MAX_VARIANTS) {
     s->ctas_done[v] = 0;
     s->decided[v] = 0;
+    s->vscore[v] = ~0ull;
     s->busy[v] = 0;
     s->lb[v] = 0;
     s->aborted[v] = 0;
@@ -143,6 +145,7 @@ struct PubArgs {
   uint64_t *tl;         // report timeline, nullable
   uint32_t K;
   uint32_t E;           // eager (light) slots
+  uint32_t def;         // pool index of the initial version (switch margin, A-50)
 };
 constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
 
@@ -151,7 +154,15 @@ __device__ __forceinline__ void decided_publish(const PubArgs a) {
   const uint32_t vd = atomicAdd(&a.st->variants_done, 1u) + 1u;
   if (vd != a.K) return;
   __threadfence();
-  const unsigned long long fin = atomicAdd((unsigned long long *)&a.st->best, 0ull);
+  unsigned long long fin = atomicAdd((unsigned long long *)&a.st->best, 0ull);
+  // reading A-50 (switch margin): a challenger within 1/8 of the initial
+  // version's own completed score does not replace it — switching costs the
+  // winner's launch and the default's drain, and closer scores are within
+  // the profile's noise
+  if ((uint32_t)(fin & 0xffu) != a.def) {
+    const unsigned long long ds = ld_relaxed_u64(&a.st->vscore[a.def]);
+    if (ds != ~0ull && (fin >> 8) * 9ull > (ds >> 8) * 8ull) fin = ds;
+  }
   atomicExch((unsigned long long *)&a.st->sel, fin);
   const uint64_t old = atomicOr((unsigned long long *)&a.st->c1, 1ull << 32);   // close the eager range
   const uint64_t S = min(((uint64_t)(uint32_t)old + kSlots - 1) / kSlots * kSlots, (uint64_t)a.E);
@@ -332,7 +343,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
   // default ("first") variant writes y, the others their own sandbox
   const bool productive = !p.hybrid || pv == p.def;
   const bool sandbox = !productive;
-  const PubArgs pub{st, p.host_sel, p.tl, p.K, eager_slots(p)};
+  const PubArgs pub{st, p.host_sel, p.tl, p.K, eager_slots(p), p.def};
   if (tid == 0) {
     s_abort = 0;
     s_last = dysel_globaltimer();
@@ -416,6 +427,8 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
       unsigned long long score = p.score_mode == 1 ? cy / p.c : p.score_mode == 2 ? e - a : pred;
       if (score > cap) score = cap;
       atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
+      st->vscore[pv] = (score << 8) | pv;
+      __threadfence();
       atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
       decided_publish(pub);
     }
