@@ -7,6 +7,10 @@
   (reading A-6).
 * Winner: argmin; ties -> lowest variant id, which is what one atomicMin on
   (score << 8 | v) produces (readings A-7, A-8).
+* Switch margin (reading A-50, the SpMV / SpMTV device paths): the argmin
+  replaces the initial version d only if its score is below 8/9 of d's own
+  completed score (score[best] * 9 <= score[d] * 8); a dominated d (maximal
+  score) never blocks the switch.
 * Exhaustive oracle: "the single pure version that delivers the shortest
   runtime" (§4.1): T* = min_v T_v.
 * Known-cost model: a variant that spins c_v ns per unit has score ∝ c_v, so
@@ -34,6 +38,17 @@ def select(scores) -> int:
     """argmin with lowest-id tie-break (the packed-min semantics)."""
     best = min(pack(s, v) for v, s in enumerate(scores))
     return best & 0xFF
+
+
+def select_with_margin(scores, default: int) -> int:
+    """Reading A-50: argmin (packed-min semantics) unless the initial
+    version's completed score is within 1/9 of it, then the initial version."""
+    best = select(scores)
+    cap = (1 << 56) - 1
+    sd = min(int(scores[default]), cap)
+    if best != default and sd != cap and min(int(scores[best]), cap) * 9 > sd * 8:
+        return default
+    return best
 
 
 def exhaustive_best(times) -> int:

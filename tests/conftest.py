@@ -30,13 +30,9 @@ def gpu():
 
 
 def expected_selection(rep, ids, default_vid):
-    """The device selection rule on a report: the argmin of the live scores
-    (ties -> pool order), except that a challenger must predict more than
-    1/9 faster than the initial version's own completed score (switch margin,
-    DESIGN.md A-50)."""
-    cap = (1 << 56) - 1
-    live = [v for v in ids if rep["score"][v] != cap]
-    best = min(live, key=lambda v: (rep["score"][v], ids.index(v)))
-    if best != default_vid and default_vid in live and rep["score"][best] * 9 > rep["score"][default_vid] * 8:
-        return default_vid
-    return best
+    """The device selection rule on a report (oracle.selection.select_with_margin,
+    DESIGN.md A-50) over the pool's variant ids: argmin of the scores (ties ->
+    pool order) unless the initial version's completed score is within 1/9."""
+    from oracle import selection
+    scores = [rep["score"][v] for v in ids]
+    return ids[selection.select_with_margin(scores, ids.index(default_vid))]

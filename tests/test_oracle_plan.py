@@ -196,3 +196,14 @@ def test_unit_order_hand_example():
     # uniform rows: nothing heavy or long -> index order
     rp2 = np.arange(0, 2 * 6 * 256 + 1, 2)
     assert P.unit_order(rp2, 1) == (None, 6)
+
+
+def test_select_with_margin_hand_cases():
+    """A-50 on hand cases: 1/9 margin around the initial version's score."""
+    cap = (1 << 56) - 1
+    assert S.select_with_margin([100, 90, 95], 0) == 0      # 90 * 9 = 810 > 800: within the margin
+    assert S.select_with_margin([100, 88, 95], 0) == 1      # 88 * 9 = 792 <= 800: switch
+    assert S.select_with_margin([100, 89, 95], 0) == 0      # 89 * 9 = 801 > 800: keep (boundary)
+    assert S.select_with_margin([cap, 500, 400], 0) == 2    # a dominated default never blocks the switch
+    assert S.select_with_margin([300, 200, 100], 2) == 2    # the default is the argmin
+    assert S.select_with_margin([50, 50, 60], 1) == 1       # tie: the default stays (no switch to a tie)
