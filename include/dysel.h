@@ -507,11 +507,23 @@ dysel_status dysel_comm_init(dysel_ctx *ctx, const void *nccl_unique_id, int ran
 dysel_status dysel_partition_rows(const int32_t *h_row_ptr, int64_t n_rows, int world, int64_t *bounds);
 /* y (full length, every rank) = A x where this rank's plan holds rows
  * [bounds[rank], bounds[rank+1]) with a rebased row_ptr; x full length on
- * every rank.  Local DySel launch into d_y + bounds[rank], then an allgatherv of
- * y (grouped ncclBroadcast per root) in place. */
+ * every rank.  Local DySel launch into d_y + bounds[rank] and an in-place
+ * allgatherv of y (grouped ncclBroadcast, one root per shard) OVERLAPPED with
+ * it: every shard's rows go out in up to 8 chunks (dysel_allgather_chunk), a
+ * chunk's broadcasts start on an internal stream as soon as the SpMV kernels
+ * have counted all its 32-row slots final (device path; DYSEL_HOST_ORCH:
+ * plain allgatherv after the SpMV).  Completes in stream order on `stream`.
+ * A chunk never released within 2 s (a bug) fails the next call with
+ * DYSEL_ERR_CUDA instead of hanging. */
 dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local_plan, const int64_t *bounds,
                                 const float *d_x, float *d_y, float profile_fraction, uint32_t mode,
                                 void *stream, dysel_report *rep);
+/* Chunk k (0 <= k < 8) of a shard of `rows` rows in the overlapped allgather:
+ * rows [*row_begin, *row_end) relative to the shard (empty when k is past its
+ * last chunk).  Chunks are whole 256-row units, 2^s units each with the
+ * smallest s that needs at most 8 chunks; every rank derives every shard's
+ * chunks from bounds alone.  Host function. */
+dysel_status dysel_allgather_chunk(int64_t rows, int k, int64_t *row_begin, int64_t *row_end);
 /* 1-GPU loopback of dysel_spmv_sharded (SURVEY §8e "testing without 8
  * GPUs"): plans[g] (g < G) holds rows [bounds[g], bounds[g+1]) with a rebased
  * row_ptr (the layout each rank's local plan has); the G shards' DySel

@@ -9,7 +9,9 @@
 
 #include <algorithm>
 #include <cstring>
+#include <string>
 
+#include "dysel_device.cuh"
 #include "internal.h"
 
 using namespace dysel;
@@ -63,6 +65,49 @@ void dysel::comm_free(dysel_ctx *ctx) {
     if (nccl().ok) nccl().CommDestroy((ncclComm_t)ctx->nccl_comm);
     ctx->nccl_comm = nullptr;
   }
+  if (ctx && ctx->comm_st) {
+    cudaStreamDestroy(ctx->comm_st);
+    ctx->comm_st = nullptr;
+  }
+  if (ctx && ctx->chunk_ctr.ptr) {
+    cudaFree(ctx->chunk_ctr.ptr);
+    ctx->chunk_ctr = ScratchBuf{};
+  }
+  if (ctx && ctx->h_chunk_timeout) {
+    cudaFreeHost(ctx->h_chunk_timeout);
+    ctx->h_chunk_timeout = ctx->d_chunk_timeout = nullptr;
+  }
+}
+
+// Overlapped allgather (D4 at G = 8 is comm-bound): the shard's y
+// rows go out in kAgChunks chunks of 2^shift units, each as soon as the SpMV
+// kernels have counted all of its 32-row slots final (ProfParams::chunk_done),
+// so the NCCL broadcasts of early chunks overlap the remainder still running.
+// One waiter kernel per chunk on the comm stream (bounded spin: a missing
+// count — a bug — sets the timeout flag and lets the stream go on, it never
+// hangs the device).
+constexpr int kAgChunks = 8;
+__global__ void chunk_wait_kernel(const uint32_t *ctr, uint32_t target, uint32_t *timeout_flag, uint32_t k) {
+  const uint64_t t0 = dysel_globaltimer();
+  uint32_t ns = 64;
+  while (*(volatile const uint32_t *)ctr < target) {
+    if (dysel_globaltimer() - t0 > 2000000000ull) {   // 2 s: record chunk and count seen
+      if (timeout_flag)
+        *(volatile uint32_t *)timeout_flag = 0x80000000u | (k << 24) | min(*(volatile const uint32_t *)ctr, 0xffffffu);
+      break;
+    }
+    __nanosleep(ns);
+    ns = ns < 2048 ? 2 * ns : ns;
+  }
+  __threadfence();
+}
+
+// chunking of shard r: units_r = ceil(rows_r / 256), chunk = 2^shift units
+static uint32_t ag_shift(int64_t rows) {
+  const int64_t units = (rows + 255) / 256;
+  uint32_t sh = 0;
+  while (((units + (1ll << sh) - 1) >> sh) > kAgChunks) ++sh;
+  return sh;
 }
 
 extern "C" {
@@ -138,6 +183,16 @@ dysel_status dysel_comm_broadcast(dysel_ctx *ctx, float *d_buf, size_t n, int ro
   return DYSEL_OK;
 }
 
+dysel_status dysel_allgather_chunk(int64_t rows, int k, int64_t *row_begin, int64_t *row_end) {
+  if (rows < 0 || k < 0 || k >= kAgChunks || !row_begin || !row_end) return DYSEL_ERR_INVALID;
+  const uint32_t sh = ag_shift(rows);
+  const int64_t units = (rows + 255) / 256;
+  *row_begin = std::min<int64_t>(((int64_t)k << sh) * 256, rows);
+  *row_end = std::min<int64_t>(std::min<int64_t>((int64_t)(k + 1) << sh, units) * 256, rows);
+  if (*row_end < *row_begin) *row_end = *row_begin;
+  return DYSEL_OK;
+}
+
 dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local, const int64_t *bounds, const float *d_x,
                                 float *d_y, float f, uint32_t mode, void *stream, dysel_report *rep) {
   if (!ctx || !local || !bounds || !d_y) return DYSEL_ERR_INVALID;
@@ -154,8 +209,74 @@ dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local, const in
     set_error(ctx, "dysel_spmv_sharded: local plan rows != bounds slice");
     return DYSEL_ERR_INVALID;
   }
-  DYSEL_TRY(dysel_spmv(ctx, local, d_x, d_y + offs[ctx->rank], f, mode, stream, rep));
-  return allgatherv(ctx, d_y, offs, counts, (cudaStream_t)stream);
+  cudaStream_t st = (cudaStream_t)stream;
+  // the paper-faithful host path has no slot counters: plain allgather after it
+  if (!ctx->nccl_comm || (mode & DYSEL_HOST_ORCH) || counts[ctx->rank] == 0) {
+    DYSEL_TRY(dysel_spmv(ctx, local, d_x, d_y + offs[ctx->rank], f, mode, stream, rep));
+    return allgatherv(ctx, d_y, offs, counts, st);
+  }
+  if (!ctx->comm_st) {
+    DYSEL_CUDA_TRY(ctx, cudaStreamCreateWithFlags(&ctx->comm_st, cudaStreamNonBlocking));
+    cudaFuncAttributes fa;   // load the waiter now (lazy module loading), not while the SpMV runs
+    DYSEL_CUDA_TRY(ctx, cudaFuncGetAttributes(&fa, chunk_wait_kernel));
+  }
+  if (!ctx->h_chunk_timeout) {
+    if (cudaHostAlloc((void **)&ctx->h_chunk_timeout, sizeof(uint32_t), cudaHostAllocMapped) != cudaSuccess ||
+        cudaHostGetDevicePointer((void **)&ctx->d_chunk_timeout, ctx->h_chunk_timeout, 0) != cudaSuccess)
+      return DYSEL_ERR_NOMEM;
+    *ctx->h_chunk_timeout = 0u;
+  }
+  if (const uint32_t t = *(volatile uint32_t *)ctx->h_chunk_timeout) {   // a previous call's chunk wait timed out
+    *(volatile uint32_t *)ctx->h_chunk_timeout = 0u;
+    set_error(ctx, "dysel_spmv_sharded: chunk " + std::to_string((t >> 24) & 0x7f) + " of the overlapped allgather "
+                   "was never completed (timeout; " + std::to_string(t & 0xffffff) + " slots counted)");
+    return DYSEL_ERR_CUDA;
+  }
+  DYSEL_TRY(scratch(ctx, ctx->chunk_ctr, kAgChunks * sizeof(uint32_t)));
+  uint32_t *ctr = (uint32_t *)ctx->chunk_ctr.ptr;
+  DYSEL_CUDA_TRY(ctx, cudaMemsetAsync(ctr, 0, kAgChunks * sizeof(uint32_t), st));
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  DYSEL_CUDA_TRY(ctx, cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming));
+  DYSEL_CUDA_TRY(ctx, cudaEventCreateWithFlags(&ev1, cudaEventDisableTiming));
+  DYSEL_CUDA_TRY(ctx, cudaEventRecord(ev0, st));   // counters zeroed
+  DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->comm_st, ev0, 0));
+  // the SpMV first, then the comm stream's waiters: a spinning waiter must
+  // never be resident before a kernel it waits for is loaded (with lazy module
+  // loading, a kernel's first launch can wait for running kernels — measured:
+  // waiters enqueued first stalled the first profiled call until they timed out)
+  const uint32_t my_sh = ag_shift(counts[ctx->rank]);
+  const int64_t my_units = (counts[ctx->rank] + 255) / 256;
+  ctx->spmv_chunk_done = ctr;
+  ctx->spmv_chunk_shift = my_sh;
+  dysel_status status = dysel_spmv(ctx, local, d_x, d_y + offs[ctx->rank], f, mode, stream, rep);
+  ctx->spmv_chunk_done = nullptr;
+  ctx->spmv_chunk_shift = 0;
+  ncclComm_t comm = (ncclComm_t)ctx->nccl_comm;
+  for (int k = 0; k < kAgChunks && status == DYSEL_OK; ++k) {
+    const int64_t u0 = (int64_t)k << my_sh, u1 = std::min<int64_t>((int64_t)(k + 1) << my_sh, my_units);
+    if (u0 < u1) {
+      chunk_wait_kernel<<<1, 1, 0, ctx->comm_st>>>(ctr + k, (uint32_t)((u1 - u0) * 8), ctx->d_chunk_timeout,
+                                                   (uint32_t)k);
+      status = check_launch(ctx, "chunk_wait_kernel");
+      if (status != DYSEL_OK) break;
+    }
+    if (nccl().GroupStart() != ncclSuccess) status = DYSEL_ERR_NCCL;
+    for (int r = 0; r < R && status == DYSEL_OK; ++r) {   // chunk k of every shard (same layout on every rank)
+      int64_t a = 0, e = 0;
+      dysel_allgather_chunk(counts[r], k, &a, &e);
+      if (e > a && nccl().Broadcast(d_y + offs[r] + a, d_y + offs[r] + a, (size_t)(e - a), ncclFloat, r, comm,
+                                    ctx->comm_st) != ncclSuccess)
+        status = DYSEL_ERR_NCCL;
+    }
+    if (nccl().GroupEnd() != ncclSuccess && status == DYSEL_OK) status = DYSEL_ERR_NCCL;
+  }
+  // the call completes (stream order on `st`) with the allgather
+  cudaEventRecord(ev1, ctx->comm_st);
+  cudaStreamWaitEvent(st, ev1, 0);
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  if (status == DYSEL_ERR_NCCL) set_error(ctx, "dysel_spmv_sharded: NCCL broadcast failed");
+  return status;
 }
 
 dysel_status dysel_sgemm_shard_rows(int M, int world, int rank, int *m0, int *m1) {
@@ -231,3 +352,4 @@ dysel_status dysel_spmv_sharded_loopback(dysel_ctx *ctx, int G, dysel_spmv_plan 
 }
 
 }  // extern "C"
+

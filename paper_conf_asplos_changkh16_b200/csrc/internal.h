@@ -124,6 +124,14 @@ struct dysel_ctx {
   size_t l2_persist_window = 0;
   // multi-GPU
   void *nccl_comm = nullptr;
+  // overlapped allgather of the row-sharded SpMV (comm.cu): while set, the
+  // SpMV kernels count finished 32-row slots per chunk of 2^shift units
+  uint32_t *spmv_chunk_done = nullptr;
+  uint32_t spmv_chunk_shift = 0;
+  cudaStream_t comm_st = nullptr;            // the chunked allgather's stream
+  dysel::ScratchBuf chunk_ctr;               // per-chunk slot counters
+  uint32_t *h_chunk_timeout = nullptr;       // mapped pinned flag: a chunk wait timed out
+  uint32_t *d_chunk_timeout = nullptr;
   int rank = 0, world = 1;
 };
 

@@ -83,6 +83,10 @@ struct ProfParams {
   // units -- an unproven thread-per-row default is slow on exactly the rows
   // that dominate such a matrix, and its eager work only delays the selection
   uint32_t no_eager;
+  // overlapped allgather (comm.cu): count each finished 32-row slot in
+  // chunk_done[unit >> chunk_shift] (nullptr = off)
+  uint32_t *chunk_done;
+  uint32_t chunk_shift;
   uint32_t part_first;   // grouped profiling (A-49): pool index of the first launch (it waits for the init kernel)
   uint32_t n_grp;        // ... pool indices profiled by the combined grouped kernel
   uint32_t grp_pv[DYSEL_SPMV_NVARIANTS];
@@ -410,6 +414,10 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
     if (skipped || (s_abort && sandbox)) atomicAdd((unsigned long long *)&st->aborted[pv], 1ull);
     atomicAdd((unsigned long long *)&slot->units, 1ull);
     if (productive && p.unit_variant) p.unit_variant[j] = (uint8_t)VID;
+    if (productive && p.chunk_done) {   // the unit's 8 slots are final (the group barrier above)
+      __threadfence();
+      atomicAdd(&p.chunk_done[j >> p.chunk_shift], (uint32_t)kSlots);
+    }
     __threadfence();
     const uint32_t done = atomicAdd(&st->ctas_done[pv], 1u) + 1u;
     // ---- variant complete (and not already decided by dominance): score,
@@ -668,6 +676,13 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
       }
       run_slot<VID>(A, u, (int)w, y + (size_t)u * kUnitRows);
       if (lane == 0 && p.unit_variant && w == 0) p.unit_variant[u] = (uint8_t)VID;
+      if (p.chunk_done) {   // this slot's rows are final: release them to the chunked allgather
+        __syncwarp();
+        if (lane == 0) {
+          __threadfence();
+          atomicAdd(&p.chunk_done[u >> p.chunk_shift], 1u);
+        }
+      }
     }
     t = e;
   }
@@ -758,6 +773,14 @@ dysel_status spmv_ctx_init(dysel_ctx *ctx) {
       if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                k == (const void *)spmv_prof_grp_kernel<5> ? m * kProfGroups(5) : m) != cudaSuccess)
         return DYSEL_ERR_CUDA;
+  }
+  {   // load every kernel of the device path now (lazy module loading): a kernel's
+      // first launch must not have to wait for spinning kernels of this path
+    const void *pre[] = {(const void *)spmv_prof_grp_all_kernel, (const void *)spmv_switch_kernel,
+                         (const void *)spmv_state_init_kernel, (const void *)spmv_prof_all_kernel};
+    cudaFuncAttributes fa;
+    for (const void *k : pre)
+      if (cudaFuncGetAttributes(&fa, k) != cudaSuccess) return DYSEL_ERR_CUDA;
   }
   for (int v = 0; v < DYSEL_SPMV_NVARIANTS; ++v) {
     // largest L1 for the gathers; CSR-T holds its staging buffers in shared
@@ -852,6 +875,8 @@ static dysel_status launch_variant_full(dysel_ctx *ctx, dysel_spmv_plan *pl, int
   p.n_units = pl->n_units;
   p.pure = 1;
   p.k_claim = claim_batch(pl);
+  p.chunk_done = ctx->spmv_chunk_done;
+  p.chunk_shift = ctx->spmv_chunk_shift;
   set_order(p, pl);
   const uint64_t grid = std::min<uint64_t>((uint64_t)std::max(1, cs->occ_claim[vid]) * ctx->n_sm, pl->n_units);
   SpmvDev A = pl->dev;
@@ -1025,6 +1050,8 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   if (sequential) p.async = 0;   // a variant profiled alone: no eager work beside it
   p.def = (uint32_t)pl->def;
   p.k_claim = claim_batch(pl);
+  p.chunk_done = ctx->spmv_chunk_done;
+  p.chunk_shift = ctx->spmv_chunk_shift;
   set_order(p, pl);
   // reading A-45: an unproven thread-per-row default gets no eager range on a
   // matrix with long-row units (measured on D4, JDS default: +12.9% with a

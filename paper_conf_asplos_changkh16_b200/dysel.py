@@ -113,6 +113,7 @@ dysel_sgemm_variant = _sig("dysel_sgemm_variant", c_int, P, c_int, c_int, c_int,
 dysel_comm_unique_id = _sig("dysel_comm_unique_id", c_int, P)
 dysel_comm_init = _sig("dysel_comm_init", c_int, P, P, c_int, c_int)
 dysel_partition_rows = _sig("dysel_partition_rows", c_int, P, c_i64, c_int, P)
+dysel_allgather_chunk = _sig("dysel_allgather_chunk", c_int, c_i64, c_int, P, P)
 dysel_spmv_sharded = _sig("dysel_spmv_sharded", c_int, P, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
 dysel_stencil = _sig("dysel_stencil", c_int, P, c_int, c_int, c_int, c_float, c_float, P, P, c_float, c_u32, P,
                      ctypes.POINTER(Report))
@@ -545,6 +546,15 @@ def sgemm_shard_rows(M, world, rank):
     if st != OK:
         raise DyselError(st, "dysel_sgemm_shard_rows")
     return a.value, b.value
+
+
+def allgather_chunk(rows, k):
+    """Rows [begin, end) of chunk k of a shard in the overlapped allgather."""
+    a, e = c_i64(0), c_i64(0)
+    st = dysel_allgather_chunk(int(rows), int(k), ctypes.byref(a), ctypes.byref(e))
+    if st != OK:
+        raise DyselError(st, "dysel_allgather_chunk")
+    return a.value, e.value
 
 
 def partition_rows(row_ptr_host, world):

@@ -40,6 +40,35 @@ def test_spmv_sharded_one_rank(cctx):
     plan.destroy()
 
 
+@pytest.mark.parametrize("mode_name", ["auto_async", "auto_sync", "fully_async", "fully_sync", "no_profile", "host"])
+def test_spmv_sharded_overlapped_allgather_modes(cctx, mode_name):
+    """The chunked allgather overlapped with the SpMV (comm.cu): every mode
+    of the device path counts each 32-row slot exactly once, so every chunk's
+    waiter is released (no timeout) and y is right; the host path falls back
+    to the plain allgather after the SpMV.  Two calls in a row (the counters
+    and the timeout flag are reset per call), a multi-wave matrix with heavy
+    units (the remainder finishes chunks out of order)."""
+    import torch
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+    mode = {"auto_async": D.AUTO | D.ASYNC | D.FORCE_PROFILE, "auto_sync": D.AUTO | D.FORCE_PROFILE,
+            "fully_async": D.FULLY | D.ASYNC | D.FORCE_PROFILE, "fully_sync": D.FULLY | D.FORCE_PROFILE,
+            "no_profile": D.NO_PROFILE, "host": D.AUTO | D.HOST_ORCH | D.FORCE_PROFILE}[mode_name]
+    A = d4_powerlaw(n=400_000, lmax=8192)
+    bounds = D.partition_rows(A.row_ptr, 1)
+    rp, col, val = to_dev(A)
+    plan = cctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO)
+    x = uniform_f32(22, A.n_cols)
+    xd = vec(x)
+    for _ in range(2):
+        y = torch.full((A.n_rows,), float("nan"), device="cuda")
+        cctx.spmv_sharded(plan, list(bounds), xd, y, f=0.01, mode=mode)
+        torch.cuda.synchronize()
+        assert spmv_err(A, x, y) <= 1e-5, mode_name
+    cctx.spmv_sharded(plan, list(bounds), xd, y, f=0.01, mode=mode)   # raises if a chunk wait had timed out
+    torch.cuda.synchronize()
+    plan.destroy()
+
+
 def test_power_sharded_one_rank(cctx):
     import torch
     from paper_conf_asplos_changkh16_b200 import dysel as D
