@@ -222,7 +222,7 @@ struct ProfPoll {
   // true = stop this unit (sandbox of a dominated variant)
   __device__ __forceinline__ bool operator()() const {
     if (*s_abort) return !PRODUCTIVE;
-    return due() && report() && !PRODUCTIVE;
+    return due() && report(true) && !PRODUCTIVE;
   }
   // warp-cooperative loops: only lane 0 reads the timer (the caller combines
   // with __any_sync); checked every kWarpPollEvery-th step only
@@ -231,7 +231,7 @@ struct ProfPoll {
     if ((++tick & (kWarpPollEvery - 1)) != 0) return false;   // warp-uniform
     if (*s_abort) return !PRODUCTIVE;
     if ((threadIdx.x & 31) != 0) return false;
-    return due() && report() && !PRODUCTIVE;
+    return due() && report(false) && !PRODUCTIVE;
   }
   // Global values read by this thread's previous report, issued without
   // waiting (a blocking global atomic / load per report stalled the polling
@@ -240,13 +240,24 @@ struct ProfPoll {
   // best_total only shrinks (a stale best decides later, never wrongly).
   mutable unsigned long long lb_seen = 0, best_seen = ~0ull, t0_seen = ~0ull;
   mutable uint32_t dec_seen = 0;
-  __device__ __forceinline__ bool report() const {
+  // fresh: take lb from the atomic's return (thread-per-row variants: many
+  // threads of a unit poll, each rarely wins the report, so a per-thread
+  // stale lb_seen lagged the variant's bound by most of its reports — D4's
+  // JDS sandboxes were decided ~25 us late, delaying the selection)
+  __device__ __forceinline__ bool report(bool fresh) const {
     const unsigned long long now = dysel_globaltimer();
     const unsigned long long last = *(volatile unsigned long long *)s_last;
     if (now - last < kPollNs) return false;
     if (atomicCAS(s_last, last, now) != last) return *s_abort != 0;   // another thread reports
-    atomicAdd(lb, now - last);   // no return value: a fire-and-forget RED
-    const unsigned long long l = lb_seen + (now - last);
+    unsigned long long l;
+    if (fresh) {
+      l = atomicAdd(lb, now - last) + (now - last);
+      best_seen = ld_relaxed_u64(best_total);
+      dec_seen = ld_relaxed_u32(decided);
+    } else {
+      atomicAdd(lb, now - last);   // no return value: a fire-and-forget RED
+      l = lb_seen + (now - last);
+    }
     unsigned long long cost;
     if (makespan) {
       cost = t0_seen == ~0ull ? 0ull : now - t0_seen;
