@@ -23,7 +23,24 @@ for dflt in (D.SPMV_DEFAULT_AUTO, D.SPMV_CSR_VECTOR, D.SPMV_JDS):
         ctx.spmv(plan, xd, y, f=0.05, mode=mode | D.FORCE_PROFILE)
         errs[f"spmv d{dflt} m{mode}"] = ospmv.rel_error(y.cpu().numpy(), ys, den)
     plan.destroy()
+# every format (CSR-T's grouped profiling kernel, its host-ordered remainder)
+F = d3_fem(grid=300)
+xf = uniform_f32(5, F.n_cols)
+rpf, colf, valf = (torch.from_numpy(a).cuda() for a in (F.row_ptr, F.col, F.val))
+yfs, denf = ospmv.spmv(F.row_ptr, F.col, F.val, xf), ospmv.spmv_abs(F.row_ptr, F.col, F.val, xf)
+for dflt in (D.SPMV_ELL, D.SPMV_CSR_TMA):
+    pf = ctx.spmv_prepare(rpf, colf, valf, F.n_cols, default=dflt, formats=D.FMT_ALL)
+    for mode in (D.FULLY | D.ASYNC, D.FULLY):
+        y = torch.full((F.n_rows,), float("nan"), device="cuda")
+        ctx.spmv(pf, torch.from_numpy(xf).cuda(), y, f=0.05, mode=mode | D.FORCE_PROFILE)
+        errs[f"spmv fmt_all d{dflt} m{mode}"] = ospmv.rel_error(y.cpu().numpy(), yfs, denf)
+    pf.destroy()
+# row-sharded path on a one-rank communicator (overlapped chunked allgather)
+ctx.comm_init(0, 1, D.comm_unique_id())
 plan = ctx.spmv_prepare(rp, col, val, A.n_cols)
+y = torch.full((A.n_rows,), float("nan"), device="cuda")
+ctx.spmv_sharded(plan, [0, A.n_rows], xd, y, f=0.05, mode=D.AUTO | D.ASYNC | D.FORCE_PROFILE)
+errs["sharded"] = ospmv.rel_error(y.cpu().numpy(), ys, den)
 xt, y0 = uniform_f32(2, A.n_rows), uniform_f32(3, A.n_cols)
 yt = torch.from_numpy(y0.copy()).cuda()
 ctx.spmtv(plan, torch.from_numpy(xt).cuda(), yt, f=0.05, mode=D.AUTO | D.FORCE_PROFILE)
