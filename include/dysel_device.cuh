@@ -143,7 +143,15 @@ __device__ __forceinline__ void dysel_prof_begin(const dysel_slice &s, dysel_pro
  * thread (the one that ran dysel_prof_begin's thread-0 part, i.e. tid 0)
  * reports and checks; it returns the dominated flag but nothing stops the
  * CTA — it only lets the selection be published without waiting for it. */
-__device__ __forceinline__ bool dysel_prof_poll_thread(const dysel_slice &s, dysel_prof_smem &sm) {
+/* Progress form (reading A-51): the caller also passes how much of its CTA's
+ * work is done (done of total, uniform steps, e.g. K-slabs or z-planes).
+ * Besides the strict lower bound above, thread 0 extrapolates the CTA's
+ * final cycles (elapsed x total / done) to the variant's score; a projection
+ * above 5/4 of the best completed score decides the variant as well.  An
+ * estimate, not a bound: the 5/4 margin covers per-step variation (a GEMM
+ * tile's K-slabs, a stencil column's planes are uniform work). */
+__device__ __forceinline__ bool dysel_prof_poll_thread(const dysel_slice &s, dysel_prof_smem &sm, uint32_t done = 0u,
+                                                       uint32_t total = 0u) {
   if (s.timer == nullptr || s.lb == nullptr) return false;
   if (!sm.dominated) {
     const unsigned long long now = dysel_clock64();
@@ -157,7 +165,13 @@ __device__ __forceinline__ bool dysel_prof_poll_thread(const dysel_slice &s, dys
       /* a lower bound of the final score (tot <= final cycle sum, un >= final
        * units); makespan scores have no cycle bound */
       const bool cyc = s.score_cycles || (s.grid_ctas && s.wave_ctas && s.units_per_cta) || s.occupancy;
-      const unsigned long long lbs = cyc ? dysel_cycle_score(s, tot, un) : 0ull;
+      unsigned long long lbs = cyc ? dysel_cycle_score(s, tot, un) : 0ull;
+      if (cyc && best < cap && done > 0u && total > done && s.ctas_total > 0u) {
+        const unsigned long long el = now - sm.c0[0];
+        const unsigned long long proj = el / done * total * (unsigned long long)s.ctas_total;
+        const unsigned long long ps = dysel_cycle_score(s, proj, un);
+        if (ps > best + best / 4 && ps > lbs) lbs = ps;
+      }
       if (best < cap && lbs > best) {
         d = 1;
         if (atomicCAS(s.decided, 0u, 2u) == 0u) dysel_variant_decided(s);
@@ -168,10 +182,11 @@ __device__ __forceinline__ bool dysel_prof_poll_thread(const dysel_slice &s, dys
   return sm.dominated != 0;
 }
 
-__device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof_smem &sm) {
+__device__ __forceinline__ bool dysel_prof_poll(const dysel_slice &s, dysel_prof_smem &sm, uint32_t done = 0u,
+                                                uint32_t total = 0u) {
   if (s.timer == nullptr || s.lb == nullptr) return false;
   const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
-  if (tid == 0) dysel_prof_poll_thread(s, sm);
+  if (tid == 0) dysel_prof_poll_thread(s, sm, done, total);
   __syncthreads();
   return sm.dominated != 0;
 }

@@ -24,7 +24,8 @@ struct SgemmArgs {
 
 // BM x BN tile, TM x TN per thread, BK deep, 256 threads; register-staged
 // double buffering of the next K-slab.
-// poll(): called by all threads every 16 K-slabs; true => abandon the tile
+// poll(done, total): called by all threads every 4 K-slabs (progress for the
+// projected dominance test, A-51); true => abandon the tile
 // (a dominated sandbox copy, reading A-32: its output would be discarded).
 template <int BM, int BN, int BK, int TM, int TN, class Poll>
 __device__ __forceinline__ void simt_tile(const SgemmArgs &g, float *__restrict__ C, int m0, int n0,
@@ -92,7 +93,7 @@ __device__ __forceinline__ void simt_tile(const SgemmArgs &g, float *__restrict_
     }
     if (kt + 1 < nk) store(buf ^ 1);
     __syncthreads();
-    if ((kt & 15) == 15 && poll()) return;
+    if ((kt & 3) == 3 && poll(kt + 1, nk)) return;
   }
 #pragma unroll
   for (int i = 0; i < TM; ++i) {
@@ -122,7 +123,7 @@ __global__ void __launch_bounds__(256) sgemm_simt_kernel(SgemmArgs g, float *__r
     for (uint64_t cta = blockIdx.x; cta < n; cta += gridDim.x) {
       uint64_t u[3];
       if (dysel_cta_origin(s, wa, cta, u))
-        simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32, []() { return false; });
+        simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32, [](int, int) { return false; });
       __syncthreads();   // the tile's shared buffers are reused
     }
     return;
@@ -132,7 +133,10 @@ __global__ void __launch_bounds__(256) sgemm_simt_kernel(SgemmArgs g, float *__r
   const bool ok = dysel_cta_origin(s, wa, blockIdx.x, u);
   if (ok)
     simt_tile<BM, BN, BK, TM, TN>(g, C, (int)u[1] * 32, (int)u[0] * 32,
-                                  [&]() { return dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_SANDBOX; });
+                                  [&](int done, int total) {
+                                    return dysel_prof_poll(s, psm, (uint32_t)done, (uint32_t)total) &&
+                                           s.role == DYSEL_ROLE_SANDBOX;
+                                  });
   dysel_prof_end(s, psm, ok ? wa[0] * wa[1] : 0u);   // units (32x32 tiles) this CTA covered
 }
 

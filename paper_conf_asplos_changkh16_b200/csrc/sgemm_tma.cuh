@@ -168,7 +168,7 @@ __global__ void __launch_bounds__(192, 1)
       for (int kb = 0; kb < nk; ++kb) {
         // dominance report (A-32): a losing tiling is decided without waiting
         // for its profiled tiles (they still complete: no abort inside the pipeline)
-        if ((kb & 15) == 15) dysel_prof_poll_thread(s, psm);
+        if ((kb & 15) == 15) dysel_prof_poll_thread(s, psm, (uint32_t)(kb + 1), (uint32_t)nk);
         const int st = kb % S;
         if (kb >= S) mbar_wait(&empty_[st], (uint32_t)(((kb / S) - 1) & 1));
         mbar_expect_tx(&full[st], Cfg::TX);

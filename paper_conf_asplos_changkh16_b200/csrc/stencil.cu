@@ -100,7 +100,7 @@ __device__ __forceinline__ void zmarch_column(const StencilArgs &g, float *__res
   float zm = (col && z0 > 0) ? __ldg(pin - sz) : 0.0f;
   float c = col ? __ldg(pin) : 0.0f;
   for (int z = z0; z < z1; z += kZq) {
-    if (((z - z0) & 15) == 15 - (kZq - 1) && poll()) return;
+    if (((z - z0) & 15) == 15 - (kZq - 1) && poll(z - z0 + kZq, z1 - z0)) return;
     float up[kZq], ym[kZq], yp[kZq], xm[kZq], xp[kZq];
 #pragma unroll
     for (int q = 0; q < kZq; ++q) {
@@ -151,9 +151,12 @@ __global__ void __launch_bounds__(128, TIMED ? 1 : 16)
     const int z0 = (int)u[2], z1 = min(z0 + 64, g.nz);
     if constexpr (TIMED)
       zmarch_column(g, out, x, y, z0, z1,
-                    [&]() { return dysel_prof_poll(s, psm) && s.role == DYSEL_ROLE_SANDBOX; });
+                    [&](int done, int total) {
+                      return dysel_prof_poll(s, psm, (uint32_t)done, (uint32_t)total) &&
+                             s.role == DYSEL_ROLE_SANDBOX;
+                    });
     else
-      zmarch_column(g, out, x, y, z0, z1, []() { return false; });
+      zmarch_column(g, out, x, y, z0, z1, [](int, int) { return false; });
     units = (uint32_t)(z1 - z0);
   }
   }
@@ -320,7 +323,7 @@ __global__ void __launch_bounds__(kStThreads, 3)
       if (warp > 0)
 #pragma unroll 1
         for (int e = 0; e < 4; ++e)
-          zmarch_column(g, out, I.x0 + 4 * lane + e, I.y0 + warp - 1, I.zs, I.ze, []() { return false; });
+          zmarch_column(g, out, I.x0 + 4 * lane + e, I.y0 + warp - 1, I.zs, I.ze, [](int, int) { return false; });
       units += I.units;
     }
     if constexpr (TIMED) dysel_prof_end(s, psm, units);
