@@ -30,18 +30,46 @@ static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
   return fn;
 }
 
-// 2-D fp32 tensor map, 128-byte swizzle, zero fill out of bounds.
+// 2-D fp32 tensor map, 128-byte swizzle, zero fill out of bounds.  Encoded
+// maps are cached per thread (a few us of driver work per encode; a DySel
+// SGEMM launches up to K profiling copies, the eager wave and K gated
+// remainders, each with the same two maps).
+struct MapKey {
+  const float *base;
+  uint64_t inner, outer, ld;
+  uint32_t box_inner, box_outer;
+  int swz;
+  bool operator==(const MapKey &o) const {
+    return base == o.base && inner == o.inner && outer == o.outer && ld == o.ld && box_inner == o.box_inner &&
+           box_outer == o.box_outer && swz == o.swz;
+  }
+};
 static bool make_map(CUtensorMap *m, const float *base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
                      uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz) {
+  constexpr int kSlots = 8;
+  thread_local MapKey keys[kSlots] = {};
+  thread_local CUtensorMap maps[kSlots];
+  thread_local int next = 0;
+  const MapKey k{base, inner, outer, ld_elems, box_inner, box_outer, (int)swz};
+  for (int i = 0; i < kSlots; ++i)
+    if (keys[i].base && keys[i] == k) {
+      *m = maps[i];
+      return true;
+    }
   auto enc = tensor_map_encoder();
   if (!enc) return false;
   const cuuint64_t dims[2] = {inner, outer};
   const cuuint64_t strides[1] = {ld_elems * sizeof(float)};
   const cuuint32_t box[2] = {box_inner, box_outer};
   const cuuint32_t estr[2] = {1, 1};
-  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)base, dims, strides, box, estr,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+  if (enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)base, dims, strides, box, estr,
+          CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return false;
+  keys[next] = k;
+  maps[next] = *m;
+  next = (next + 1) % kSlots;
+  return true;
 }
 
 // tcgen05 path: TMA pipeline when the operands allow TMA (16-byte aligned
@@ -55,7 +83,7 @@ static dysel_status launch_tc(const SgemmArgs &g, float *C, const dysel_slice &s
     // A: K-major SW128 (16-byte granules); B: MN-major tf32 needs 32-byte atoms
     if (make_map(&ta, g.A, (uint64_t)g.K, (uint64_t)g.M, (uint64_t)g.lda, 32, 128, CU_TENSOR_MAP_SWIZZLE_128B) &&
         make_map(&tb, g.B, (uint64_t)g.N, (uint64_t)g.K, (uint64_t)g.ldb, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) {
-      sgemm_tma_kernel<BN><<<ctas, 192, TmaCfg<BN>::SMEM, st>>>(ta, tb, g, C, s);
+      sgemm_tma_kernel<BN><<<ctas, kTmaThreads, TmaCfg<BN>::SMEM, st>>>(ta, tb, g, C, s);
       return cudaGetLastError() == cudaSuccess ? DYSEL_OK : DYSEL_ERR_CUDA;
     }
   }
@@ -109,8 +137,8 @@ dysel_status sgemm_register(dysel_ctx *ctx) {
   int o[4] = {0, 0, 0, 0};
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[0], sgemm_simt_kernel<64, 64, 16, 4, 4>, 256, 0);
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[1], sgemm_simt_kernel<128, 128, 8, 8, 8>, 256, 0);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], sgemm_tma_kernel<64>, 192, TmaCfg<64>::SMEM);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[3], sgemm_tma_kernel<128>, 192, TmaCfg<128>::SMEM);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[2], sgemm_tma_kernel<64>, kTmaThreads, TmaCfg<64>::SMEM);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o[3], sgemm_tma_kernel<128>, kTmaThreads, TmaCfg<128>::SMEM);
   cudaGetLastError();
   const uint64_t n = (uint64_t)ctx->n_sm;
   g_simt_wave[0] = (uint64_t)o[0] * n;
