@@ -30,6 +30,8 @@
 
 namespace dysel {
 
+constexpr int kTmaThreads = 192;   // producer warp, MMA warp, 4 converter / epilogue warps
+
 template <int BN>
 struct TmaCfg {
   static constexpr int A_BYTES = 128 * 128;   // A staging: 128 rows x 32 fp32 (TMA lands here)
@@ -120,7 +122,7 @@ __device__ __forceinline__ void tc_mma_tf32_ts(uint32_t tmem_d, uint32_t tmem_a,
 }
 
 template <int BN>
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(kTmaThreads, 1)
     sgemm_tma_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, SgemmArgs g,
                      float *__restrict__ C, dysel_slice s) {
   using Cfg = TmaCfg<BN>;
