@@ -1,6 +1,8 @@
-"""Pipeline-stage ablation of the tcgen05 SGEMM (exp builds DYSEL_EXP_SG=1 no MMA,
-2 no conversion, 3 neither): per-call GPU time of pure-variant calls replayed
-from a CUDA graph (host launch cost excluded), and the host cost per call."""
+"""Per-call GPU time of pure SGEMM variant calls replayed from a CUDA graph
+(host launch cost excluded), and the host cost per call; DYSEL_LIB selects an
+A/B build.  Used for profiles/sgemm_pipeline_r2.txt (its stage ablation used
+temporary compile-time knobs, since removed).
+python scripts/exp_sgemm_pipe.py [MxKxN ...]  (env VARIANTS=2,3)"""
 import os, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
