@@ -647,6 +647,10 @@ def secondary_workloads(ctx, D, args, stream, pk):
     del At
     # SGEMM: D2s (Parboil small), D2m (Parboil medium), D7 8192^3 (extra, labelled)
     tf32_ceiling = pk["bf16_tflops"] * 0.5 / 3.0   # 3xTF32: three tf32 MMAs per fp32 product
+    # the tensor core's own issue bound, measured (scripts/mma_rate.cu, profiles/mma_rate_r2.txt):
+    # a kind::tf32 M128 MMA takes 64 cycles at N >= 128 = 4,092 flop/clk/SM -> 1,190 TF/s at
+    # 1.965 GHz on 148 SMs; 3xTF32 issues three per product -> 397 TF/s
+    tf32_issue = 4092.0 * 148 * 1.965e9 / 1e12 / 3.0
     for name, (M, K, N), f_sg, reps in (("d2s_sgemm_128x96x160", (128, 96, 160), 0.5, 50),
                                          ("d2m_sgemm", (1024, 992, 1056), 0.06, 30),
                                          ("d7_sgemm_8192", (8192, 8192, 8192), 0.005, 5)):
@@ -686,7 +690,13 @@ def secondary_workloads(ctx, D, args, stream, pk):
                      "roofline": {"bound": "tensor", "achieved": round(flops / tv[bestg] / 1e12, 2),
                                   "peak": round(tf32_ceiling, 1), "unit": "TFLOP/s",
                                   "frac": round(flops / tv[bestg] / 1e12 / tf32_ceiling, 4),
-                                  "peak_note": "3xTF32 ceiling = measured bf16 TF/s x 1/2 (nominal tf32 ratio) / 3"},
+                                  "peak_note": "3xTF32 ceiling = measured bf16 TF/s x 1/2 (nominal tf32 ratio) / 3",
+                                  "issue_bound": round(tf32_issue, 1),
+                                  "frac_of_issue_bound": round(flops / tv[bestg] / 1e12 / tf32_issue, 4),
+                                  "issue_note": "measured tcgen05 kind::tf32 issue rate (64 cycles per M128 x N128 "
+                                                "x K8 MMA, profiles/mma_rate_r2.txt) / 3: the tile stream is bound "
+                                                "by the SM's shared-memory + TMEM traffic per k-slab below it "
+                                                "(profiles/sgemm_pipeline_r2.txt)"},
                      "dysel_us": round(tdg * 1e6, 2), "profiled": repg["profiled"], "selected": repg["selected_name"],
                      "overhead_pct": round((tdg / tp - 1) * 100, 2),
                      "forced_single_shot_overhead_pct": round((tforced / tp - 1) * 100, 2),
