@@ -293,7 +293,12 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
     I.n_light = pl->seq ? (int32_t)pl->n_light : (int32_t)nu;
   }
   if (default_variant == DYSEL_SPMV_DEFAULT_AUTO) {   // reading A-30: initial version from row statistics
-    if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
+    // A-30b: a uniform matrix whose CSR arrays exceed L2 streams from HBM --
+    // CSR-T (bulk-staged col / val) when it is in the pool; an L2-resident one: ELL
+    const uint64_t csr_bytes = 8ull * (uint64_t)nnz + 4ull * (uint64_t)(n_rows + 1);
+    if (I.uniform && csr_bytes > ctx->l2_bytes && spmv_pool_index(pl, DYSEL_SPMV_CSR_TMA) >= 0)
+      default_variant = DYSEL_SPMV_CSR_TMA;
+    else if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
     else if (spmv_pool_index(pl, DYSEL_SPMV_CSR_STREAM) >= 0) default_variant = DYSEL_SPMV_CSR_STREAM;
     else default_variant = DYSEL_SPMV_CSR_VECTOR;
   }
