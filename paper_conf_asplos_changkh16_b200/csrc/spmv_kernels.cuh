@@ -125,16 +125,12 @@ __device__ __forceinline__ float4 ld_stream4(const float *p, uint64_t pol) {
   return v;
 }
 // x gather: L1-cached (banded matrices reuse it across neighbouring rows),
-// kept in L2.
+// kept in L2.  (D4 CSR-W, cold: 0.815 ms; with L1::no_allocate 0.811-0.813,
+// through L2 only (.cg) 0.813 -- within noise: the gathers are bound by the
+// L1TEX request rate either way.)
 __device__ __forceinline__ float ld_x(const float *p, uint64_t pol) {
   float v;
-#if defined(DYSEL_EXP_LDX) && DYSEL_EXP_LDX == 1
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
-#elif defined(DYSEL_EXP_LDX) && DYSEL_EXP_LDX == 2
-  asm volatile("ld.global.cg.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
-#else
   asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
-#endif
   return v;
 }
 
