@@ -475,3 +475,30 @@ def test_hybrid_unaligned_output_view(ctx, D):
         torch.cuda.synchronize()
         assert spmv_err(A, x, y) <= SPMV_TOL
     plan.destroy()
+
+
+def test_auto_initial_version_by_l2_residency(ctx, D):
+    """Reading A-30b: a uniform matrix whose CSR arrays exceed the L2 gets CSR-T
+    as its initial version (when in the pool); an L2-resident one ELL; a
+    non-uniform one CSR-W.  The result is exact either way."""
+    import torch
+    from workloads import d3_fem
+    l2 = torch.cuda.get_device_properties(0).L2_cache_size
+    big = d3_fem(grid=1500)                      # 56.2M nnz: 0.46 GB of CSR
+    assert 8 * big.nnz + 4 * (big.n_rows + 1) > l2
+    small = d3_fem(grid=383)                     # 30.9 MB of CSR
+    assert 8 * small.nnz + 4 * (small.n_rows + 1) < l2
+    for A, want in ((big, D.SPMV_CSR_TMA), (small, D.SPMV_ELL), (MATS["powerlaw"](), D.SPMV_CSR_STREAM)):
+        plan = prepared(ctx, A, default=D.SPMV_DEFAULT_AUTO)
+        assert plan.info.default_variant == want, (D.SPMV_NAMES[plan.info.default_variant], D.SPMV_NAMES[want])
+        plan.destroy()
+    plan = prepared(ctx, big, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ELL | D.FMT_STREAM)   # no CSR-T
+    assert plan.info.default_variant == D.SPMV_ELL
+    x = uniform_f32(15, big.n_cols)
+    y = torch.empty(big.n_rows, device="cuda")
+    plan2 = prepared(ctx, big, default=D.SPMV_DEFAULT_AUTO)
+    ctx.spmv(plan2, vec(x), y, f=0.02, mode=D.AUTO | D.ASYNC)
+    torch.cuda.synchronize()
+    assert spmv_err(big, x, y) <= SPMV_TOL
+    plan.destroy()
+    plan2.destroy()
