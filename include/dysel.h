@@ -241,11 +241,16 @@ typedef struct {
   uint8_t *unit_variant;    /* optional caller HOST array, one byte per granule: variant that
                                productively computed it (debug / c-6 tests; costs a D2H copy + sync) */
   uint64_t unit_variant_cap;
-  /* SpMV device path, filled only when a report is requested (diagnostics):
-   * ns since the first profiling CTA started — [0] 0, [1] selection
-   * published, [2] last profiling CTA ended, [3] first eager CTA started,
-   * [4] last eager CTA ended, [5] first remainder CTA started, [6] last
-   * remainder CTA ended, [7] longest profiling unit (ns); ~0 = did not happen. */
+  /* Filled only when a report is requested (diagnostics); ~0 = did not happen.
+   * SpMV device path: ns since the first profiling CTA started -- [0] 0, [1]
+   * selection published, [2] last profiling CTA ended, [3] first eager CTA
+   * started, [4] last eager CTA ended, [5] first remainder CTA started, [6]
+   * last remainder CTA ended, [7] longest profiling unit (ns).
+   * Generic launcher (dysel_launch, SGEMM, stencil, f-2 pools): ns since the
+   * call's init kernel -- [0] first profiling CTA started, [1] selection
+   * published (%globaltimer); event-timed: [2] selection known on the gate
+   * stream, [3] the default's gated remainder done, [4] every gated remainder
+   * done, [5] every profiling copy done, [6] the call done. */
   uint64_t timeline_ns[8];
   /* Table 1 allocation record of this launch: extra output
    * buffers the profiling slices wrote instead of the real output, and their

@@ -58,6 +58,7 @@ struct DevProf {
   uint64_t best;
   uint64_t sel;
   uint64_t t_publish;   // %globaltimer when the selection was published (written at sel + 1, dysel_device.cuh)
+  uint64_t t_init;      // %globaltimer of the call's init kernel (report timeline origin)
 };
 
 struct Registered {

@@ -204,6 +204,7 @@ __global__ void init_prof_kernel(DevProf *p, int K, int def) {
     p->best = (((1ull << 56) - 1) << 8) | (uint64_t)def;
     p->sel = ~0ull;
     p->t_publish = 0;
+    p->t_init = dysel_globaltimer();
   }
 }
 
@@ -974,16 +975,19 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     }
     rep->selected = selected;
     rep->eager_units = eager_units;
-    {   // timeline: [0] first profiling CTA, [1] selection published (device paths);
-        // event-timed from the call's first kernel: [2] selection known on the
-        // gate stream, [3] the default's remainder done, [4] every remainder
-        // done, [5] every profiling copy done, [6] the call done
+    {   // timeline, all from the call's init kernel: [0] first profiling CTA,
+        // [1] selection published (device paths) -- %globaltimer; event-timed
+        // (the event before the init kernel; same origin within ~1 us): [2]
+        // selection known on the gate stream, [3] the default's remainder
+        // done, [4] every remainder done, [5] every profiling copy done, [6]
+        // the call done
       uint64_t t0 = ~0ull;
       for (int v = 0; v < K; ++v) t0 = std::min<uint64_t>(t0, ctx->h_prof->slot[v].t_start_min);
+      const uint64_t ti = ctx->h_prof->t_init;
       for (int i = 0; i < 8; ++i) rep->timeline_ns[i] = ~0ull;
-      if (t0 != ~0ull) {
-        rep->timeline_ns[0] = 0;
-        if (!host_orch && ctx->h_prof->t_publish > t0) rep->timeline_ns[1] = ctx->h_prof->t_publish - t0;
+      if (t0 != ~0ull && t0 >= ti) {
+        rep->timeline_ns[0] = t0 - ti;
+        if (!host_orch && ctx->h_prof->t_publish > ti) rep->timeline_ns[1] = ctx->h_prof->t_publish - ti;
       }
       if (!host_orch) {
         cudaStreamSynchronize(st);
