@@ -138,6 +138,28 @@ def cpu_single_thread_sample(A, x, rows=1_000_000):
     return spmv_bytes(r1, A.n_cols, hi) / t / 1e9, f"first {r1} rows of D4 ({hi} nnz), 1 thread, fp64"
 
 
+def cpu_library_context(A, x, rows=1_000_000):
+    """Context only: scipy.sparse CSR SpMV (single-threaded
+    library routine) in fp64 and fp32 on the same first-`rows` sample."""
+    import scipy.sparse as sp
+    r1 = min(rows, A.n_rows)
+    hi = int(A.row_ptr[r1])
+    nb = spmv_bytes(r1, A.n_cols, hi)
+    out = {"sample": f"first {r1} rows of D4 ({hi} nnz), scipy.sparse csr_matrix @ x, "
+                     f"median of 3", "cores": 1}
+    for dt in (np.float64, np.float32):
+        M = sp.csr_matrix((A.val[:hi].astype(dt), A.col[:hi], A.row_ptr[:r1 + 1]), shape=(r1, A.n_cols))
+        xv = x.astype(dt)
+        M @ xv
+        ts = []
+        for _ in range(3):
+            t0 = time.perf_counter()
+            M @ xv
+            ts.append(time.perf_counter() - t0)
+        out[f"scipy_{np.dtype(dt).name}_gbs"] = round(nb / float(np.median(ts)) / 1e9, 3)
+    return out
+
+
 # ------------------------------------------------------------- workloads
 def make_d4(n):
     from workloads import d4_powerlaw, uniform_f32
@@ -442,7 +464,8 @@ def dysel_arm(args, world, rank, local_rank, A=None, x=None):
         cpu = {"value": round(nbytes_total / Tc / 1e9, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
                "sample": f"full D4 matrix ({A.nnz} nnz), fp64 CSR SpMV in plain C/OpenMP, median of "
                          f"{args.cpu_reps} passes",
-               "single_thread": {"value": round(g1, 3), "unit": "GB/s", "cores": 1, "sample": s1}}
+               "single_thread": {"value": round(g1, 3), "unit": "GB/s", "cores": 1, "sample": s1},
+               "library_context": cpu_library_context(A, x)}
     if rank == 0:
         h2d = int(x.nbytes) * world
         d2h = int(A.n_rows) * 4
