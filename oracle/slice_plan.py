@@ -43,6 +43,11 @@ V_NONUNIFORM = 2
 ROLE_PRODUCTIVE, ROLE_SANDBOX, ROLE_BATCH, ROLE_PRIVATE = 0, 1, 2, 3
 
 MIN_CTAS = 128
+# reading A-52 (SpMV device path, grouped profiling): a slice of fewer than
+# MIN_PROF_UNITS units per variant grows to MIN_PROF_UNITS when K x
+# MIN_PROF_UNITS x MIN_PROF_FRAC <= G_n (applied after A-2 and activation)
+MIN_PROF_UNITS = 12
+MIN_PROF_FRAC = 16
 
 
 class Unsupported(Exception):
@@ -94,12 +99,16 @@ def resolve_mode(mode, vflags):
     return base
 
 
-def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, wave_units=0) -> Plan:
+def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, wave_units=0,
+         min_c=0) -> Plan:
     """U: units per dim (3-tuple); wa: per-variant 3-tuples of units per CTA.
 
     wave_units (reading A-3b, SpMV device path): profiling is also off when
     the whole grid (G_n granules) fits in one wave of the default variant —
     everything runs concurrently, so no remainder can benefit.
+    min_c (reading A-52, SpMV device path with grouped profiling: pass
+    MIN_PROF_UNITS): an active slice smaller than min_c granules per variant
+    grows to min_c when K * min_c * MIN_PROF_FRAC <= G_n.
     """
     K = len(wa)
     vflags = vflags or [0] * K
@@ -134,6 +143,8 @@ def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, 
             active = c >= 1
         else:
             active = c >= 1 and default_ctas >= min_ctas and Gn > wave_units
+    if active and min_c and c < min_c and K * min_c * MIN_PROF_FRAC <= Gn:
+        c = min_c
     p = Plan(K, g, G, Gn, h, c if active else 0, active, rmode)
     if not active:
         p.remainder = list(range(Gn))

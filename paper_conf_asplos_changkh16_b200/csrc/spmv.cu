@@ -866,6 +866,8 @@ constexpr int64_t kClaimNnz = DYSEL_CLAIM_NNZ;
 #define DYSEL_GROUPED_PROFILING 1
 #endif
 constexpr bool kGroupedProfiling = DYSEL_GROUPED_PROFILING != 0;   // reading A-49
+constexpr uint64_t kMinProfUnits = 12;   // reading A-52: three full groups of 4 units
+constexpr uint64_t kMinProfFrac = 16;    // ... while K x 12 units stay within 1/16 of the matrix
 static uint32_t claim_batch(const dysel_spmv_plan *pl) {
   const int64_t slots = (int64_t)pl->n_units * kSlots;
   const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
@@ -1020,6 +1022,16 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       P.c = 0;
     }
   }
+  // reading A-52: grouped profiling (A-49) measures a variant at the per-SM
+  // load of the full run only when its slice fills several groups: with fewer
+  // than kMinProfUnits units per variant, CSR-S's LSU saturation hid again
+  // (regular FEM, default pool: CSR-S picked over ELL 10/10 at c = 1-4, 2/10
+  // at c = 6, 0-1/10 at c = 8, 0/10 at c >= 9; +39% when it happens).  The
+  // slice grows to kMinProfUnits when that keeps the profiled prefix within
+  // 1/kMinProfFrac of the units.
+  if (P.active && kGroupedProfiling && !(mode & DYSEL_SEQUENTIAL) && P.c < kMinProfUnits &&
+      (uint64_t)pl->K * kMinProfUnits * kMinProfFrac <= P.Gn)
+    P.c = kMinProfUnits;
   if (rep) {
     rep->mode_used = P.mode | (async ? DYSEL_ASYNC : 0);
     rep->profiled = P.active ? 1 : 0;

@@ -12,12 +12,12 @@ def cold(fn, reps=20):
         flush.fill_(1.0); a, b = torch.cuda.Event(True), torch.cuda.Event(True)
         a.record(s); fn(); b.record(s); torch.cuda.synchronize(); ts.append(a.elapsed_time(b))
     return float(np.median(ts[3:])) * 1e3
-for grid in (383, 1500):
+for grid in [int(g) for g in os.environ.get("GRIDS", "383,1500").split(",")]:
     A = d3_fem(grid=grid)
     x = torch.from_numpy(uniform_f32(385, A.n_cols)).cuda()
     rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
     y = torch.empty(A.n_rows, device="cuda")
-    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ALL)
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO, **({} if os.environ.get("DEFAULT_POOL") else {"formats": D.FMT_ALL}))
     res = {D.SPMV_NAMES[v]: cold(lambda: ctx.spmv_variant(plan, v, x, y)) for v in plan.variant_ids}
     best = min(res.values())
     for name, mode in (("auto_async", D.AUTO | D.ASYNC), ("auto_sync", D.AUTO), ("forced_async", D.AUTO | D.ASYNC | D.FORCE_PROFILE)):

@@ -100,3 +100,33 @@ def test_sgemm_sharded_one_rank(cctx):
     torch.cuda.synchronize()
     ref, den = osg.sgemm(A, B, C0, 1.5, -0.5), osg.sgemm_abs(A, B, C0, 1.5, -0.5)
     assert float((np.abs(C.cpu().numpy() - ref) / den).max()) <= osg.SGEMM_TOL
+
+
+@pytest.mark.parametrize("mode_name", ["auto_async", "auto_sync", "host_orch", "no_profile"])
+def test_spmv_host_chunked_copy_out(mode_name):
+    """dysel_spmv_host: pinned x in, y out in chunks released by the SpMV's slot
+    counters; h_y equals the device buffer bitwise once the stream is done and
+    matches the oracle (ragged row count: the last chunk is partial)."""
+    import torch
+    from oracle.spmv import SPMV_TOL
+    from paper_conf_asplos_changkh16_b200 import dysel as D
+    ctx = D.Context(0)
+    A = d4_powerlaw(n=300_001, lmax=4096)
+    x = uniform_f32(31, A.n_cols)
+    rp, col, val = (torch.from_numpy(a).cuda() for a in (A.row_ptr, A.col, A.val))
+    plan = ctx.spmv_prepare(rp, col, val, A.n_cols, default=D.SPMV_DEFAULT_AUTO)
+    mode = {"auto_async": D.AUTO | D.ASYNC, "auto_sync": D.AUTO, "host_orch": D.AUTO | D.HOST_ORCH,
+            "no_profile": D.NO_PROFILE}[mode_name] | (D.FORCE_PROFILE if mode_name != "no_profile" else 0)
+    hx = torch.from_numpy(x).pin_memory()
+    hy = torch.full((A.n_rows,), float("nan")).pin_memory()
+    dx = torch.empty(A.n_cols, device="cuda")
+    dy = torch.empty(A.n_rows, device="cuda")
+    for _ in range(3):
+        hy.fill_(float("nan"))
+        ctx.spmv_host(plan, hx, hy, dx, dy, f=0.01, mode=mode)
+        torch.cuda.synchronize()
+        assert torch.isfinite(hy).all()
+        assert torch.equal(hy, dy.cpu())
+        assert spmv_err(A, x, hy) <= SPMV_TOL
+    plan.destroy()
+    ctx.close()

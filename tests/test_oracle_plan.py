@@ -91,6 +91,25 @@ def test_sm_rounding_reading_a2():
     assert p.c == 2
 
 
+def test_min_profiling_slice_reading_a52():
+    # D3x default pool: G_n = 8789, K = 5, f = 0.002 -> c = 3 < 12, and
+    # 5 * 12 * 16 = 960 <= 8789 -> c = 12 (hand computed)
+    p = P.plan((8789,), [(1,)] * 5, 0.002, 148, 0, P.FULLY, min_c=P.MIN_PROF_UNITS)
+    assert p.active and p.c == 12
+    assert p.slices[0].granules == [5 * i for i in range(12)] and p.remainder[0] == 60
+    assert P.plan((8789,), [(1,)] * 5, 0.002, 148, 0, P.FULLY).c == 3        # without the rule
+    # D4 at f = 0.001: c = floor(39063 * 0.001 / 4) = 9 -> 12; f = 0.02 -> 195 (A-2: multiple of 37) unchanged
+    assert P.plan((39063,), [(1,)] * 4, 0.001, 148, 0, P.HYBRID, min_c=12).c == 12
+    assert P.plan((39063,), [(1,)] * 4, 0.02, 148, 0, P.HYBRID, min_c=12).c == 185
+    # small grid: K * 12 * 16 = 768 > 700 -> the slice stays as computed
+    assert P.plan((700,), [(1,)] * 4, 0.02, 148, 0, P.FULLY, min_c=12).c == 3
+    # boundary: G_n = 768 grows, 767 does not
+    assert P.plan((768,), [(1,)] * 4, 0.02, 148, 0, P.FULLY, min_c=12).c == 12
+    assert P.plan((767,), [(1,)] * 4, 0.02, 148, 0, P.FULLY, min_c=12).c == 3
+    # inactive plans are untouched
+    assert P.plan((8789,), [(1,)] * 5, 0.002, 148, 0, P.FULLY | P.NO_PROFILE, min_c=12).c == 0
+
+
 @pytest.mark.parametrize("mode", [P.FULLY, P.FULLY | P.CONTIGUOUS, P.HYBRID, P.SWAP])
 def test_cover_invariant_exhaustive(mode):
     for U in (1, 5, 17, 64):

@@ -174,8 +174,10 @@ def test_dysel_composition(ctx, D, name, m):
     uv = rep["unit_variant"]
     K = len(plan.variant_ids)
     # oracle plan: same c, same granule count
+    grouped = not (m.endswith("host") or "seq" in m)   # device path, grouped profiling (A-49, A-52)
     p = slice_plan.plan((plan.n_units,), [(1,)] * K, 0.1, ctx.n_sm, plan.variant_ids.index(0), mode,
-                        [0 if plan.info.uniform else slice_plan.V_NONUNIFORM] * K)
+                        [0 if plan.info.uniform else slice_plan.V_NONUNIFORM] * K,
+                        min_c=slice_plan.MIN_PROF_UNITS if grouped else 0)
     assert rep["c"] == p.c and rep["n_granules"] == p.Gn
     sel = rep["selected"]
     assert sel in plan.variant_ids
@@ -502,3 +504,27 @@ def test_auto_initial_version_by_l2_residency(ctx, D):
     assert spmv_err(big, x, y) <= SPMV_TOL
     plan.destroy()
     plan2.destroy()
+
+
+def test_min_profiling_slice_a52(ctx, D):
+    """Reading A-52: at a tiny f the device path grows each variant's slice to
+    12 units (oracle plan with min_c), the result stays exact, and on a
+    regular FEM matrix the selection is ELL (the pure best) instead of CSR-S."""
+    import torch
+    from workloads import d3_fem
+    A = d3_fem(grid=1500)
+    x = uniform_f32(5, A.n_cols)
+    plan = prepared(ctx, A, default=D.SPMV_DEFAULT_AUTO, formats=D.FMT_ELL | D.FMT_JDS | D.FMT_STREAM)
+    K = len(plan.variant_ids)
+    y = torch.empty(A.n_rows, device="cuda")
+    sels = []
+    for _ in range(5):
+        rep = ctx.spmv(plan, vec(x), y, f=0.001, mode=D.AUTO | D.ASYNC, report=True)
+        sels.append(rep["selected_name"])
+    p = slice_plan.plan((plan.n_units,), [(1,)] * K, 0.001, ctx.n_sm, plan.variant_ids.index(plan.info.default_variant),
+                        D.AUTO | D.ASYNC, [0] * K, wave_units=0, min_c=slice_plan.MIN_PROF_UNITS)
+    assert rep["c"] == p.c == slice_plan.MIN_PROF_UNITS
+    torch.cuda.synchronize()
+    assert spmv_err(A, x, y) <= SPMV_TOL
+    assert sels.count("ell") >= 4, sels
+    plan.destroy()
