@@ -393,6 +393,11 @@ def dysel_arm(args, world, rank, local_rank, A=None, x=None):
     if world > 1:
         dist.barrier()
     T_e2e_serial = time_b2b(e2e_step, args.steps, stream)
+    # the same through dysel_spmv_host (y copied out in chunks released by the
+    # SpMV's slot counters): no gain on D4 -- every chunk holds heavy units,
+    # which the winner runs first, so the chunks complete only at the end
+    T_e2e_chunked = (time_b2b(lambda: ctx.spmv_host(plan, xh, yh, xd, yl, f=f, mode=mode), args.steps, stream)
+                     if world == 1 else None)
     if world > 1:
         t = torch.tensor([T_e2e_serial], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -496,9 +501,13 @@ def dysel_arm(args, world, rank, local_rank, A=None, x=None):
                     "ms_per_step": round(T_e2e_serial * 1e3, 4),
                     "pipelined_value": (round(nbytes_total / T_e2e_pipe / 1e9, 3) if T_e2e_pipe else None),
                     "pipelined_ms_per_step": round(T_e2e_pipe * 1e3, 4) if T_e2e_pipe else None,
+                    "chunked_copy_out_value": (round(nbytes_total / T_e2e_chunked / 1e9, 3) if T_e2e_chunked
+                                               else None),
                     "note": "value: dependent steps (x H2D from pinned memory, the DySel SpMV, y D2H, in stream "
-                            "order each step); pipelined: independent requests, the copies of steps k+1 / k-1 "
-                            "overlap step k's SpMV on three streams (double buffers)"},
+                            "order each step); chunked_copy_out: the same through dysel_spmv_host (y D2H in up to "
+                            "8 chunks, each released by the SpMV's per-chunk slot counters); pipelined: "
+                            "independent requests, the copies of steps k+1 / k-1 overlap step k's SpMV on three "
+                            "streams (double buffers)"},
             "step": {"eager_units": rep["eager_units"], "tail_units": rep["tail_units"],
                      "aborted_sandbox_units": {D.SPMV_NAMES[v]: rep["aborted"][v] for v in plan.variant_ids},
                      "busy_us_per_unit": {D.SPMV_NAMES[v]: round(rep["busy_ns"][v] / max(1, rep["units"][v]) / 1e3, 2)

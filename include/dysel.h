@@ -363,6 +363,19 @@ void dysel_spmv_plan_destroy(dysel_spmv_plan *plan);
 dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *d_x, float *d_y,
                         float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
 
+/* dysel_spmv with HOST buffers (serving): h_x [n_cols] is copied to the
+ * caller's device staging d_x, the DySel SpMV writes d_y [n_rows], and y is
+ * copied back to h_y in up to 8 chunks of whole 256-row units
+ * (dysel_allgather_chunk layout), each on an internal stream as soon as the
+ * SpMV kernels have counted all of its 32-row slots final (a stream
+ * wait-value, no SM needed) -- the copy-out overlaps the rest of the SpMV
+ * (DYSEL_HOST_ORCH: one copy after it).  h_x / h_y: caller-owned host memory,
+ * pinned for asynchronous copies; d_x / d_y: caller-owned device memory.
+ * Stream-ordered on `stream`: h_y is complete when `stream` is; nothing
+ * blocks the host.  Errors as dysel_spmv. */
+dysel_status dysel_spmv_host(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *h_x, float *h_y, float *d_x,
+                             float *d_y, float profile_fraction, uint32_t mode, void *stream, dysel_report *rep);
+
 /* One full-grid run of pool variant `variant_id` (a DYSEL_SPMV_* id) with no
  * profiling: the "single pure version" the exhaustive oracle times
  * and what DYSEL_NO_PROFILE runs. */
@@ -520,8 +533,11 @@ dysel_status dysel_partition_rows(const int32_t *h_row_ptr, int64_t n_rows, int 
  * chunk's broadcasts start on an internal stream as soon as the SpMV kernels
  * have counted all its 32-row slots final (device path; DYSEL_HOST_ORCH:
  * plain allgatherv after the SpMV).  Completes in stream order on `stream`.
- * A chunk never released within 2 s (a bug) fails the next call with
- * DYSEL_ERR_CUDA instead of hanging. */
+ * The release is a stream wait-value on the chunk's counter (needs no SM;
+ * it has no timeout -- the counts are exact by construction); where stream
+ * memory operations are unavailable a one-thread waiter kernel releases it,
+ * and a chunk it never sees complete within 2 s (a bug) fails the next call
+ * with DYSEL_ERR_CUDA instead of hanging. */
 dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local_plan, const int64_t *bounds,
                                 const float *d_x, float *d_y, float profile_fraction, uint32_t mode,
                                 void *stream, dysel_report *rep);

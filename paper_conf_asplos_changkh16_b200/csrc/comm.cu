@@ -6,6 +6,8 @@
 // (grouped ncclBroadcast, one root per shard = allgatherv, in place).
 #include <dlfcn.h>
 #include <nccl.h>
+#include <cuda.h>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
 #include <cstring>
@@ -100,6 +102,34 @@ __global__ void chunk_wait_kernel(const uint32_t *ctr, uint32_t target, uint32_t
     ns = ns < 2048 ? 2 * ns : ns;
   }
   __threadfence();
+}
+
+// The chunk release itself: a stream memory operation (cuStreamWaitValue32,
+// GEQ) executed by the GPU's front end -- it needs no SM.  The waiter KERNEL
+// above was never scheduled before the SpMV had finished: the SpMV's claim
+// kernel keeps every SM full (its grid is one wave at full occupancy and the
+// shared-memory carveout is sized to it, leaving no room for even a one-thread
+// CTA), so the copies of round 2's first version started only after the last
+// slot (measured: first release 1,057 us into a 1,070 us call, 9M-row FEM).
+// The kernel remains the fallback when stream memory operations are
+// unavailable.
+static PFN_cuStreamWaitValue32_v11070 wait_value_fn() {
+  static PFN_cuStreamWaitValue32_v11070 fn = [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      p = nullptr;
+    cudaGetLastError();
+    return (PFN_cuStreamWaitValue32_v11070)p;
+  }();
+  return fn;
+}
+static dysel_status wait_chunk(dysel_ctx *ctx, const uint32_t *ctr, uint32_t target, uint32_t k, cudaStream_t st) {
+  if (auto fn = wait_value_fn())
+    if (fn((CUstream)st, (CUdeviceptr)ctr, target, CU_STREAM_WAIT_VALUE_GEQ) == CUDA_SUCCESS) return DYSEL_OK;
+  chunk_wait_kernel<<<1, 1, 0, st>>>(ctr, target, ctx->d_chunk_timeout, k);
+  return check_launch(ctx, "chunk_wait_kernel");
 }
 
 // chunking of shard r: units_r = ceil(rows_r / 256), chunk = 2^shift units
@@ -255,9 +285,7 @@ dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local, const in
   for (int k = 0; k < kAgChunks && status == DYSEL_OK; ++k) {
     const int64_t u0 = (int64_t)k << my_sh, u1 = std::min<int64_t>((int64_t)(k + 1) << my_sh, my_units);
     if (u0 < u1) {
-      chunk_wait_kernel<<<1, 1, 0, ctx->comm_st>>>(ctr + k, (uint32_t)((u1 - u0) * 8), ctx->d_chunk_timeout,
-                                                   (uint32_t)k);
-      status = check_launch(ctx, "chunk_wait_kernel");
+      status = wait_chunk(ctx, ctr + k, (uint32_t)((u1 - u0) * 8), (uint32_t)k, ctx->comm_st);
       if (status != DYSEL_OK) break;
     }
     if (nccl().GroupStart() != ncclSuccess) status = DYSEL_ERR_NCCL;
@@ -278,6 +306,106 @@ dysel_status dysel_spmv_sharded(dysel_ctx *ctx, dysel_spmv_plan *local, const in
   if (status == DYSEL_ERR_NCCL) set_error(ctx, "dysel_spmv_sharded: NCCL broadcast failed");
   return status;
 }
+
+// Host buffers in and out (serving): x host -> device, the DySel SpMV, and
+// y device -> host in up to kAgChunks chunks, each copied as soon as the SpMV
+// kernels have counted all of its 32-row slots final -- the per-chunk
+// counters and releases of the overlapped allgather, so the PCIe copy of y
+// overlaps the rest of the SpMV.
+dysel_status dysel_spmv_host(dysel_ctx *ctx, dysel_spmv_plan *plan, const float *h_x, float *h_y, float *d_x,
+                             float *d_y, float f, uint32_t mode, void *stream, dysel_report *rep) {
+  if (!ctx || !plan) return DYSEL_ERR_INVALID;
+  dysel_spmv_plan_info info;
+  DYSEL_TRY(dysel_spmv_plan_get_info(plan, &info));
+  if ((info.n_cols > 0 && (!h_x || !d_x)) || (info.n_rows > 0 && (!h_y || !d_y))) {
+    set_error(ctx, "dysel_spmv_host: invalid arguments");
+    return DYSEL_ERR_INVALID;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  if (info.n_cols > 0)
+    DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(d_x, h_x, (size_t)info.n_cols * sizeof(float), cudaMemcpyHostToDevice, st));
+  if (info.n_rows == 0) return DYSEL_OK;
+  const size_t ybytes = (size_t)info.n_rows * sizeof(float);
+  if (mode & DYSEL_HOST_ORCH) {   // the paper-faithful host path has no slot counters
+    DYSEL_TRY(dysel_spmv(ctx, plan, d_x, d_y, f, mode, stream, rep));
+    DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(h_y, d_y, ybytes, cudaMemcpyDeviceToHost, st));
+    return DYSEL_OK;
+  }
+  if (!ctx->comm_st) {
+    DYSEL_CUDA_TRY(ctx, cudaStreamCreateWithFlags(&ctx->comm_st, cudaStreamNonBlocking));
+    cudaFuncAttributes fa;   // load the fallback waiter now (lazy module loading), not while the SpMV runs
+    DYSEL_CUDA_TRY(ctx, cudaFuncGetAttributes(&fa, chunk_wait_kernel));
+  }
+  if (!ctx->h_chunk_timeout) {
+    if (cudaHostAlloc((void **)&ctx->h_chunk_timeout, sizeof(uint32_t), cudaHostAllocMapped) != cudaSuccess ||
+        cudaHostGetDevicePointer((void **)&ctx->d_chunk_timeout, ctx->h_chunk_timeout, 0) != cudaSuccess)
+      return DYSEL_ERR_NOMEM;
+    *ctx->h_chunk_timeout = 0u;
+  }
+  if (const uint32_t t = *(volatile uint32_t *)ctx->h_chunk_timeout) {
+    *(volatile uint32_t *)ctx->h_chunk_timeout = 0u;
+    set_error(ctx, "dysel_spmv_host: chunk " + std::to_string((t >> 24) & 0x7f) + " of y was never completed "
+                   "(timeout; " + std::to_string(t & 0xffffff) + " slots counted)");
+    return DYSEL_ERR_CUDA;
+  }
+  DYSEL_TRY(scratch(ctx, ctx->chunk_ctr, kAgChunks * sizeof(uint32_t)));
+  uint32_t *ctr = (uint32_t *)ctx->chunk_ctr.ptr;
+  DYSEL_CUDA_TRY(ctx, cudaMemsetAsync(ctr, 0, kAgChunks * sizeof(uint32_t), st));
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  DYSEL_CUDA_TRY(ctx, cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming));
+  DYSEL_CUDA_TRY(ctx, cudaEventCreateWithFlags(&ev1, cudaEventDisableTiming));
+  DYSEL_CUDA_TRY(ctx, cudaEventRecord(ev0, st));   // x copied in, counters zeroed
+#ifdef DYSEL_EXP_CHUNK_EV
+  {
+    extern cudaEvent_t g_chunk_ev[10];
+    if (!g_chunk_ev[0]) for (int i = 0; i < 10; ++i) cudaEventCreate(&g_chunk_ev[i]);
+    cudaEventRecord(g_chunk_ev[0], st);
+  }
+#endif
+  DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->comm_st, ev0, 0));
+  const uint32_t sh = ag_shift(info.n_rows);
+  const int64_t units = (info.n_rows + 255) / 256;
+  ctx->spmv_chunk_done = ctr;   // the SpMV first, then the releases (see dysel_spmv_sharded)
+  ctx->spmv_chunk_shift = sh;
+  dysel_status status = dysel_spmv(ctx, plan, d_x, d_y, f, mode, stream, rep);
+  ctx->spmv_chunk_done = nullptr;
+  ctx->spmv_chunk_shift = 0;
+  for (int k = 0; k < kAgChunks && status == DYSEL_OK; ++k) {
+    const int64_t u0 = (int64_t)k << sh, u1 = std::min<int64_t>((int64_t)(k + 1) << sh, units);
+    if (u0 >= u1) continue;
+    status = wait_chunk(ctx, ctr + k, (uint32_t)((u1 - u0) * 8), (uint32_t)k, ctx->comm_st);
+    int64_t a = 0, e = 0;
+    dysel_allgather_chunk(info.n_rows, k, &a, &e);
+    if (status == DYSEL_OK && e > a &&
+        cudaMemcpyAsync(h_y + a, d_y + a, (size_t)(e - a) * sizeof(float), cudaMemcpyDeviceToHost, ctx->comm_st) !=
+            cudaSuccess)
+      status = DYSEL_ERR_CUDA;
+#ifdef DYSEL_EXP_CHUNK_EV
+    {
+      extern cudaEvent_t g_chunk_ev[10];
+      if (!g_chunk_ev[0]) for (int i = 0; i < 10; ++i) cudaEventCreate(&g_chunk_ev[i]);
+      cudaEventRecord(g_chunk_ev[k + 1], ctx->comm_st);
+    }
+#endif
+  }
+  // the call completes (stream order on `st`) with the last chunk's copy
+  cudaEventRecord(ev1, ctx->comm_st);
+  cudaStreamWaitEvent(st, ev1, 0);
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  if (status == DYSEL_ERR_CUDA) set_error(ctx, "dysel_spmv_host: chunked copy-out failed");
+  return status;
+}
+
+#ifdef DYSEL_EXP_CHUNK_EV
+cudaEvent_t g_chunk_ev[10] = {};
+extern "C" dysel_status dysel_debug_chunk_ev(float *ms, void *st) {
+  cudaEventRecord(g_chunk_ev[9], (cudaStream_t)st);
+  cudaEventSynchronize(g_chunk_ev[9]);
+  for (int i = 1; i < 10; ++i) ms[i - 1] = -1.0f, cudaEventElapsedTime(&ms[i - 1], g_chunk_ev[0], g_chunk_ev[i]);
+  return DYSEL_OK;
+}
+#endif
 
 dysel_status dysel_sgemm_shard_rows(int M, int world, int rank, int *m0, int *m1) {
   if (M < 0 || world < 1 || rank < 0 || rank >= world || !m0 || !m1) return DYSEL_ERR_INVALID;

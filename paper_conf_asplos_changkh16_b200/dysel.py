@@ -104,6 +104,7 @@ dysel_spmv_plan_get_info = _sig("dysel_spmv_plan_get_info", c_int, P, ctypes.POI
 dysel_spmv_plan_destroy = _sig("dysel_spmv_plan_destroy", None, P)
 dysel_spmv_plan_copy_array = _sig("dysel_spmv_plan_copy_array", c_int, P, c_int, P, ctypes.POINTER(c_size))
 dysel_spmv = _sig("dysel_spmv", c_int, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
+dysel_spmv_host = _sig("dysel_spmv_host", c_int, P, P, P, P, P, P, c_float, c_u32, P, ctypes.POINTER(Report))
 dysel_spmv_variant = _sig("dysel_spmv_variant", c_int, P, P, c_int, P, P, P)
 dysel_spmv_gather_probe = _sig("dysel_spmv_gather_probe", c_int, P, P, c_int, P, P, P)
 dysel_sgemm = _sig("dysel_sgemm", c_int, P, c_int, c_int, c_int, c_float, P, c_int, P, c_int, c_float, P, c_int,
@@ -153,6 +154,15 @@ class DyselError(RuntimeError):
     def __init__(self, status, msg):
         super().__init__(f"{dysel_status_str(status).decode()}: {msg}")
         self.status = status
+
+
+def _hptr(t):
+    """Host pointer of a CPU tensor (pinned for asynchronous copies)."""
+    if not isinstance(t, torch.Tensor) or t.is_cuda:
+        raise ValueError("host tensor expected")
+    if not t.is_contiguous():
+        raise ValueError("contiguous host tensor expected")
+    return ctypes.c_void_p(t.data_ptr())
 
 
 def _ptr(t):
@@ -333,6 +343,16 @@ class Context:
         if rep is None:
             return None
         return report_dict(rep, SPMV_NAMES, bytes(uv) if uv is not None else None)
+
+    def spmv_host(self, plan, h_x, h_y, d_x, d_y, f=0.02, mode=DEFAULT_MODE, report=False, stream=None):
+        """dysel_spmv_host: pinned host x in, host y out (chunked copy-out overlapped with the SpMV);
+        d_x / d_y are the device staging buffers.  Stream-ordered: h_y is valid once `stream` is done."""
+        rep, keep, uv = (_make_report(0) if report else (None, None, None))
+        self._check(dysel_spmv_host(self.h, plan.handle, _hptr(h_x), _hptr(h_y), _ptr(d_x), _ptr(d_y), float(f),
+                                    int(mode), _stream(stream), ctypes.byref(rep) if rep is not None else None))
+        if rep is None:
+            return None
+        return report_dict(rep, SPMV_NAMES, None)
 
     def spmv_power(self, plan, x, y, n_iter, profile_every=0, f=0.02, mode=DEFAULT_MODE, norms=None, report=False,
                    stream=None):
