@@ -355,13 +355,6 @@ dysel_status dysel_spmv_host(dysel_ctx *ctx, dysel_spmv_plan *plan, const float 
   DYSEL_CUDA_TRY(ctx, cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming));
   DYSEL_CUDA_TRY(ctx, cudaEventCreateWithFlags(&ev1, cudaEventDisableTiming));
   DYSEL_CUDA_TRY(ctx, cudaEventRecord(ev0, st));   // x copied in, counters zeroed
-#ifdef DYSEL_EXP_CHUNK_EV
-  {
-    extern cudaEvent_t g_chunk_ev[10];
-    if (!g_chunk_ev[0]) for (int i = 0; i < 10; ++i) cudaEventCreate(&g_chunk_ev[i]);
-    cudaEventRecord(g_chunk_ev[0], st);
-  }
-#endif
   DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(ctx->comm_st, ev0, 0));
   const uint32_t sh = ag_shift(info.n_rows);
   const int64_t units = (info.n_rows + 255) / 256;
@@ -380,13 +373,6 @@ dysel_status dysel_spmv_host(dysel_ctx *ctx, dysel_spmv_plan *plan, const float 
         cudaMemcpyAsync(h_y + a, d_y + a, (size_t)(e - a) * sizeof(float), cudaMemcpyDeviceToHost, ctx->comm_st) !=
             cudaSuccess)
       status = DYSEL_ERR_CUDA;
-#ifdef DYSEL_EXP_CHUNK_EV
-    {
-      extern cudaEvent_t g_chunk_ev[10];
-      if (!g_chunk_ev[0]) for (int i = 0; i < 10; ++i) cudaEventCreate(&g_chunk_ev[i]);
-      cudaEventRecord(g_chunk_ev[k + 1], ctx->comm_st);
-    }
-#endif
   }
   // the call completes (stream order on `st`) with the last chunk's copy
   cudaEventRecord(ev1, ctx->comm_st);
@@ -397,15 +383,6 @@ dysel_status dysel_spmv_host(dysel_ctx *ctx, dysel_spmv_plan *plan, const float 
   return status;
 }
 
-#ifdef DYSEL_EXP_CHUNK_EV
-cudaEvent_t g_chunk_ev[10] = {};
-extern "C" dysel_status dysel_debug_chunk_ev(float *ms, void *st) {
-  cudaEventRecord(g_chunk_ev[9], (cudaStream_t)st);
-  cudaEventSynchronize(g_chunk_ev[9]);
-  for (int i = 1; i < 10; ++i) ms[i - 1] = -1.0f, cudaEventElapsedTime(&ms[i - 1], g_chunk_ev[0], g_chunk_ev[i]);
-  return DYSEL_OK;
-}
-#endif
 
 dysel_status dysel_sgemm_shard_rows(int M, int world, int rank, int *m0, int *m1) {
   if (M < 0 || world < 1 || rank < 0 || rank >= world || !m0 || !m1) return DYSEL_ERR_INVALID;
