@@ -66,6 +66,10 @@ struct Registered {
   std::vector<std::vector<int>> sandbox_args;
   std::vector<std::string> names;
   int def = 0;
+  // a built-in pool (SGEMM, stencil, SpMTV, f-2, the SpMV host path): its
+  // variants always report, so the gate may be a stream wait-value with no
+  // timeout (user pools keep the bounded wait kernel)
+  bool builtin = false;
 };
 
 // Selection words copied D2H asynchronously after device-path launches; the
@@ -165,4 +169,5 @@ dysel_status stencil_register(dysel_ctx *ctx);
 dysel_status spmtv_register(dysel_ctx *ctx);
 // comm.cu
 void comm_free(dysel_ctx *ctx);
+void mark_builtin(dysel_ctx *ctx, const char *sig);
 }  // namespace dysel

@@ -8,6 +8,8 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <chrono>
 #include <cmath>
 #include <cstring>
@@ -252,6 +254,30 @@ __global__ void wait_selection_kernel(uint64_t *sel, uint32_t *timeout_flag, int
     }
     __nanosleep(ns);
   }
+}
+
+void mark_builtin(dysel_ctx *ctx, const char *sig) {
+  auto it = ctx->reg.find(sig);
+  if (it != ctx->reg.end()) it->second.builtin = true;
+}
+
+// The selection gate as a stream memory operation: wait until the 64-bit
+// selection word is no longer all ones (CU_STREAM_WAIT_VALUE_NOR with value 0:
+// ~(*sel | 0) != 0).  Executed by the GPU front end -- unlike the one-thread
+// wait kernel it needs no SM, so it opens at the publish even when the
+// profiling copies and the eager wave fill every SM.
+static bool gate_wait_value(cudaStream_t st, const uint64_t *sel) {
+  static PFN_cuStreamWaitValue64_v11070 fn = [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue64", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      p = nullptr;
+    cudaGetLastError();
+    return (PFN_cuStreamWaitValue64_v11070)p;
+  }();
+  if (getenv("DYSEL_GATE_KERNEL")) return false;
+  return fn && fn((CUstream)st, (CUdeviceptr)sel, 0ull, CU_STREAM_WAIT_VALUE_NOR) == CUDA_SUCCESS;
 }
 
 __global__ void timer_calib_kernel(uint64_t samples, uint64_t spin_ns, uint64_t *out) {
@@ -810,9 +836,13 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
     // dominance, behind dominated variants finishing productive tiles
     cudaStream_t gate_st = ctx->wsel;
     DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_start, 0));
+    bool wv_gate = false;   // the gate is a stream wait-value on gate_st (built-in pools)
     if (dominance) {
-      wait_selection_kernel<<<1, 1, 0, gate_st>>>(&ctx->d_prof->sel, ctx->d_sel_timeout, def, P.mode == DYSEL_SWAP);
-      DYSEL_TRY(check_launch(ctx, "wait_selection_kernel"));
+      wv_gate = R.builtin && gate_wait_value(gate_st, &ctx->d_prof->sel);
+      if (!wv_gate) {
+        wait_selection_kernel<<<1, 1, 0, gate_st>>>(&ctx->d_prof->sel, ctx->d_sel_timeout, def, P.mode == DYSEL_SWAP);
+        DYSEL_TRY(check_launch(ctx, "wait_selection_kernel"));
+      }
     } else {
       for (int v = 0; v < K; ++v) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(gate_st, ctx->ev_join[v], 0));
     }
@@ -833,9 +863,15 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
       // the default's gated copy goes first and on a high-priority stream: when
       // it wins (the usual case with a good initial version), the block
       // scheduler dispatches its CTAs ahead of the exiting CTAs of the losers
+      // With the wait-value gate the default's copy is enqueued on the gate
+      // stream itself: it starts at the publish, without the ~10 us hop of an
+      // event to another stream (measured: the selection reached the other
+      // streams 11-14 us after the publish)
+      // (not in swap mode: there the remainder also waits for the copy-in on `st`)
+      cudaStream_t def_st = (wv_gate && P.mode != DYSEL_SWAP) ? gate_st : ctx->rem_hi;
       for (int k = 0; k < K; ++k) {
         const int v = k == 0 ? def : (k <= def ? k - 1 : k);
-        cudaStream_t rs = k == 0 ? ctx->rem_hi : ctx->rem[v];
+        cudaStream_t rs = k == 0 ? def_st : ctx->rem[v];
         dysel_slice s = base_slice(P);
         s.variant = v;
         s.role = DYSEL_ROLE_BATCH;
@@ -843,14 +879,14 @@ dysel_status dysel::launch_keyed(dysel_ctx *ctx, const char *sig, const char *ke
         s.granule_count = rem_end - rem_begin;
         s.gate = &ctx->d_prof->sel;
         s.gate_full_grid = k == 0 ? 1u : 0u;
-        DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(rs, ctx->ev_fork2, 0));
+        if (!(k == 0 && def_st == gate_st)) DYSEL_CUDA_TRY(ctx, cudaStreamWaitEvent(rs, ctx->ev_fork2, 0));
         DYSEL_TRY(R.v[v].fn(&s, base_args.data(), rs, R.v[v].user));
         DYSEL_TRY(check_launch(ctx, "variant gated batch"));
         DYSEL_CUDA_TRY(ctx, cudaEventRecord(ctx->ev_join2[v], rs));
 
       }
       if (rep) {   // each remainder stream's completion
-        cudaEventRecord(tev[2], ctx->rem_hi);
+        cudaEventRecord(tev[2], def_st);
         for (int v = 0; v < K; ++v) cudaStreamWaitEvent(ctx->query, ctx->ev_join2[v], 0);
         cudaEventRecord(tev[3], ctx->query);
       }

@@ -151,7 +151,9 @@ dysel_status sgemm_register(dysel_ctx *ctx) {
       {"tc3xtf32_128x128", sgemm_variant_fn<3>, {4, 4, 1}, sb, 1, 0, nullptr, (uint64_t)o[3] * n},
   };
   // initial ("default") version on B200: the tensor-core tiling (A-5)
-  return dysel_register_variants(ctx, kSgemmSig, v, DYSEL_SGEMM_NVARIANTS, DYSEL_SGEMM_T128x64);
+  DYSEL_TRY(dysel_register_variants(ctx, kSgemmSig, v, DYSEL_SGEMM_NVARIANTS, DYSEL_SGEMM_T128x64));
+  mark_builtin(ctx, kSgemmSig);
+  return DYSEL_OK;
 }
 
 static dysel_status check_args(dysel_ctx *ctx, int M, int N, int K, const float *A, int lda, const float *B, int ldb,

@@ -172,7 +172,9 @@ dysel_status spmtv_register(dysel_ctx *ctx) {
   // first at high priority, so the initial version should be the variant
   // that usually wins; warp per row (coalesced entry loads)
   const int def = DYSEL_SPMTV_SCATTER_WARP;
-  return dysel_register_variants(ctx, kSpmtvSig, v, DYSEL_SPMTV_NVARIANTS, def);
+  DYSEL_TRY(dysel_register_variants(ctx, kSpmtvSig, v, DYSEL_SPMTV_NVARIANTS, def));
+  mark_builtin(ctx, kSpmtvSig);
+  return DYSEL_OK;
 }
 
 // ---------------------------------------------------------------------------

@@ -824,7 +824,9 @@ dysel_status spmv_register_pool(dysel_ctx *ctx, dysel_spmv_plan *pl) {
   for (int i = 0; i < pl->K; ++i)
     vv[i] = dysel_variant{kVariantNames[pl->vids[i]], kVariantFns[pl->vids[i]], {1, 1, 1}, sb, 1,
                           pl->info.uniform ? 0u : (uint32_t)DYSEL_V_NONUNIFORM, pl};
-  return dysel_register_variants(ctx, pl->sig.c_str(), vv, pl->K, pl->def);
+  DYSEL_TRY(dysel_register_variants(ctx, pl->sig.c_str(), vv, pl->K, pl->def));
+  mark_builtin(ctx, pl->sig.c_str());
+  return DYSEL_OK;
 }
 
 template <int VID>

@@ -277,6 +277,7 @@ static dysel_status place_pool(dysel_ctx *ctx, dysel_spmv_plan *pl, cudaStream_t
                           (uint64_t)std::max(1, g_place_occ[i]) * ctx->n_sm};
   const std::string sig = pl->sig + "/placement";
   DYSEL_TRY(dysel_register_variants(ctx, sig.c_str(), vv, DYSEL_SPMV_PLACE_NVARIANTS, DYSEL_SPMV_PLACE_LDG));
+  mark_builtin(ctx, sig.c_str());
   pl->place_sig = sig;
   return DYSEL_OK;
 }
@@ -587,6 +588,7 @@ dysel_status dysel_spmv_jds_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_co
   dysel_status rs = dysel_register_variants(ctx, jp->sig.c_str(), vv, DYSEL_SPMV_JDS_NVARIANTS,
                                             DYSEL_SPMV_JDS_UNROLL_PREFETCH);
   if (rs != DYSEL_OK) return fail(rs);
+  mark_builtin(ctx, jp->sig.c_str());
   jp->prep_ns = now_ns() - t0;
   *out = jp;
   return DYSEL_OK;

@@ -561,7 +561,9 @@ dysel_status stencil_register(dysel_ctx *ctx) {
   // initial version (A-5): the TMA tile (the B200-first design:
   // planes streamed into shared memory, the fastest on grids larger than L2).
   // A grid whose items fit in one wave of it is not profiled (reading A-3b).
-  return dysel_register_variants(ctx, kStencilSig, v, DYSEL_STENCIL_NVARIANTS, DYSEL_STENCIL_TILED);
+  DYSEL_TRY(dysel_register_variants(ctx, kStencilSig, v, DYSEL_STENCIL_NVARIANTS, DYSEL_STENCIL_TILED));
+  mark_builtin(ctx, kStencilSig);
+  return DYSEL_OK;
 }
 
 static dysel_status stencil_check(dysel_ctx *ctx, int nx, int ny, int nz, const float *in, float *out) {
