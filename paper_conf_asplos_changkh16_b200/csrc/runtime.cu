@@ -276,7 +276,6 @@ static bool gate_wait_value(cudaStream_t st, const uint64_t *sel) {
     cudaGetLastError();
     return (PFN_cuStreamWaitValue64_v11070)p;
   }();
-  if (getenv("DYSEL_GATE_KERNEL")) return false;
   return fn && fn((CUstream)st, (CUdeviceptr)sel, 0ull, CU_STREAM_WAIT_VALUE_NOR) == CUDA_SUCCESS;
 }
 
