@@ -294,9 +294,15 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
   }
   if (default_variant == DYSEL_SPMV_DEFAULT_AUTO) {   // reading A-30: initial version from row statistics
     // A-30b: a uniform matrix whose CSR arrays exceed L2 streams from HBM --
-    // CSR-T (bulk-staged col / val) when it is in the pool; an L2-resident one: ELL
+    // CSR-T (bulk-staged col / val) when it is in the pool and its warp slots
+    // suit one bulk copy each: every slot fits the staging buffer (max row
+    // <= 32: 32 rows x 32 <= kTmaCap) and holds >= 256 entries (mean row >=
+    // 8); otherwise (or L2-resident) ELL.  Measured (scripts/sel_sweep.py):
+    // CSR-T is the best on the 25-entry FEM rows, 1.6x slower than ELL on
+    // 5-entry rows, 5-13x slower where slots overflow the buffer (50 / 500).
     const uint64_t csr_bytes = 8ull * (uint64_t)nnz + 4ull * (uint64_t)(n_rows + 1);
-    if (I.uniform && csr_bytes > ctx->l2_bytes && spmv_pool_index(pl, DYSEL_SPMV_CSR_TMA) >= 0)
+    if (I.uniform && csr_bytes > ctx->l2_bytes && W <= 32 && (int64_t)8 * n_rows <= nnz &&
+        spmv_pool_index(pl, DYSEL_SPMV_CSR_TMA) >= 0)
       default_variant = DYSEL_SPMV_CSR_TMA;
     else if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
     else if (spmv_pool_index(pl, DYSEL_SPMV_CSR_STREAM) >= 0) default_variant = DYSEL_SPMV_CSR_STREAM;

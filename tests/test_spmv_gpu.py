@@ -490,7 +490,13 @@ def test_auto_initial_version_by_l2_residency(ctx, D):
     assert 8 * big.nnz + 4 * (big.n_rows + 1) > l2
     small = d3_fem(grid=383)                     # 30.9 MB of CSR
     assert 8 * small.nnz + 4 * (small.n_rows + 1) < l2
-    for A, want in ((big, D.SPMV_CSR_TMA), (small, D.SPMV_ELL), (MATS["powerlaw"](), D.SPMV_CSR_STREAM)):
+    import numpy as np
+    from workloads import csr_from_lengths
+    long_rows = csr_from_lengths(np.full(1_000_000, 48, np.int64), 1_000_000, 21, 22)   # > L2, rows of 48 > 32
+    short_rows = csr_from_lengths(np.full(4_000_000, 5, np.int64), 4_000_000, 23, 24)   # > L2, rows of 5 < 8
+    assert 8 * long_rows.nnz > l2 and 8 * short_rows.nnz > l2
+    for A, want in ((big, D.SPMV_CSR_TMA), (small, D.SPMV_ELL), (MATS["powerlaw"](), D.SPMV_CSR_STREAM),
+                    (long_rows, D.SPMV_ELL), (short_rows, D.SPMV_ELL)):
         plan = prepared(ctx, A, default=D.SPMV_DEFAULT_AUTO)
         assert plan.info.default_variant == want, (D.SPMV_NAMES[plan.info.default_variant], D.SPMV_NAMES[want])
         plan.destroy()
