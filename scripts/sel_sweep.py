@@ -6,7 +6,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 from bench import time_b2b
 from paper_conf_asplos_changkh16_b200 import dysel as D
-from workloads import (csr_from_lengths, d3_fem, d4_powerlaw, d6_diag, d6_random, powerlaw_lengths,
+from workloads import (csr_from_lengths, d3_fem, d4_powerlaw, d6_diag, d6_random, laplacian_2d, powerlaw_lengths,
                        uniform_f32)
 ctx = D.Context(0); s = torch.cuda.current_stream()
 def fixed(n, L, seed):
@@ -16,7 +16,8 @@ def uni(n, lo, hi, seed):
 MATS_ALL = [("fem_2.25M", lambda: d3_fem(grid=1500)), ("powerlaw_2M", lambda: d4_powerlaw(n=2_000_000, lmax=4096)),
         ("d6_random", d6_random), ("d6_diag", d6_diag), ("rows5_4M", lambda: fixed(4_000_000, 5, 11)),
         ("rows50_1M", lambda: fixed(1_000_000, 50, 12)), ("rows500_200k", lambda: fixed(200_000, 500, 13)),
-        ("uni1-64_2M", lambda: uni(2_000_000, 1, 64, 14)), ("uni1-2000_200k", lambda: uni(200_000, 1, 2000, 15))]
+        ("uni1-64_2M", lambda: uni(2_000_000, 1, 64, 14)), ("uni1-2000_200k", lambda: uni(200_000, 1, 2000, 15)),
+            ("laplace5_4M", lambda: laplacian_2d(2000))]
 MATS = [m for m in MATS_ALL if not os.environ.get("ONLY") or m[0] in os.environ["ONLY"].split(",")]
 res = []
 for name, mk in MATS:
