@@ -293,7 +293,8 @@ enum { DYSEL_SPMV_CSR_SCALAR = 0, DYSEL_SPMV_CSR_VECTOR = 1, DYSEL_SPMV_ELL = 2,
        DYSEL_SPMV_CSR_STREAM = 4, DYSEL_SPMV_CSR_TMA = 5, DYSEL_SPMV_NVARIANTS = 6 };
 /* default_variant = DYSEL_SPMV_DEFAULT_AUTO: the library picks the initial
  * version from the prepare-time row statistics (reading A-30): uniform rows
- * (A-13) -> CSR-T when in the pool, the CSR arrays exceed the L2 size and
+ * (A-13) of fewer than 8 entries on average -> CSR-S (A-30c); other uniform
+ * rows -> CSR-T when in the pool, the CSR arrays exceed the L2 size and
  * rows hold 8..32 entries (A-30b: an HBM-streaming matrix whose 32-row warp
  * slots suit one bulk copy), else ELL when in the pool; otherwise
  * CSR-W when in the pool, else CSR-V.  The choice is visible in

@@ -300,9 +300,14 @@ dysel_status dysel_spmv_prepare(dysel_ctx *ctx, int64_t n_rows, int64_t n_cols, 
     // 8); otherwise (or L2-resident) ELL.  Measured (scripts/sel_sweep.py):
     // CSR-T is the best on the 25-entry FEM rows, 1.6x slower than ELL on
     // 5-entry rows, 5-13x slower where slots overflow the buffer (50 / 500).
+    // A-30c: uniform rows of fewer than 8 entries -> CSR-S (thread per row):
+    // 5-point Laplacian CSR-S 62 vs ELL 77 us, 2M diagonal 34 vs 43, random
+    // 5-entry rows within 6% of ELL (scripts/sel_sweep.py)
     const uint64_t csr_bytes = 8ull * (uint64_t)nnz + 4ull * (uint64_t)(n_rows + 1);
-    if (I.uniform && csr_bytes > ctx->l2_bytes && W <= 32 && (int64_t)8 * n_rows <= nnz &&
-        spmv_pool_index(pl, DYSEL_SPMV_CSR_TMA) >= 0)
+    if (I.uniform && (int64_t)8 * n_rows > nnz && spmv_pool_index(pl, DYSEL_SPMV_CSR_SCALAR) >= 0)
+      default_variant = DYSEL_SPMV_CSR_SCALAR;
+    else if (I.uniform && csr_bytes > ctx->l2_bytes && W <= 32 && (int64_t)8 * n_rows <= nnz &&
+             spmv_pool_index(pl, DYSEL_SPMV_CSR_TMA) >= 0)
       default_variant = DYSEL_SPMV_CSR_TMA;
     else if (I.uniform && spmv_pool_index(pl, DYSEL_SPMV_ELL) >= 0) default_variant = DYSEL_SPMV_ELL;
     else if (spmv_pool_index(pl, DYSEL_SPMV_CSR_STREAM) >= 0) default_variant = DYSEL_SPMV_CSR_STREAM;

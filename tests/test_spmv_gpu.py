@@ -480,8 +480,9 @@ def test_hybrid_unaligned_output_view(ctx, D):
 
 
 def test_auto_initial_version_by_l2_residency(ctx, D):
-    """Reading A-30b: a uniform matrix whose CSR arrays exceed the L2 gets CSR-T
-    as its initial version (when in the pool); an L2-resident one ELL; a
+    """Readings A-30b / A-30c: a uniform matrix whose CSR arrays exceed the L2
+    and whose rows hold 8..32 entries gets CSR-T as its initial version (when
+    in the pool); uniform rows of < 8 entries CSR-S; other uniform ones ELL; a
     non-uniform one CSR-W.  The result is exact either way."""
     import torch
     from workloads import d3_fem
@@ -496,7 +497,7 @@ def test_auto_initial_version_by_l2_residency(ctx, D):
     short_rows = csr_from_lengths(np.full(4_000_000, 5, np.int64), 4_000_000, 23, 24)   # > L2, rows of 5 < 8
     assert 8 * long_rows.nnz > l2 and 8 * short_rows.nnz > l2
     for A, want in ((big, D.SPMV_CSR_TMA), (small, D.SPMV_ELL), (MATS["powerlaw"](), D.SPMV_CSR_STREAM),
-                    (long_rows, D.SPMV_ELL), (short_rows, D.SPMV_ELL)):
+                    (long_rows, D.SPMV_ELL), (short_rows, D.SPMV_CSR_SCALAR)):
         plan = prepared(ctx, A, default=D.SPMV_DEFAULT_AUTO)
         assert plan.info.default_variant == want, (D.SPMV_NAMES[plan.info.default_variant], D.SPMV_NAMES[want])
         plan.destroy()
