@@ -72,6 +72,7 @@ struct ProfParams {
   uint8_t *unit_variant; // optional debug map (variant id per unit)
   uint32_t pure;         // pure full-grid run of one variant (self-resetting counters, no init kernel)
   uint32_t k_claim;      // claim kernels: max slots per claim (~kClaimNnz nonzeros of work)
+  uint32_t k_min;        // ... min slots per claim (~kClaimMinNnz of work: short-row matrices)
   // unit order (reading A-45): seq[0, n_light) = light units in index order,
   // seq[n_light, n_units) = the rest, nonzeros descending (A-40); nullptr =
   // identity (every unit light).  Profiling takes seq[0, p_end); the eager
@@ -589,7 +590,7 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
   // stuck on a long slot holds its prefetched one back).
   auto batch = [&](uint32_t rest) -> uint32_t {
     const uint32_t k = rest / (2u * n_warps);
-    return k < 1u ? 1u : (k > p.k_claim ? p.k_claim : k);
+    return k < p.k_min ? p.k_min : (k > p.k_claim ? p.k_claim : k);
   };
   // phase 0: pure run; 1: eager (default, ASYNC) from c1; 2: winner after the selection
   int phase = p.pure ? 0 : ((pv == p.def && p.async) ? 1 : 2);
@@ -633,7 +634,7 @@ __global__ void __launch_bounds__(kUnitRows, kClaimMinBlocks[VID])
         // per eager claim, which bounds a losing default's drain to ~2 slots.
         const uint32_t k = VID == DYSEL_SPMV_CSR_VECTOR ? 1u
                            : VID == DYSEL_SPMV_CSR_STREAM ? batch(Ee - min(e, Ee))
-                                                          : min(2u, batch(Ee - min(e, Ee)));
+                                                          : min(max(2u, p.k_min), batch(Ee - min(e, Ee)));
         const uint64_t r = claim(k);
         t = (uint32_t)r;
         uint32_t lim = Ee;
@@ -875,6 +876,17 @@ static uint32_t claim_batch(const dysel_spmv_plan *pl) {
   const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
   return (uint32_t)std::min<int64_t>(kSlots, std::max<int64_t>(1, kClaimNnz / per_slot));
 }
+// Smallest claim: ~kClaimMinNnz nonzeros of work.  The claim counter
+// serialises (~1 claim per ns); on short rows a 1-2 slot claim is ~0.1 us of
+// work, and the winner's phase after an eager phase claimed 2 slots at a time
+// (5-point Laplacian: 4,700 units after the publish took 45 us, 2.5x the
+// kernel's own rate).  Cheap slots make larger claims harmless for balance.
+constexpr int64_t kClaimMinNnz = 1024;
+static uint32_t claim_min(const dysel_spmv_plan *pl) {
+  const int64_t slots = (int64_t)pl->n_units * kSlots;
+  const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
+  return (uint32_t)std::min<int64_t>(claim_batch(pl), std::max<int64_t>(1, kClaimMinNnz / per_slot));
+}
 
 // Pure version of one variant over the whole grid: the variant's claim kernel
 // with every slot its own, in the winner's order (the same code, occupancy
@@ -890,6 +902,7 @@ static dysel_status launch_variant_full(dysel_ctx *ctx, dysel_spmv_plan *pl, int
   p.n_units = pl->n_units;
   p.pure = 1;
   p.k_claim = claim_batch(pl);
+  p.k_min = claim_min(pl);
   p.chunk_done = ctx->spmv_chunk_done;
   p.chunk_shift = ctx->spmv_chunk_shift;
   set_order(p, pl);
@@ -1075,6 +1088,7 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
   if (sequential) p.async = 0;   // a variant profiled alone: no eager work beside it
   p.def = (uint32_t)pl->def;
   p.k_claim = claim_batch(pl);
+  p.k_min = claim_min(pl);
   p.chunk_done = ctx->spmv_chunk_done;
   p.chunk_shift = ctx->spmv_chunk_shift;
   set_order(p, pl);
