@@ -871,10 +871,14 @@ constexpr int64_t kClaimNnz = DYSEL_CLAIM_NNZ;
 constexpr bool kGroupedProfiling = DYSEL_GROUPED_PROFILING != 0;   // reading A-49
 constexpr uint64_t kMinProfUnits = 12;   // reading A-52: three full groups of 4 units
 constexpr uint64_t kMinProfFrac = 16;    // ... while K x 12 units stay within 1/16 of the matrix
+#ifndef DYSEL_CLAIM_MAX_SLOTS
+#define DYSEL_CLAIM_MAX_SLOTS 8
+#endif
+constexpr int64_t kClaimMaxSlots = DYSEL_CLAIM_MAX_SLOTS;   // one unit (32 slots measured: 2M diagonal 26 -> 45 us)
 static uint32_t claim_batch(const dysel_spmv_plan *pl) {
   const int64_t slots = (int64_t)pl->n_units * kSlots;
   const int64_t per_slot = slots ? std::max<int64_t>(1, pl->info.nnz / slots) : 1;
-  return (uint32_t)std::min<int64_t>(kSlots, std::max<int64_t>(1, kClaimNnz / per_slot));
+  return (uint32_t)std::min<int64_t>(kClaimMaxSlots, std::max<int64_t>(1, kClaimNnz / per_slot));
 }
 // Smallest claim: ~kClaimMinNnz nonzeros of work.  The claim counter
 // serialises (~1 claim per ns); on short rows a 1-2 slot claim is ~0.1 us of
