@@ -48,6 +48,9 @@ MIN_CTAS = 128
 # MIN_PROF_UNITS x MIN_PROF_FRAC <= G_n (applied after A-2 and activation)
 MIN_PROF_UNITS = 12
 MIN_PROF_FRAC = 16
+# reading A-3c (SpMV device path): a matrix below MIN_PROF_BYTES of
+# algorithmic bytes is not profiled unless FORCE_PROFILE
+MIN_PROF_BYTES = 64 << 20
 
 
 class Unsupported(Exception):
@@ -100,7 +103,7 @@ def resolve_mode(mode, vflags):
 
 
 def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, wave_units=0,
-         min_c=0) -> Plan:
+         min_c=0, work_bytes=None) -> Plan:
     """U: units per dim (3-tuple); wa: per-variant 3-tuples of units per CTA.
 
     wave_units (reading A-3b, SpMV device path): profiling is also off when
@@ -109,6 +112,8 @@ def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, 
     min_c (reading A-52, SpMV device path with grouped profiling: pass
     MIN_PROF_UNITS): an active slice smaller than min_c granules per variant
     grows to min_c when K * min_c * MIN_PROF_FRAC <= G_n.
+    work_bytes (reading A-3c, SpMV device path): when given and below
+    MIN_PROF_BYTES, profiling is off unless FORCE_PROFILE.
     """
     K = len(wa)
     vflags = vflags or [0] * K
@@ -142,7 +147,8 @@ def plan(U, wa, f, n_sm, default_variant, mode, vflags=None, min_ctas=MIN_CTAS, 
                 c = 1 if (Gn >= K if rmode == FULLY else Gn >= 1) else 0
             active = c >= 1
         else:
-            active = c >= 1 and default_ctas >= min_ctas and Gn > wave_units
+            active = c >= 1 and default_ctas >= min_ctas and Gn > wave_units and (
+                work_bytes is None or work_bytes >= MIN_PROF_BYTES)
     if active and min_c and c < min_c and K * min_c * MIN_PROF_FRAC <= Gn:
         c = min_c
     p = Plan(K, g, G, Gn, h, c if active else 0, active, rmode)

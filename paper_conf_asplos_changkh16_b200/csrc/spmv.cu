@@ -870,6 +870,7 @@ constexpr int64_t kClaimNnz = DYSEL_CLAIM_NNZ;
 #endif
 constexpr bool kGroupedProfiling = DYSEL_GROUPED_PROFILING != 0;   // reading A-49
 constexpr uint64_t kMinProfUnits = 12;   // reading A-52: three full groups of 4 units
+constexpr uint64_t kMinProfBytes = 64ull << 20;   // reading A-3c: smaller matrices run unprofiled
 constexpr uint64_t kMinProfFrac = 16;    // ... while K x 12 units stay within 1/16 of the matrix
 #ifndef DYSEL_CLAIM_MAX_SLOTS
 #define DYSEL_CLAIM_MAX_SLOTS 8
@@ -1037,6 +1038,17 @@ dysel_status dysel_spmv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, f
       // entirely concurrently — there is no remainder for a selection to speed up
     const uint64_t wave = (uint64_t)std::max(1, cs->occ_slice[pl->vids[pl->def]]) * ctx->n_sm;
     if (P.active && !(mode & DYSEL_FORCE_PROFILE) && P.Gn <= wave) {
+      P.active = false;
+      P.c = 0;
+    }
+  }
+  {   // reading A-3c: a matrix of fewer than kMinProfBytes algorithmic bytes
+      // runs in a few tens of us -- within ~2x the measured profiling latency
+      // (~20-25 us to the publish on B200) -- so a single-shot profile cannot
+      // pay for itself; the initial version runs (FORCE_PROFILE overrides)
+    const uint64_t bytes = 8ull * (uint64_t)pl->info.nnz + 4ull * (uint64_t)(pl->dev.n_rows + 1) +
+                           4ull * (uint64_t)pl->dev.n_cols + 4ull * (uint64_t)pl->dev.n_rows;
+    if (P.active && !(mode & DYSEL_FORCE_PROFILE) && bytes < kMinProfBytes) {
       P.active = false;
       P.c = 0;
     }

@@ -91,6 +91,17 @@ def test_sm_rounding_reading_a2():
     assert p.c == 2
 
 
+def test_small_matrix_deactivation_reading_a3c():
+    # D6 diagonal: 2^21 rows, 1 nnz: 8*2^21 + 4*(2^21+1) + 4*2^21 + 4*2^21 = 41,943,044 B < 64 MiB
+    b = 8 * 2 ** 21 + 4 * (2 ** 21 + 1) + 4 * 2 ** 21 + 4 * 2 ** 21
+    assert b == 41943044
+    assert not P.plan((8192,), [(1,)] * 5, 0.02, 148, 0, P.FULLY, work_bytes=b).active
+    assert P.plan((8192,), [(1,)] * 5, 0.02, 148, 0, P.FULLY | P.FORCE_PROFILE, work_bytes=b).active
+    assert P.plan((8192,), [(1,)] * 5, 0.02, 148, 0, P.FULLY, work_bytes=64 << 20).active      # boundary: on
+    assert not P.plan((8192,), [(1,)] * 5, 0.02, 148, 0, P.FULLY, work_bytes=(64 << 20) - 1).active
+    assert P.plan((8192,), [(1,)] * 5, 0.02, 148, 0, P.FULLY).active                          # rule not applied
+
+
 def test_min_profiling_slice_reading_a52():
     # D3x default pool: G_n = 8789, K = 5, f = 0.002 -> c = 3 < 12, and
     # 5 * 12 * 16 = 960 <= 8789 -> c = 12 (hand computed)

@@ -535,3 +535,26 @@ def test_min_profiling_slice_a52(ctx, D):
     assert spmv_err(A, x, y) <= SPMV_TOL
     assert sels.count("ell") >= 4, sels
     plan.destroy()
+
+
+def test_small_matrix_unprofiled_a3c(ctx, D):
+    """Reading A-3c: below 64 MiB of algorithmic bytes a call is not profiled
+    (the initial version runs: CSR-S for the 1-entry diagonal, A-30c) unless
+    FORCE_PROFILE; the oracle plan with work_bytes agrees; results exact."""
+    import torch
+    from workloads import d6_diag
+    A = d6_diag()
+    x = uniform_f32(17, A.n_cols)
+    plan = prepared(ctx, A, default=D.SPMV_DEFAULT_AUTO)
+    assert plan.info.default_variant == D.SPMV_CSR_SCALAR
+    b = 8 * A.nnz + 4 * (A.n_rows + 1) + 4 * A.n_cols + 4 * A.n_rows
+    K = len(plan.variant_ids)
+    y = torch.empty(A.n_rows, device="cuda")
+    for mode, want in ((D.AUTO | D.ASYNC, False), (D.AUTO | D.ASYNC | D.FORCE_PROFILE, True)):
+        rep = ctx.spmv(plan, vec(x), y, f=0.02, mode=mode, report=True)
+        p = slice_plan.plan((plan.n_units,), [(1,)] * K, 0.02, ctx.n_sm, plan.variant_ids.index(D.SPMV_CSR_SCALAR),
+                            mode, [0] * K, work_bytes=b, min_c=slice_plan.MIN_PROF_UNITS)
+        assert rep["profiled"] == want == p.active, (rep["profiled"], want, p.active)
+        torch.cuda.synchronize()
+        assert spmv_err(A, x, y) <= SPMV_TOL
+    plan.destroy()
