@@ -642,7 +642,8 @@ def secondary_workloads(ctx, D, args, stream, pk):
             "amortized_overhead_pct": round((tam3 / ts3[b3] - 1) * 100, 2),
             "all_us": {k: round(v * 1e6, 2) for k, v in ts3.items()},
             "note": f"in + out {sb3 / 1e6:.0f} MB, b2b; fully|async f = 0.02 (profiled unless the default's grid "
-                    "fits one wave, A-3b); forced: profile once; amortised: forced once + 19 activation-flag calls"}
+                    "fits one wave, A-3b, or the sweep is under ~650 MB, A-3c: then the initial version runs); forced: "
+                    "profile once; amortised: forced once + 19 activation-flag calls"}
         del a3, o3
     # SpMTV (f-1): y += A^T x by atomic scatter -> swap-mode profiling
     At = d4_powerlaw(n=2_000_000, lmax=4096)

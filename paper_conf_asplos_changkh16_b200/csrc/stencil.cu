@@ -580,6 +580,8 @@ using namespace dysel;
 
 extern "C" {
 
+constexpr uint64_t kStencilMinProfBytes = 650ull * 1000 * 1000;   // 2 x 50 us x 6.5 TB/s (reading A-3c)
+
 dysel_status dysel_stencil(dysel_ctx *ctx, int nx, int ny, int nz, float c0, float c1, const float *d_in,
                            float *d_out, float f, uint32_t mode, void *stream, dysel_report *rep) {
   if (!ctx) return DYSEL_ERR_INVALID;
@@ -592,6 +594,12 @@ dysel_status dysel_stencil(dysel_ctx *ctx, int nx, int ny, int nz, float c0, flo
   const size_t sbytes[1] = {(size_t)nx * ny * nz * sizeof(float)};
   const std::string key = std::string(kStencilSig) + "#" + std::to_string(nx) + "x" + std::to_string(ny) + "x" +
                           std::to_string(nz);
+  // reading A-3c for the stencil pool: the selection is published ~45-50 us
+  // into a profiled call (each profiling CTA streams 4 items); a sweep whose
+  // in + out bytes take less than twice that at HBM speed (~650 MB) cannot
+  // recover it in one call -- run the cached / initial version (FORCE_PROFILE
+  // overrides; iterated sweeps amortise one profile with the activation flag)
+  if (!(mode & DYSEL_FORCE_PROFILE) && 2ull * sbytes[0] < kStencilMinProfBytes) mode |= DYSEL_NO_PROFILE;
   return launch_keyed(ctx, kStencilSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep);
 }
 
