@@ -475,7 +475,10 @@ __device__ __forceinline__ void unit_csr_stream_s(const SpmvDev &A, uint32_t j, 
 // (Measured alternative, A-41b: lanes owning 8 contiguous entries
 // with lane-local row sums and direct row writes issued 1.8x the instructions
 // and ran 12% slower on D4.)
-constexpr int kStreamVec = 2;   // 128-entry chunks in flight per warp (8 x gathers per lane)
+#ifndef DYSEL_STREAM_VEC
+#define DYSEL_STREAM_VEC 2
+#endif
+constexpr int kStreamVec = DYSEL_STREAM_VEC;   // 128-entry chunks in flight per warp (8 x gathers per lane; D4 cold: 2 -> 0.816 ms, 3 -> 0.844, 4 -> 0.872)
 template <class Poll>
 __device__ __forceinline__ void unit_csr_stream(const SpmvDev &A, uint32_t j, int w, float *__restrict__ out,
                                                 const Poll &poll) {
