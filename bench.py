@@ -656,6 +656,8 @@ def secondary_workloads(ctx, D, args, stream, pk):
     bt = min(tt, key=tt.get)
     tdt = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO), 20, stream)
     rept = ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO, report=True)
+    tdta = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO | D.ASYNC), 20, stream)
+    repta = ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO | D.ASYNC, report=True)
     tht = time_b2b(lambda: ctx.spmtv(plant, xt, yt, f=0.01, mode=D.SWAP | D.HOST_ORCH), 10, stream)
     def amortt():
         ctx.spmtv(plant, xt, yt, f=0.01, mode=D.AUTO)
@@ -669,13 +671,18 @@ def secondary_workloads(ctx, D, args, stream, pk):
                                 "selected": rept["selected_name"], "profiled": rept["profiled"],
                                 "mode_used": rept["mode_used"], "sandbox_buffers": rept["sandbox_buffers"],
                                 "overhead_pct": round((tdt / tt[bt] - 1) * 100, 2),
+                                "async_dysel_us": round(tdta * 1e6, 2),
+                                "async_overhead_pct": round((tdta / tt[bt] - 1) * 100, 2),
+                                "async_selected": repta["selected_name"], "async_eager_units": repta["eager_units"],
                                 "host_orch_overhead_pct": round((tht / tt[bt] - 1) * 100, 2),
                                 "amortized_overhead_pct": round((tat / tt[bt] - 1) * 100, 2),
                                 "selections_10": {n: sels_t.count(n) for n in sorted(set(sels_t))},
                                 "all_us": {k: round(v * 1e6, 2) for k, v in tt.items()},
                                 "note": "y += A^T x (red.global.add per nonzero): AUTO -> swap, device path (A-47: "
-                                        "zeroed private outputs, the winner's reduced into y), f = 0.01, sync only "
-                                        "(Table 1); host_orch = the paper's copy-based swap"}
+                                        "zeroed private outputs, the winner's reduced into y), f = 0.01, sync (Table 1); "
+                                        "async_*: AUTO|ASYNC, the default reduces light units into y until the "
+                                        "selection (A-47b: the additive swap's final output is y); host_orch = the "
+                                        "paper's copy-based swap"}
     plant.destroy()
     del At
     # SGEMM: D2s (Parboil small), D2m (Parboil medium), D7 8192^3 (extra, labelled)

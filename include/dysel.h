@@ -500,9 +500,15 @@ dysel_status dysel_stencil_variant(dysel_ctx *ctx, int variant_id, int nx, int n
  * global atomics, i.e. the paper's case for swap-based partial-productive
  * profiling (§2.2, §3.3, Table 1
  * P:L735-739).  All three built-in variants carry DYSEL_V_ATOMICS: AUTO resolves
- * to SWAP (each variant profiles the same slice into a private copy of y
- * initialised from y; the winner's copy is swapped in; the winner runs the
- * rest); SWAP|ASYNC returns DYSEL_ERR_UNSUPPORTED.  Unit = 256 rows of A.
+ * to SWAP.  With DYSEL_HOST_ORCH it is the paper's copy-back swap (each
+ * variant profiles the same slice into a private copy of y initialised from y;
+ * the winner's copy is swapped in; the winner runs the rest) and SWAP|ASYNC
+ * returns DYSEL_ERR_UNSUPPORTED (the final output space is not
+ * determined until profiling ends).  Without it (default) the swap is additive
+ * (DESIGN A-47): private outputs start at zero, the winner's is ADDED into y,
+ * so the final output space is y itself and ASYNC is accepted (A-47b): the
+ * default's kernel reduces light units straight into y until the selection
+ * (report.eager_units).  Unit = 256 rows of A.
  * Variants: 0 scatter-thread (thread per row), 1 scatter-warp (warp per row,
  * entries strided over lanes), 2 scatter-segment (warp per 32-row segment,
  * its nonzeros as one flat stream).  One fp32 red.global.add per nonzero, in no

@@ -6,7 +6,8 @@
 // Table 1): every variant profiles the SAME slice into a private
 // copy of y (initialised from y), the winner's copy is swapped in, and the
 // winner runs the rest.  Variants carry DYSEL_V_ATOMICS, so AUTO resolves to
-// swap and SWAP|ASYNC is rejected by the planner.
+// swap and SWAP|ASYNC is rejected by the planner -- except on the device path's
+// additive swap (readings A-47 / A-47b below), whose final output is y itself.
 //
 // Unit = 256 consecutive rows of A (= entries of x), as for dysel_spmv.
 //   V0 scatter-thread  thread per row, the row's entries in CSR order
@@ -199,10 +200,18 @@ dysel_status spmtv_register(dysel_ctx *ctx) {
 //      (nonzeros descending, A-40), then the other light units.
 // The result equals y0 + A^T x up to the (already free) order of the fp32
 // additions; Table 1's K private outputs are kept (report.sandbox_buffers).
-constexpr int kSwapAddChunk = 16384;   // floats of the winner's private output per add-in ticket
+constexpr int kSwapAddChunk = 16384;
+constexpr int kSwapMaxSm = 256;
+__device__ __forceinline__ uint32_t swap_smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r % kSwapMaxSm;
+}   // floats of the winner's private output per add-in ticket
 
 struct SwapState {
-  uint32_t rem_ctr;
+  uint32_t rem_ctr;      // tickets: add-in chunks, then heavy units
+  uint32_t light_ctr;    // the other light units (eager phase and remainder share it, A-47b)
+  uint32_t eager_units;  // light units done before the selection (ASYNC, A-47b)
   uint32_t variants_done;
   uint64_t best;
   uint64_t sel;
@@ -216,6 +225,7 @@ struct SwapState {
   dysel_timer_slot slot[DYSEL_SPMTV_NVARIANTS];
   uint64_t vscore[DYSEL_SPMTV_NVARIANTS];   // packed final score of each completed variant (~0: dominated / none)
   uint64_t tl[4];   // 0 first profiling CTA, 1 publish, 2 first remainder claim, 3 last remainder claim
+  uint32_t prof_on_sm[kSwapMaxSm];   // profiling CTAs resident per SM (the eager phase yields there, A-47b)
 };
 
 struct SwapParams {
@@ -229,6 +239,7 @@ struct SwapParams {
   uint32_t occ[DYSEL_SPMTV_NVARIANTS];
   uint32_t add_chunks;
   uint32_t abort;
+  uint32_t eager;   // ASYNC (A-47b): the default's kernel claims light units into y before the selection
   uint64_t *host_sel;
   uint64_t *tl;
 };
@@ -257,8 +268,14 @@ __device__ __forceinline__ void swap_decided(SwapState *st, const SwapParams &p)
   __threadfence();
 }
 
-__global__ void spmtv_swap_init_kernel(SwapState *st, int def) {
+// Resets the state and zeroes the K private outputs (additive swap) in one
+// grid: the profiling kernel's griddepcontrol.wait sees both complete.
+__global__ void spmtv_swap_init_kernel(SwapState *st, int def, float4 *priv, uint64_t n4) {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const float4 z = make_float4(0.0f, 0.0f, 0.0f, 0.0f);
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (uint64_t)gridDim.x * blockDim.x)
+    priv[i] = z;
+  if (blockIdx.x != 0) return;
   const int v = threadIdx.x;
   if (v < DYSEL_SPMTV_NVARIANTS) {
     st->ctas_done[v] = 0;
@@ -271,8 +288,11 @@ __global__ void spmtv_swap_init_kernel(SwapState *st, int def) {
     st->slot[v].cycles = 0;
   }
   if (v < 4) st->tl[v] = (v == 0 || v == 2) ? ~0ull : 0ull;
+  for (int i = v; i < kSwapMaxSm; i += blockDim.x) st->prof_on_sm[i] = 0;
   if (v == 0) {
     st->rem_ctr = 0;
+    st->light_ctr = 0;
+    st->eager_units = 0;
     st->variants_done = 0;
     st->best = (((1ull << 56) - 1) << 8) | (uint64_t)def;
     st->sel = ~0ull;
@@ -317,6 +337,12 @@ struct SwapStop {
 
 __global__ void __launch_bounds__(256, 1) spmtv_swap_prof_kernel(SwapParams p, SwapState *st) {
   asm volatile("griddepcontrol.wait;" ::: "memory");
+  const uint32_t sm = swap_smid();
+  if (threadIdx.x == 0) {   // before the remainder kernel may launch: its eager phase yields on this SM
+    atomicAdd(&st->prof_on_sm[sm], 1u);
+    __threadfence();
+  }
+  __syncthreads();
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   __shared__ unsigned long long s_last, s_start;
   __shared__ int s_abort, s_skip;
@@ -350,6 +376,7 @@ __global__ void __launch_bounds__(256, 1) spmtv_swap_prof_kernel(SwapParams p, S
     }
   }
   __syncthreads();
+  if (tid == 0) atomicSub(&st->prof_on_sm[sm], 1u);
   if (tid >= 32) return;
   unsigned long long t0 = tid < 8 ? t0s[tid] : ~0ull, t1 = tid < 8 ? t1s[tid] : 0ull;
   unsigned long long c0 = tid < 8 ? c0s[tid] : ~0ull, c1 = tid < 8 ? c1s[tid] : 0ull;
@@ -394,13 +421,35 @@ __device__ __forceinline__ void red_add_v4(float *q, float4 v) {
                : "memory");
 }
 
-// Persistent remainder of variant VID (pool index = VID): exits unless VID
-// won; tickets: add-in chunks, then heavy units, then the other light units.
+// Persistent remainder of variant VID (pool index = VID).  ASYNC (reading
+// A-47b): the default's kernel first claims light units eagerly, straight into
+// y, until the selection is published.  Then it exits unless VID won; tickets:
+// add-in chunks, then heavy units, then the light units nobody claimed yet.
 template <int VID>
 __global__ void __launch_bounds__(256) spmtv_swap_rem_kernel(SwapParams p, SwapState *st) {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   __shared__ uint32_t s_t;
   __shared__ int s_go;
+  const uint32_t L1 = max(p.c, p.n_light);
+  const uint32_t n_heavy = p.n_units - L1, n_lt = L1 - p.c;
+  if (p.eager && (uint32_t)VID == p.def) {
+    const volatile uint32_t *on_sm = &st->prof_on_sm[swap_smid()];
+    for (;;) {
+      if (threadIdx.x == 0) {
+        // yield while a profiling CTA shares this SM: its units are timed as
+        // in the synchronous flow (per-SM contention would bias the scores)
+        for (uint32_t ns = 64; *on_sm != 0u && swap_ld_relaxed(&st->sel) == ~0ull; ns = ns < 1024 ? 2 * ns : ns)
+          __nanosleep(ns);
+        s_t = swap_ld_relaxed(&st->sel) != ~0ull ? ~0u : atomicAdd(&st->light_ctr, 1u);
+      }
+      __syncthreads();
+      const uint32_t t = s_t;
+      __syncthreads();
+      if (t >= n_lt) break;   // selected (~0u) or no light unit left
+      spmtv_unit<VID>(p.a, p.y, swap_unit_at(p, p.c + t), NoStop());
+      if (threadIdx.x == 0) atomicAdd(&st->eager_units, 1u);
+    }
+  }
   if (threadIdx.x == 0) {
     uint64_t sel = swap_ld_relaxed(&st->sel);
     for (uint32_t ns = 32; sel == ~0ull; ns = ns < 1024 ? 2 * ns : ns) {
@@ -412,21 +461,24 @@ __global__ void __launch_bounds__(256) spmtv_swap_rem_kernel(SwapParams p, SwapS
   __syncthreads();
   if (!s_go) return;
   const float *pw = p.priv + (uint64_t)VID * p.stride;
-  const uint32_t L1 = max(p.c, p.n_light);
-  const uint32_t n_heavy = p.n_units - L1, n_lt = L1 - p.c;
-  const uint32_t total = p.add_chunks + n_heavy + n_lt;
+  const uint32_t n_first = p.add_chunks + n_heavy;
   const bool y_vec = ((uintptr_t)p.y & 15) == 0;
   bool first = true;
   for (;;) {
     if (threadIdx.x == 0) {
-      s_t = atomicAdd(&st->rem_ctr, 1u);
+      uint32_t t = atomicAdd(&st->rem_ctr, 1u);
+      if (t >= n_first) {   // light units: shared counter with the eager phase
+        const uint32_t l = atomicAdd(&st->light_ctr, 1u);
+        t = l < n_lt ? n_first + l : ~0u;
+      }
+      s_t = t;
       if (p.tl && first) atomicMin((unsigned long long *)&p.tl[2], (unsigned long long)dysel_globaltimer());
     }
     first = false;
     __syncthreads();
     const uint32_t t = s_t;
     __syncthreads();
-    if (t >= total) break;
+    if (t == ~0u) break;
     if (t < p.add_chunks) {   // y += the winner's private output (its profiled units' contributions)
       const int64_t i0 = (int64_t)t * kSwapAddChunk, i1 = min(i0 + (int64_t)kSwapAddChunk, (int64_t)p.n_cols);
       if (y_vec) {
@@ -516,13 +568,15 @@ static dysel_status spmtv_swap_device(dysel_ctx *ctx, dysel_spmv_plan *pl, const
   for (int i = 0; i < K; ++i) p.occ[i] = (uint32_t)std::max(1, g_swap_occ[i]);
   p.add_chunks = (uint32_t)((pl->dev.n_cols + kSwapAddChunk - 1) / kSwapAddChunk);
   p.abort = (mode & DYSEL_NO_ABORT) ? 0u : 1u;
+  p.eager = (mode & DYSEL_ASYNC) ? 1u : 0u;
   const size_t priv_bytes = (size_t)K * p.stride * sizeof(float);
   DYSEL_TRY(scratch(ctx, ctx->sandbox[0], priv_bytes));
   p.priv = (float *)ctx->sandbox[0].ptr;
   if (rep) p.tl = dst->tl;
   const int pend = reserve_pending_sel(ctx, &p.host_sel);
-  DYSEL_CUDA_TRY(ctx, cudaMemsetAsync(p.priv, 0, priv_bytes, st));   // private outputs start at 0 (additive swap)
-  spmtv_swap_init_kernel<<<1, 32, 0, st>>>(dst, def);
+  const uint64_t n4 = priv_bytes / sizeof(float4);   // private outputs start at 0 (additive swap)
+  const unsigned init_grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)ctx->n_sm * 4, (n4 + 255) / 256));
+  spmtv_swap_init_kernel<<<init_grid, 256, 0, st>>>(dst, def, (float4 *)p.priv, n4);
   DYSEL_TRY(check_launch(ctx, "spmtv_swap_init_kernel"));
   void *args[] = {&p, &dst};
   DYSEL_CUDA_TRY(ctx, swap_launch((const void *)spmtv_swap_prof_kernel, p.K * p.c, 256, st, args, true));
@@ -539,14 +593,14 @@ static dysel_status spmtv_swap_device(dysel_ctx *ctx, dysel_spmv_plan *pl, const
     DYSEL_CUDA_TRY(ctx, cudaMemcpyAsync(&h, dst, sizeof(h), cudaMemcpyDeviceToHost, st));
     DYSEL_CUDA_TRY(ctx, cudaStreamSynchronize(st));
     const uint64_t cap = (1ull << 56) - 1;
-    rep->mode_used = DYSEL_SWAP;
+    rep->mode_used = DYSEL_SWAP | (p.eager ? DYSEL_ASYNC : 0);
     rep->profiled = 1;
     rep->selected = (int)(h.sel & 0xff);
     rep->n_variants = K;
     rep->c = P.c;
     rep->n_granules = P.Gn;
-    rep->eager_units = 0;
-    rep->tail_units = p.n_units - p.c;
+    rep->eager_units = h.eager_units;
+    rep->tail_units = p.n_units - p.c - h.eager_units;
     rep->sandbox_buffers = (uint32_t)K;
     rep->sandbox_bytes = priv_bytes;
     for (int v = 0; v < DYSEL_MAX_VARIANTS; ++v)
@@ -611,12 +665,18 @@ dysel_status dysel_spmtv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, 
       wa[v][0] = wa[v][1] = wa[v][2] = 1;
       vflags[v] = it->second.v[v].flags;
     }
+    // reading A-47b: the additive swap fixes the final output space (y itself), so
+    // ASYNC is accepted here; the paper's copy-back swap (HOST_ORCH, the generic
+    // launcher) still rejects it (Table 1)
     Plan P;
-    DYSEL_TRY(make_plan(ctx, U, wa, DYSEL_SPMTV_NVARIANTS, f, ctx->n_sm, DYSEL_SPMTV_SCATTER_WARP, mode, vflags, &P));
-    // reading A-3b: a grid within one wave of the default is not profiled (the generic path runs it)
-    const bool one_wave = !(mode & DYSEL_FORCE_PROFILE) && P.Gn <= g_spmtv_wave[DYSEL_SPMTV_SCATTER_WARP];
-    if (P.active && P.mode == DYSEL_SWAP && !one_wave)
-      return spmtv_swap_device(ctx, pl, d_x, d_y, P, mode, (cudaStream_t)stream, rep, key);
+    DYSEL_TRY(make_plan(ctx, U, wa, DYSEL_SPMTV_NVARIANTS, f, ctx->n_sm, DYSEL_SPMTV_SCATTER_WARP,
+                        mode & ~(uint32_t)DYSEL_ASYNC, vflags, &P));
+    if (P.mode == DYSEL_SWAP) {
+      // reading A-3b: a grid within one wave of the default is not profiled (the generic path runs it)
+      const bool one_wave = !(mode & DYSEL_FORCE_PROFILE) && P.Gn <= g_spmtv_wave[DYSEL_SPMTV_SCATTER_WARP];
+      if (P.active && !one_wave) return spmtv_swap_device(ctx, pl, d_x, d_y, P, mode, (cudaStream_t)stream, rep, key);
+      mode &= ~(uint32_t)DYSEL_ASYNC;   // unprofiled: no eager phase to run
+    }
   }
   return launch_keyed(ctx, kSpmtvSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep);
 }

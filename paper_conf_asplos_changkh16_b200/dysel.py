@@ -368,7 +368,8 @@ class Context:
         self._check(dysel_spmv_variant(self.h, plan.handle, int(variant_id), _ptr(x), _ptr(y), _stream(stream)))
 
     def spmtv(self, plan, x, y, f=0.02, mode=AUTO, report=False, unit_map=False, stream=None):
-        """y += A^T x through the atomic scatter pool (dysel_spmtv; AUTO -> swap mode)."""
+        """y += A^T x through the atomic scatter pool (dysel_spmtv; AUTO -> swap mode; ASYNC only on
+        the additive device swap, not with HOST_ORCH: include/dysel.h, DESIGN A-47b)."""
         rep, keep, uv = (_make_report(plan.n_units if unit_map else 0) if report else (None, None, None))
         self._check(dysel_spmtv(self.h, plan.handle, _ptr(x), _ptr(y), float(f), int(mode), _stream(stream),
                                 ctypes.byref(rep) if rep is not None else None))

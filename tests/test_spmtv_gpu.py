@@ -63,7 +63,8 @@ def test_spmtv_variants_parity(ctx, D, name):
 
 
 @pytest.mark.parametrize("name", list(MATS))
-@pytest.mark.parametrize("m", ["auto", "swap_host", "fully", "no_profile", "auto_forced"])
+@pytest.mark.parametrize("m", ["auto", "swap_host", "fully", "no_profile", "auto_forced", "auto_async",
+                               "auto_async_forced"])
 def test_spmtv_modes_parity(ctx, D, name, m):
     """Every unit's contribution lands in y exactly once, whichever variant
     profiled or ran it; AUTO resolves to swap (DYSEL_V_ATOMICS)."""
@@ -73,16 +74,21 @@ def test_spmtv_modes_parity(ctx, D, name, m):
     y0 = uniform_f32(42, A.n_cols)
     plan, keep = _plan(ctx, A)
     mode = {"auto": D.AUTO, "swap_host": D.SWAP | D.HOST_ORCH, "fully": D.FULLY, "no_profile": D.AUTO | D.NO_PROFILE,
-            "auto_forced": D.AUTO | D.FORCE_PROFILE}[m]
+            "auto_forced": D.AUTO | D.FORCE_PROFILE, "auto_async": D.AUTO | D.ASYNC,
+            "auto_async_forced": D.AUTO | D.ASYNC | D.FORCE_PROFILE}[m]
     for rep_i in range(3):   # cached selection on later calls must not change the result
         y = vec(y0)
         rep = ctx.spmtv(plan, vec(x), y, f=0.05, mode=mode, report=True)
         torch.cuda.synchronize()
         assert _err(A, x, y0, y) <= SPMV_TOL, (m, rep_i)
         assert 0 <= rep["selected"] < len(D.SPMTV_NAMES)
-        if m in ("auto", "auto_forced", "swap_host") and rep["profiled"]:
+        if m != "fully" and rep["profiled"]:
             assert rep["mode_used"] & 3 == D.SWAP
-    if m == "auto_forced":
+            # reading A-47b: eager light units only on the additive (device) swap with ASYNC
+            assert bool(rep["mode_used"] & D.ASYNC) == m.startswith("auto_async")
+            if not m.startswith("auto_async"):
+                assert rep["eager_units"] == 0
+    if m in ("auto_forced", "auto_async_forced"):
         assert rep["profiled"]
     if name == "powerlaw" and m == "auto":
         assert rep["profiled"]
@@ -98,7 +104,8 @@ def test_spmtv_small_integer_bit_exact(ctx, D):
     ys = spmtv(A.row_ptr, A.col, A.val, x, y0)
     assert np.max(np.abs(ys)) < 2 ** 24
     plan, keep = _plan(ctx, A)
-    for mode in (D.AUTO | D.FORCE_PROFILE, D.SWAP | D.HOST_ORCH, D.FULLY | D.FORCE_PROFILE):
+    for mode in (D.AUTO | D.FORCE_PROFILE, D.AUTO | D.ASYNC | D.FORCE_PROFILE, D.SWAP | D.HOST_ORCH,
+                 D.FULLY | D.FORCE_PROFILE):
         y = vec(y0)
         ctx.spmtv(plan, vec(x), y, f=0.05, mode=mode)
         torch.cuda.synchronize()
@@ -107,15 +114,18 @@ def test_spmtv_small_integer_bit_exact(ctx, D):
 
 
 def test_spmtv_swap_async_rejected_and_edges(ctx, D):
+    """Table 1 / P:L735-740: the copy-back swap (HOST_ORCH) cannot run
+    asynchronously; the additive device swap can (reading A-47b)."""
     import torch
     from paper_conf_asplos_changkh16_b200.dysel import DyselError
     A = MATS["ragged_nonsquare"]()
     plan, keep = _plan(ctx, A)
     x, y = vec(uniform_f32(51, A.n_rows)), vec(uniform_f32(52, A.n_cols))
     with pytest.raises(DyselError):
-        ctx.spmtv(plan, x, y, f=0.05, mode=D.SWAP | D.ASYNC)
+        ctx.spmtv(plan, x, y, f=0.05, mode=D.SWAP | D.ASYNC | D.HOST_ORCH)
     with pytest.raises(DyselError):
-        ctx.spmtv(plan, x, y, f=0.05, mode=D.AUTO | D.ASYNC)   # AUTO -> swap, still no async (Table 1)
+        ctx.spmtv(plan, x, y, f=0.05, mode=D.AUTO | D.ASYNC | D.HOST_ORCH)   # AUTO -> swap, no async (Table 1)
+    ctx.spmtv(plan, x, y, f=0.05, mode=D.SWAP | D.ASYNC)   # additive swap: the final output is y (A-47b)
     with pytest.raises(DyselError):
         ctx.spmtv_variant(plan, 7, x, y)
     plan.destroy()
@@ -140,11 +150,14 @@ def test_spmtv_bench_size_parity(ctx, D):
     x = uniform_f32(61, A.n_rows)
     y0 = uniform_f32(62, A.n_cols)
     plan, keep = _plan(ctx, A)
-    for mode in (D.AUTO, D.AUTO | D.NO_PROFILE):
+    for mode in (D.AUTO, D.AUTO | D.ASYNC, D.AUTO | D.NO_PROFILE):
         y = vec(y0)
         rep = ctx.spmtv(plan, vec(x), y, f=0.01, mode=mode, report=True)
         torch.cuda.synchronize()
-        assert rep["profiled"] == (mode == D.AUTO)
+        assert rep["profiled"] == (mode != D.AUTO | D.NO_PROFILE)
+        if mode == D.AUTO | D.ASYNC:   # the idle SMs reduced light units before the selection (A-47b)
+            assert rep["eager_units"] > 0 and rep["mode_used"] & D.ASYNC
+            assert rep["eager_units"] + rep["tail_units"] + rep["c"] == rep["n_granules"]
         assert _err(A, x, y0, y) <= SPMV_TOL, mode
     plan.destroy()
 
@@ -160,7 +173,7 @@ def test_spmtv_swap_odd_columns_and_unaligned_y(ctx, D, offset):
     x = uniform_f32(71, A.n_rows)
     y0 = uniform_f32(72, A.n_cols)
     plan, keep = _plan(ctx, A)
-    for mode in (D.AUTO, D.SWAP | D.HOST_ORCH):
+    for mode in (D.AUTO, D.AUTO | D.ASYNC, D.SWAP | D.HOST_ORCH):
         buf = torch.empty(A.n_cols + 1, device="cuda")
         y = buf[offset:offset + A.n_cols]
         y.copy_(vec(y0))
