@@ -711,17 +711,20 @@ def secondary_workloads(ctx, D, args, stream, pk):
         # interleaved rounds (pure best, then each DySel form): long tensor-core
         # runs heat the GPU (sw power cap), so every ratio compares neighbours
         R = 3
-        rounds = {k: [] for k in ("pure", "dysel", "forced", "hybrid", "amort")}
+        rounds = {k: [] for k in ("pure", "dysel", "fully_async", "forced", "hybrid", "amort")}
         for _ in range(R):
             rounds["pure"].append(time_b2b(lambda: ctx.sgemm_variant(vbest, Ad, Bd, C), reps, stream))
             rounds["dysel"].append(time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY), reps, stream))
+            rounds["fully_async"].append(time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.ASYNC), reps,
+                                                  stream))
             rounds["forced"].append(time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE),
                                              reps, stream))
             rounds["hybrid"].append(time_b2b(lambda: ctx.sgemm(Ad, Bd, C, f=f_sg,
                                                                mode=D.HYBRID | D.ASYNC | D.FORCE_PROFILE), reps, stream))
             rounds["amort"].append(time_b2b(amort, 2, stream) / I)
         tp = float(np.median(rounds["pure"]))
-        tdg, tforced, th, tam = (float(np.median(rounds[k])) for k in ("dysel", "forced", "hybrid", "amort"))
+        tdg, tfa, tforced, th, tam = (float(np.median(rounds[k]))
+                                      for k in ("dysel", "fully_async", "forced", "hybrid", "amort"))
         tv[bestg] = min(tv[bestg], tp)
         repg = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY, report=True)
         repf = ctx.sgemm(Ad, Bd, C, f=f_sg, mode=D.FULLY | D.FORCE_PROFILE, report=True)
@@ -739,6 +742,7 @@ def secondary_workloads(ctx, D, args, stream, pk):
                                                 "(profiles/sgemm_pipeline_r2.txt)"},
                      "dysel_us": round(tdg * 1e6, 2), "profiled": repg["profiled"], "selected": repg["selected_name"],
                      "overhead_pct": round((tdg / tp - 1) * 100, 2),
+                     "fully_async_overhead_pct": round((tfa / tp - 1) * 100, 2),
                      "forced_single_shot_overhead_pct": round((tforced / tp - 1) * 100, 2),
                      "forced_selected": repf["selected_name"],
                      "hybrid_async_overhead_pct": round((th / tp - 1) * 100, 2),
