@@ -508,7 +508,11 @@ dysel_status dysel_stencil_variant(dysel_ctx *ctx, int variant_id, int nx, int n
  * (DESIGN A-47): private outputs start at zero, the winner's is ADDED into y,
  * so the final output space is y itself and ASYNC is accepted (A-47b): the
  * default's kernel reduces light units straight into y until the selection
- * (report.eager_units).  Unit = 256 rows of A.
+ * (report.eager_units).  Initial version (DESIGN A-30d): scatter-thread when
+ * no row exceeds 64 entries, scatter-warp otherwise; below 128 MiB of
+ * algorithmic bytes, one wave of the initial version, or with NO_PROFILE, the
+ * call runs the cached selection or the initial version unprofiled (A-3b /
+ * A-3c; FORCE_PROFILE overrides).  Unit = 256 rows of A.
  * Variants: 0 scatter-thread (thread per row), 1 scatter-warp (warp per row,
  * entries strided over lanes), 2 scatter-segment (warp per 32-row segment,
  * its nonzeros as one flat stream).  One fp32 red.global.add per nonzero, in no

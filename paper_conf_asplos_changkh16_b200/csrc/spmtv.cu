@@ -537,10 +537,9 @@ static cudaError_t swap_launch(const void *fn, unsigned grid, unsigned block, cu
 
 static dysel_status spmtv_swap_device(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, float *d_y,
                                       const Plan &P, uint32_t mode, cudaStream_t st, dysel_report *rep,
-                                      const std::string &key) {
+                                      const std::string &key, int def) {
   const uint64_t t_host0 = now_ns();
   const int K = DYSEL_SPMTV_NVARIANTS;
-  const int def = DYSEL_SPMTV_SCATTER_WARP;
   if (!g_swap_occ[0]) {
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_swap_occ[0], spmtv_swap_rem_kernel<0>, 256, 0);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_swap_occ[1], spmtv_swap_rem_kernel<1>, 256, 0);
@@ -632,6 +631,23 @@ static dysel_status spmtv_swap_device(dysel_ctx *ctx, dysel_spmv_plan *pl, const
   return DYSEL_OK;
 }
 
+// Reading A-30d: the initial version of the SpMTV pool.  A thread per row
+// issues one reduction per nonzero with no idle lanes and won every matrix
+// whose longest row is short (rows of 1-48 entries, uniform or not, FEM 5x5:
+// scripts/diag_spmtv_short.py, profiles/spmtv_shapes_r2.txt); a long row
+// serialises it (2M-row power law, rows up to 4,096: 672 us vs scatter-warp's
+// 241), so scatter-warp starts whenever some row exceeds kSpmtvThreadMaxRow.
+constexpr int kSpmtvThreadMaxRow = 64;
+static int spmtv_default(const dysel_spmv_plan *pl) {
+  return pl->info.max_row_len <= kSpmtvThreadMaxRow ? DYSEL_SPMTV_SCATTER_THREAD : DYSEL_SPMTV_SCATTER_WARP;
+}
+// Reading A-3c for the SpMTV pool: a call shorter than ~2x the profiling
+// latency (~25-35 us to the publish here) cannot pay for a single-shot
+// profile.  dysel_spmv draws that line at 64 MiB; the scatter-add pool moves
+// its bytes at about half SpMV's rate (1.5-3.3 TB/s measured: the L2
+// reductions), so the same ~50 us sits at 128 MiB.
+constexpr uint64_t kSpmtvMinProfBytes = 128ull << 20;
+
 static dysel_status spmtv_check(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *x, float *y) {
   if (!pl || pl->ctx != ctx || (pl->dev.n_rows > 0 && !x) || (pl->dev.n_cols > 0 && !y)) {
     set_error(ctx, "dysel_spmtv: invalid arguments");
@@ -668,14 +684,46 @@ dysel_status dysel_spmtv(dysel_ctx *ctx, dysel_spmv_plan *pl, const float *d_x, 
     // reading A-47b: the additive swap fixes the final output space (y itself), so
     // ASYNC is accepted here; the paper's copy-back swap (HOST_ORCH, the generic
     // launcher) still rejects it (Table 1)
+    const int def = spmtv_default(pl);
     Plan P;
-    DYSEL_TRY(make_plan(ctx, U, wa, DYSEL_SPMTV_NVARIANTS, f, ctx->n_sm, DYSEL_SPMTV_SCATTER_WARP,
-                        mode & ~(uint32_t)DYSEL_ASYNC, vflags, &P));
+    DYSEL_TRY(make_plan(ctx, U, wa, DYSEL_SPMTV_NVARIANTS, f, ctx->n_sm, def, mode & ~(uint32_t)DYSEL_ASYNC, vflags,
+                        &P));
     if (P.mode == DYSEL_SWAP) {
-      // reading A-3b: a grid within one wave of the default is not profiled (the generic path runs it)
-      const bool one_wave = !(mode & DYSEL_FORCE_PROFILE) && P.Gn <= g_spmtv_wave[DYSEL_SPMTV_SCATTER_WARP];
-      if (P.active && !one_wave) return spmtv_swap_device(ctx, pl, d_x, d_y, P, mode, (cudaStream_t)stream, rep, key);
-      mode &= ~(uint32_t)DYSEL_ASYNC;   // unprofiled: no eager phase to run
+      const bool forced = (mode & DYSEL_FORCE_PROFILE) != 0;
+      const bool one_wave = !forced && P.Gn <= g_spmtv_wave[def];   // reading A-3b
+      const uint64_t bytes = 8ull * (uint64_t)pl->info.nnz + 8ull * (uint64_t)pl->dev.n_rows + 4ull +
+                             8ull * (uint64_t)pl->dev.n_cols;
+      const bool small = !forced && bytes < kSpmtvMinProfBytes;    // reading A-3c
+      if (P.active && !one_wave && !small)
+        return spmtv_swap_device(ctx, pl, d_x, d_y, P, mode, (cudaStream_t)stream, rep, key, def);
+      // unprofiled (activation flag off, A-3b, A-3c): the cached selection, else the initial version (A-30d)
+      resolve_pending(ctx, key.c_str());
+      int v = def;
+      auto c = ctx->sel_cache.find(key);
+      if (c != ctx->sel_cache.end() && c->second >= 0 && c->second < DYSEL_SPMTV_NVARIANTS) v = c->second;
+      if (rep) {
+        const uint64_t t0 = now_ns();
+        memset(rep->score, 0, sizeof(rep->score));
+        memset(rep->makespan_ns, 0, sizeof(rep->makespan_ns));
+        memset(rep->units, 0, sizeof(rep->units));
+        memset(rep->cycles, 0, sizeof(rep->cycles));
+        memset(rep->busy_ns, 0, sizeof(rep->busy_ns));
+        memset(rep->aborted, 0, sizeof(rep->aborted));
+        rep->mode_used = DYSEL_SWAP;
+        rep->profiled = 0;
+        rep->selected = v;
+        rep->n_variants = DYSEL_SPMTV_NVARIANTS;
+        rep->c = 0;
+        rep->n_granules = P.Gn;
+        rep->eager_units = rep->tail_units = 0;
+        rep->sandbox_buffers = 0;
+        rep->sandbox_bytes = 0;
+        for (int i = 0; i < 8; ++i) rep->timeline_ns[i] = ~0ull;
+        if (rep->unit_variant)
+          for (uint64_t j = 0; j < rep->unit_variant_cap && j < P.Gn; ++j) rep->unit_variant[j] = (uint8_t)v;
+        rep->host_ns = now_ns() - t0;
+      }
+      return dysel_spmtv_variant(ctx, pl, v, d_x, d_y, stream);
     }
   }
   return launch_keyed(ctx, kSpmtvSig, key.c_str(), U, f, mode, args, 2, sbytes, stream, rep);

@@ -90,8 +90,8 @@ def test_spmtv_modes_parity(ctx, D, name, m):
                 assert rep["eager_units"] == 0
     if m in ("auto_forced", "auto_async_forced"):
         assert rep["profiled"]
-    if name == "powerlaw" and m == "auto":
-        assert rep["profiled"]
+    if name == "powerlaw" and m in ("auto", "auto_async"):
+        assert not rep["profiled"]   # 101 MiB: under the SpMTV pool's A-3c line (128 MiB)
     plan.destroy()
 
 
@@ -173,7 +173,7 @@ def test_spmtv_swap_odd_columns_and_unaligned_y(ctx, D, offset):
     x = uniform_f32(71, A.n_rows)
     y0 = uniform_f32(72, A.n_cols)
     plan, keep = _plan(ctx, A)
-    for mode in (D.AUTO, D.AUTO | D.ASYNC, D.SWAP | D.HOST_ORCH):
+    for mode in (D.AUTO | D.FORCE_PROFILE, D.AUTO | D.ASYNC | D.FORCE_PROFILE, D.SWAP | D.HOST_ORCH):
         buf = torch.empty(A.n_cols + 1, device="cuda")
         y = buf[offset:offset + A.n_cols]
         y.copy_(vec(y0))
@@ -183,3 +183,62 @@ def test_spmtv_swap_odd_columns_and_unaligned_y(ctx, D, offset):
         assert rep["sandbox_buffers"] == len(D.SPMTV_NAMES)              # Table 1: K private outputs
         assert _err(A, x, y0, y) <= SPMV_TOL, (mode, offset)
     plan.destroy()
+
+
+def test_spmtv_async_non_default_winner(ctx, D):
+    """A-47b with a winner other than the initial version: rows of 0-8 entries
+    plus one 100-entry row in 1,000 -- the longest row exceeds A-30d's 64, so
+    scatter-warp starts, but a warp per row idles most lanes and scatter-thread
+    wins: the switch kernel launches the winner's remainder while the
+    default's eager CTAs drain.  Eager light units (default), the winner's
+    add-in, heavy and remaining light units must each land in y once."""
+    import torch
+    from workloads import csr_from_lengths, rng
+    n = 3_000_000   # 146 MiB: profiled without FORCE_PROFILE (A-3c line: 128 MiB)
+    L = rng(91).integers(0, 9, n)
+    L[::1000] = 100
+    A = csr_from_lengths(L, n, 92, 93)
+    x = uniform_f32(82, A.n_rows)
+    y0 = uniform_f32(83, A.n_cols)
+    plan, keep = _plan(ctx, A)
+    assert plan.info.max_row_len == 100
+    sels = []
+    for mode in (D.AUTO | D.ASYNC, D.AUTO | D.ASYNC | D.FORCE_PROFILE, D.AUTO):
+        for _ in range(3):
+            y = vec(y0)
+            rep = ctx.spmtv(plan, vec(x), y, f=0.02, mode=mode, report=True)
+            torch.cuda.synchronize()
+            assert rep["profiled"], mode
+            assert _err(A, x, y0, y) <= SPMV_TOL, (mode, rep["selected_name"])
+            assert rep["eager_units"] + rep["tail_units"] + rep["c"] == rep["n_granules"]
+            sels.append(rep["selected_name"])
+    print("selections", sels)
+    assert any(s != "scatter_warp" for s in sels)   # the switch path ran
+    plan.destroy()
+
+
+def test_spmtv_initial_version_a30d_and_small_a3c(ctx, D):
+    """Reading A-30d: scatter-thread starts when no row exceeds 64 entries,
+    scatter-warp otherwise; reading A-3c: under 128 MiB the call runs the
+    initial version unprofiled (FORCE_PROFILE overrides).  Parity either way."""
+    import torch
+    cases = [(random_lengths_csr(1_500_000, 1_200_000, 2, 81), "scatter_thread", False),
+             (d4_powerlaw(n=1_000_000, lmax=2000), "scatter_warp", True)]
+    for A, want_def, big in cases:
+        plan, keep = _plan(ctx, A)
+        x = uniform_f32(94, A.n_rows)
+        y0 = uniform_f32(95, A.n_cols)
+        y = vec(y0)
+        rep = ctx.spmtv(plan, vec(x), y, f=0.02, mode=D.AUTO | D.ASYNC, report=True)
+        torch.cuda.synchronize()
+        assert _err(A, x, y0, y) <= SPMV_TOL
+        assert rep["profiled"] == big
+        if not big:
+            assert rep["selected_name"] == want_def and rep["mode_used"] & 3 == D.SWAP
+            y = vec(y0)
+            rep = ctx.spmtv(plan, vec(x), y, f=0.02, mode=D.AUTO | D.FORCE_PROFILE, report=True)
+            torch.cuda.synchronize()
+            assert rep["profiled"] and _err(A, x, y0, y) <= SPMV_TOL
+        else:   # the initial version is the eager one: heavy-tailed rows -> scatter-warp
+            assert rep["eager_units"] > 0
+        plan.destroy()
