@@ -222,6 +222,12 @@ def test_spmtv_async_non_default_winner(ctx, D):
             sels.append(rep["selected_name"])
     print("selections", sels)
     assert any(s != "scatter_warp" for s in sels)   # the switch path ran
+    # activation flag off: the cached selection of the last profiled call runs
+    y = vec(y0)
+    rep = ctx.spmtv(plan, vec(x), y, mode=D.AUTO | D.NO_PROFILE, report=True)
+    torch.cuda.synchronize()
+    assert not rep["profiled"] and rep["selected_name"] == sels[-1]
+    assert _err(A, x, y0, y) <= SPMV_TOL
     plan.destroy()
 
 
