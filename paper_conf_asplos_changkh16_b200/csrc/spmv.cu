@@ -34,12 +34,16 @@ namespace dysel {
 // the remainder.  DYSEL_SCORE_CYCLES: sum clock64 / units.
 // DYSEL_SCORE_MAKESPAN: the paper's earliest start .. latest end (Fig. 7b).
 struct SpmvState {
-  uint32_t c2;              // winner's remainder slot tickets (relative, after its static first slots)
+  // Hot words, each on its own 128-byte line: thousands of waiting warps poll
+  // `sw` and the eager claims hammer `c1`; sharing a line (an L2 slice) with
+  // the profiling completion chain's atomics queued those atomics behind the
+  // traffic and delayed the publish by several us.
+  alignas(128) uint64_t c1; // eager slot tickets (low 32 bits) | published (bit 32)
+  alignas(128) uint64_t sw; // (S << 8) | selected pool index, ~0 until published
+  alignas(128) uint32_t c2; // winner's remainder slot tickets (relative, after its static first slots)
+  alignas(128) uint64_t pure_ctr;   // pure full-grid runs: slot tickets; the last warp of a run resets both
   uint32_t pure_done;       // pure full-grid runs: warps finished
-  uint64_t c1;              // eager slot tickets (low 32 bits) | published (bit 32)
-  uint64_t sw;              // (S << 8) | selected pool index, ~0 until published
-  uint64_t pure_ctr;        // pure full-grid runs: slot tickets; the last warp of a run resets both
-  uint32_t variants_done;
+  alignas(128) uint32_t variants_done;
   uint32_t pad;
   uint64_t best;            // (score << 8) | pool variant
   uint64_t sel;             // final packed selection, ~0 until published
