@@ -158,11 +158,18 @@ struct PubArgs {
 };
 constexpr uint32_t kSlots = kUnitRows / 32;   // 32-row warp slots per unit
 
+// acq_rel counter increment: releases this thread's earlier writes / reds
+// (stats, scores) and, for the thread that sees the final count, acquires
+// everyone else's -- one round trip where fence + atomic + fence took three
+__device__ __forceinline__ uint32_t atom_add_acq_rel(uint32_t *q, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(q), "r"(v) : "memory");
+  return old;
+}
+
 __device__ __forceinline__ void decided_publish(const PubArgs a) {
-  __threadfence();
-  const uint32_t vd = atomicAdd(&a.st->variants_done, 1u) + 1u;
+  const uint32_t vd = atom_add_acq_rel(&a.st->variants_done, 1u) + 1u;
   if (vd != a.K) return;
-  __threadfence();
   unsigned long long fin = atomicAdd((unsigned long long *)&a.st->best, 0ull);
   // reading A-50 (switch margin): a challenger within 1/8 of the initial
   // version's own completed score does not replace it — switching costs the
@@ -434,12 +441,10 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
       __threadfence();
       atomicAdd(&p.chunk_done[j >> p.chunk_shift], (uint32_t)kSlots);
     }
-    __threadfence();
-    const uint32_t done = atomicAdd(&st->ctas_done[pv], 1u) + 1u;
+    const uint32_t done = atom_add_acq_rel(&st->ctas_done[pv], 1u) + 1u;
     // ---- variant complete (and not already decided by dominance): score,
     // packed atomicMin (A-7, A-8); the last variant decided publishes
-    if (done == p.c && atomicCAS(&st->decided[pv], 0u, 1u) == 0u) {
-      __threadfence();
+    if (done == p.c && atomicCAS(&st->decided[pv], 0u, 1u) == 0u) {   // (acquired by the add above)
       const unsigned long long a = atomicAdd((unsigned long long *)&slot->t_start_min, 0ull);
       const unsigned long long e = atomicAdd((unsigned long long *)&slot->t_end_max, 0ull);
       const unsigned long long cy = atomicAdd((unsigned long long *)&slot->cycles, 0ull);
@@ -451,8 +456,7 @@ __device__ __forceinline__ void prof_unit(const SpmvDev &A, float *__restrict__ 
       unsigned long long score = p.score_mode == 1 ? cy / p.c : p.score_mode == 2 ? e - a : pred;
       if (score > cap) score = cap;
       atomicMin((unsigned long long *)&st->best_total, p.score_mode == 2 ? e - a : pred);   // dominance units
-      st->vscore[pv] = (score << 8) | pv;
-      __threadfence();
+      st->vscore[pv] = (score << 8) | pv;   // released by decided_publish's acq_rel add
       atomicMin((unsigned long long *)&st->best, (score << 8) | pv);
       decided_publish(pub);
     }
