@@ -209,12 +209,14 @@ __device__ __forceinline__ uint32_t swap_smid() {
 }   // floats of the winner's private output per add-in ticket
 
 struct SwapState {
-  uint32_t rem_ctr;      // tickets: add-in chunks, then heavy units
-  uint32_t light_ctr;    // the other light units (eager phase and remainder share it, A-47b)
-  uint32_t eager_units;  // light units done before the selection (ASYNC, A-47b)
-  uint32_t variants_done;
+  // claim counters and the polled selection word each on its own 128-byte
+  // line, away from the profiling completion chain's atomics (as SpmvState)
+  alignas(128) uint32_t rem_ctr;      // tickets: add-in chunks, then heavy units
+  alignas(128) uint32_t light_ctr;    // the other light units (eager phase and remainder share it, A-47b)
+  alignas(128) uint32_t eager_units;  // light units done before the selection (ASYNC, A-47b)
+  alignas(128) uint64_t sel;
+  alignas(128) uint32_t variants_done;
   uint64_t best;
-  uint64_t sel;
   uint64_t best_total;
   uint32_t ctas_done[DYSEL_SPMTV_NVARIANTS];
   uint32_t decided[DYSEL_SPMTV_NVARIANTS];   // 0 running, 1 completed, 2 dominated
